@@ -1,0 +1,283 @@
+"""Seeded synthetic graph generators shared by the oracle side and the CUDA side.
+
+This module holds NONE of the method's arithmetic (no BFS, no path counting, no
+dependency accumulation).  It only produces inputs: edge lists and their CSC form
+(the input format of PAPER.md P:95-97: column v lists the rows u with A(u,v) = 1,
+i.e. the edges u -> v), plus seeded source lists.
+
+Workload recipes (restated in DESIGN.md "Inputs"):
+  cfg1  Erdos-Renyi G(n=1024, M=4096) undirected, seed 1, all sources
+  cfg2  RMAT/Kronecker scale 18, edgefactor 16, undirected, seed 2, 1024 sources
+  cfg3  Graph500 Kronecker scale 22, edgefactor 16, DIRECTED, seed 3, 4096 sources
+  cfg4  road-like 4096x4096 lattice: MST under iid U(0,1) weights + 10% of the other
+        lattice edges, undirected, seed 4, 1024 sources
+  cfg5  Graph500 Kronecker scale 25, edgefactor 16, undirected, seed 5, 8192 sources
+Kronecker: A,B,C,D = 0.57,0.19,0.19,0.05 (Graph500), seeded label permutation,
+self-loops and duplicates removed, undirected = symmetrised.
+Sources: the first k of a seeded permutation of the vertices with out-degree >= 1.
+
+Kronecker/ER generation runs in torch on whatever device is given (CUDA for the big
+configs; the RNG stream then differs from CPU, so m is recorded per generated graph).
+"""
+from __future__ import annotations
+
+import dataclasses
+import math
+
+import numpy as np
+
+try:  # torch is only needed for the large generators
+    import torch
+except Exception:  # pragma: no cover
+    torch = None
+
+
+@dataclasses.dataclass
+class Graph:
+    """A generated graph in CSC form (0-based, int64 col_ptr, int32 row_idx, sorted, deduplicated)."""
+    name: str
+    n: int
+    col_ptr: np.ndarray
+    row_idx: np.ndarray
+    directed: bool
+
+    @property
+    def nnz(self) -> int:
+        return int(self.col_ptr[-1])
+
+    def out_degree(self) -> np.ndarray:
+        return np.bincount(self.row_idx, minlength=self.n).astype(np.int64)
+
+    def in_degree(self) -> np.ndarray:
+        return np.diff(self.col_ptr)
+
+    def edges(self):
+        """(src, dst) int32 arrays of the stored edges src -> dst."""
+        dst = np.repeat(np.arange(self.n, dtype=np.int32), np.diff(self.col_ptr))
+        return self.row_idx.copy(), dst
+
+
+# ----------------------------------------------------------------------------- CSC build
+
+def csc_from_edges(n: int, src, dst, directed: bool):
+    """Edge list src->dst -> canonical CSC (sorted, dedup, self-loops removed; symmetrised if undirected)."""
+    src = np.asarray(src, dtype=np.int64)
+    dst = np.asarray(dst, dtype=np.int64)
+    keep = src != dst
+    src, dst = src[keep], dst[keep]
+    if not directed:
+        src, dst = np.concatenate([src, dst]), np.concatenate([dst, src])
+    key = np.unique(dst * n + src)           # column-major order: by dst, then src
+    col = key // n
+    row = (key - col * n).astype(np.int32)
+    col_ptr = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(np.bincount(col, minlength=n), out=col_ptr[1:])
+    return col_ptr, row
+
+
+def csc_from_edges_torch(n: int, src, dst, directed: bool):
+    """Same as :func:`csc_from_edges` but sorts on the tensors' device (for ~1e9-edge graphs)."""
+    src = src.to(torch.int64)
+    dst = dst.to(torch.int64)
+    keep = src != dst
+    src, dst = src[keep], dst[keep]
+    if not directed:
+        src, dst = torch.cat([src, dst]), torch.cat([dst, src])
+    key = dst * n + src
+    del src, dst
+    key = torch.unique(key, sorted=True)
+    col = key // n
+    row = (key - col * n).to(torch.int32)
+    counts = torch.bincount(col, minlength=n)
+    del col, key
+    col_ptr = torch.zeros(n + 1, dtype=torch.int64, device=row.device)
+    col_ptr[1:] = torch.cumsum(counts, 0)
+    return col_ptr.cpu().numpy(), row.cpu().numpy()
+
+
+# ----------------------------------------------------------------------------- generators
+
+def erdos_renyi(n: int, m_edges: int, seed: int, directed: bool = False) -> Graph:
+    """G(n, M): M distinct uniformly random (unordered if undirected) pairs, no self-loops."""
+    rng = np.random.default_rng(seed)
+    chosen = set()
+    pairs = []
+    while len(pairs) < m_edges:
+        u, v = (int(x) for x in rng.integers(0, n, size=2))
+        if u == v:
+            continue
+        key = (u, v) if directed else (min(u, v), max(u, v))
+        if key in chosen:
+            continue
+        chosen.add(key)
+        pairs.append(key)
+    p = np.asarray(pairs, dtype=np.int64).reshape(-1, 2)
+    cp, ri = csc_from_edges(n, p[:, 0], p[:, 1], directed)
+    return Graph(f"er_n{n}_M{m_edges}_s{seed}", n, cp, ri, directed)
+
+
+def kronecker(scale: int, edgefactor: int, seed: int, directed: bool, device: str = "cpu",
+              abc=(0.57, 0.19, 0.19)) -> Graph:
+    """Graph500 Kronecker/RMAT generator: edgefactor * 2^scale tuples, each bit of (src,dst)
+    drawn from the 2x2 initiator (A,B;C,D), then a seeded vertex-label permutation."""
+    if torch is None:
+        raise RuntimeError("torch required for kronecker()")
+    n = 1 << scale
+    m_t = edgefactor * n
+    a, b, c = abc
+    g = torch.Generator(device=device)
+    g.manual_seed(seed)
+    src = torch.zeros(m_t, dtype=torch.int64, device=device)
+    dst = torch.zeros(m_t, dtype=torch.int64, device=device)
+    ab = a + b
+    c_norm = c / (1.0 - ab)
+    a_norm = a / ab
+    chunk = 1 << 26
+    for lo in range(0, m_t, chunk):
+        hi = min(m_t, lo + chunk)
+        s = src[lo:hi]
+        d = dst[lo:hi]
+        for bit in range(scale):
+            r1 = torch.rand(hi - lo, generator=g, device=device)
+            r2 = torch.rand(hi - lo, generator=g, device=device)
+            ii = r1 > ab
+            jj = r2 > torch.where(ii, torch.full_like(r2, c_norm), torch.full_like(r2, a_norm))
+            s |= ii.to(torch.int64) << bit
+            d |= jj.to(torch.int64) << bit
+    perm = torch.randperm(n, generator=g, device=device)
+    src = perm[src]
+    dst = perm[dst]
+    if device == "cpu":
+        cp, ri = csc_from_edges(n, src.numpy(), dst.numpy(), directed)
+    else:
+        cp, ri = csc_from_edges_torch(n, src, dst, directed)
+    kind = "dir" if directed else "undir"
+    return Graph(f"kron_s{scale}_ef{edgefactor}_{kind}_seed{seed}", n, cp, ri, directed)
+
+
+def road_lattice(side: int, q: float, seed: int) -> Graph:
+    """Road-like lattice: the minimum spanning tree of the side x side 4-neighbour grid under iid
+    U(0,1) edge weights, plus each remaining grid edge independently with probability q."""
+    from scipy.sparse import coo_matrix
+    from scipy.sparse.csgraph import minimum_spanning_tree
+    rng = np.random.default_rng(seed)
+    n = side * side
+    idx = np.arange(n, dtype=np.int64).reshape(side, side)
+    h_u, h_v = idx[:, :-1].ravel(), idx[:, 1:].ravel()
+    v_u, v_v = idx[:-1, :].ravel(), idx[1:, :].ravel()
+    eu = np.concatenate([h_u, v_u])
+    ev = np.concatenate([h_v, v_v])
+    w = rng.random(eu.size) + 1e-12  # strictly positive so scipy keeps every edge
+    mst = minimum_spanning_tree(coo_matrix((w, (eu, ev)), shape=(n, n)).tocsr()).tocoo()
+    in_tree = np.zeros(eu.size, dtype=bool)
+    # identify tree edges by key
+    tkey = np.minimum(mst.row, mst.col).astype(np.int64) * n + np.maximum(mst.row, mst.col)
+    ekey = np.minimum(eu, ev) * n + np.maximum(eu, ev)
+    in_tree[np.isin(ekey, tkey)] = True
+    extra = (~in_tree) & (rng.random(eu.size) < q)
+    keep = in_tree | extra
+    cp, ri = csc_from_edges(n, eu[keep], ev[keep], directed=False)
+    return Graph(f"road_{side}x{side}_q{q}_s{seed}", n, cp, ri, False)
+
+
+def grid(a: int, b: int) -> Graph:
+    """P_a x P_b grid graph (undirected); vertex (i, j) has id i*b + j."""
+    idx = np.arange(a * b).reshape(a, b)
+    eu = np.concatenate([idx[:, :-1].ravel(), idx[:-1, :].ravel()])
+    ev = np.concatenate([idx[:, 1:].ravel(), idx[1:, :].ravel()])
+    cp, ri = csc_from_edges(a * b, eu, ev, directed=False)
+    return Graph(f"grid_{a}x{b}", a * b, cp, ri, False)
+
+
+def from_edges(name: str, n: int, edges, directed: bool) -> Graph:
+    e = np.asarray(list(edges), dtype=np.int64).reshape(-1, 2)
+    cp, ri = csc_from_edges(n, e[:, 0], e[:, 1], directed)
+    return Graph(name, n, cp, ri, directed)
+
+
+def star(n: int, directed_both: bool = False) -> Graph:
+    """K_{1,n-1} with centre 0. directed_both: the same symmetric pattern flagged directed."""
+    e = [(0, i) for i in range(1, n)]
+    g = from_edges(f"star{n}", n, e, directed=False)
+    g.directed = directed_both
+    return g
+
+
+def path(n: int, directed: bool = False) -> Graph:
+    return from_edges(f"path{n}", n, [(i, i + 1) for i in range(n - 1)], directed)
+
+
+def cycle(n: int) -> Graph:
+    return from_edges(f"cycle{n}", n, [(i, (i + 1) % n) for i in range(n)], False)
+
+
+def complete(n: int) -> Graph:
+    return from_edges(f"K{n}", n, [(i, j) for i in range(n) for j in range(i + 1, n)], False)
+
+
+def complete_bipartite(a: int, b: int) -> Graph:
+    return from_edges(f"K{a},{b}", a + b, [(i, a + j) for i in range(a) for j in range(b)], False)
+
+
+def random_tree(n: int, seed: int) -> Graph:
+    rng = np.random.default_rng(seed)
+    e = [(int(rng.integers(0, i)), i) for i in range(1, n)]
+    return from_edges(f"tree{n}_s{seed}", n, e, False)
+
+
+def mycielski(k: int) -> Graph:
+    """Mycielski graph M_k (networkx convention: M_1 = K_1, M_2 = K_2); the paper's
+    'mycielski15..19' (Table 3) are M_15..M_19 of SuiteSparse."""
+    if k == 1:
+        return from_edges("mycielski1", 1, [], False)
+    eu = np.array([0], dtype=np.int64)
+    ev = np.array([1], dtype=np.int64)
+    n = 2
+    for _ in range(k - 2):
+        # Mycielskian: copies u_i = i + n adjacent to N(v_i), hub w = 2n adjacent to all u_i
+        ui = np.arange(n, 2 * n, dtype=np.int64)
+        eu, ev = (np.concatenate([eu, eu, eu + n, ui]),
+                  np.concatenate([ev, ev + n, ev, np.full(n, 2 * n, dtype=np.int64)]))
+        n = 2 * n + 1
+    cp, ri = csc_from_edges(n, eu, ev, directed=False)
+    return Graph(f"mycielski{k}", n, cp, ri, False)
+
+
+# ----------------------------------------------------------------------------- sources
+
+def sources(g: Graph, k: int, seed: int) -> np.ndarray:
+    """First k of a seeded permutation of the vertices with out-degree >= 1."""
+    cand = np.nonzero(g.out_degree() > 0)[0].astype(np.int32)
+    rng = np.random.default_rng(seed)
+    perm = rng.permutation(cand.size)
+    if k > cand.size:
+        reps = math.ceil(k / max(cand.size, 1))
+        perm = np.concatenate([rng.permutation(cand.size) for _ in range(reps)])
+    return cand[perm[:k]].astype(np.int32)
+
+
+# ----------------------------------------------------------------------------- configs
+
+CONFIGS = {
+    1: dict(name="cfg1_er1024", kind="er", n=1024, M=4096, seed=1, directed=False, k=1024, src_seed=None),
+    2: dict(name="cfg2_rmat18_undir", kind="kron", scale=18, ef=16, seed=2, directed=False, k=1024, src_seed=12),
+    3: dict(name="cfg3_kron22_dir", kind="kron", scale=22, ef=16, seed=3, directed=True, k=4096, src_seed=13),
+    4: dict(name="cfg4_road4096", kind="road", side=4096, q=0.10, seed=4, directed=False, k=1024, src_seed=14),
+    5: dict(name="cfg5_kron25_undir", kind="kron", scale=25, ef=16, seed=5, directed=False, k=8192, src_seed=15),
+}
+
+
+def make_config(cfg: int, device: str = "cpu", scale_override: int | None = None,
+                side_override: int | None = None):
+    """(Graph, sources) for config 1..5; overrides shrink the graph for fast tests."""
+    c = CONFIGS[cfg]
+    if c["kind"] == "er":
+        g = erdos_renyi(c["n"], c["M"], c["seed"], c["directed"])
+        src = np.arange(g.n, dtype=np.int32)            # exact BC: all sources (Alg.1 l.6)
+    elif c["kind"] == "kron":
+        g = kronecker(scale_override or c["scale"], c["ef"], c["seed"], c["directed"], device=device)
+        src = sources(g, c["k"], c["src_seed"])
+    else:
+        g = road_lattice(side_override or c["side"], c["q"], c["seed"])
+        src = sources(g, c["k"], c["src_seed"])
+    return g, src

@@ -1,0 +1,110 @@
+"""CPU oracle for the TurboBC hot path -- TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline`` /
+``--impl reference`` legs may import this package.  The product package
+(``paper_conf_icppw_artiless21_b200``) never imports it and shares no code with it.
+
+Contents
+  * ``brandes.c``  -- textbook Brandes (Eq. 2-4) in plain C / fp64,
+    exposed here as :func:`bc`, :func:`bfs`, :func:`delta`.
+  * ``brute.py``   -- exact brute force of Freeman's Eq. 1 with rationals
+    for graphs of <= 12 vertices (a second, independent oracle used to pin the first).
+
+Every function is pinned by ``tests/test_oracle.py`` (brute force, closed forms,
+invariants, networkx); there is no "parity unpinned" function in this package.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "brandes.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile ``brandes.c`` into ``liboracle.so`` with gcc (-O3, pthreads)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O3", "-march=native", "-std=c11", "-fPIC", "-shared",
+                               "-o", tmp, _SRC, "-lpthread"])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        lib = ctypes.CDLL(build())
+        i64, i32, dbl = ctypes.c_int64, ctypes.c_int32, ctypes.c_double
+        P = ctypes.POINTER
+        lib.oracle_bc.argtypes = [i64, P(i64), P(i32), ctypes.c_int, P(i32), i64, ctypes.c_int, P(dbl)]
+        lib.oracle_bc.restype = ctypes.c_int
+        lib.oracle_bfs.argtypes = [i64, P(i64), P(i32), i32, P(i32), P(dbl)]
+        lib.oracle_bfs.restype = ctypes.c_int
+        lib.oracle_delta.argtypes = [i64, P(i64), P(i32), i32, P(dbl)]
+        lib.oracle_delta.restype = ctypes.c_int
+        _lib = lib
+    return _lib
+
+
+def _ptr(a, ct):
+    return a.ctypes.data_as(ctypes.POINTER(ct))
+
+
+def _csc(col_ptr, row_idx):
+    cp = np.ascontiguousarray(col_ptr, dtype=np.int64)
+    ri = np.ascontiguousarray(row_idx, dtype=np.int32)
+    if ri.size == 0:
+        ri = np.zeros(1, dtype=np.int32)
+    return cp, ri
+
+
+def bc(col_ptr, row_idx, directed: bool, sources, nthreads: int | None = None) -> np.ndarray:
+    """bc(v) = sum over the source list of delta_s(v) (Eq. 3), halved if undirected."""
+    lib = _load()
+    cp, ri = _csc(col_ptr, row_idx)
+    n = cp.size - 1
+    src = np.ascontiguousarray(sources, dtype=np.int32)
+    k = src.size
+    if k == 0:
+        return np.zeros(n, dtype=np.float64)
+    out = np.zeros(n, dtype=np.float64)
+    nt = nthreads if nthreads else (os.cpu_count() or 1)
+    rc = lib.oracle_bc(n, _ptr(cp, ctypes.c_int64), _ptr(ri, ctypes.c_int32), int(bool(directed)),
+                       _ptr(src, ctypes.c_int32), k, int(nt), _ptr(out, ctypes.c_double))
+    if rc != 0:
+        raise ValueError("oracle_bc: invalid input")
+    return out
+
+
+def bfs(col_ptr, row_idx, source: int):
+    """(depth int32[n], sigma float64[n]) from one source: depth(s)=0, unreachable -1."""
+    lib = _load()
+    cp, ri = _csc(col_ptr, row_idx)
+    n = cp.size - 1
+    depth = np.empty(n, dtype=np.int32)
+    sigma = np.empty(n, dtype=np.float64)
+    rc = lib.oracle_bfs(n, _ptr(cp, ctypes.c_int64), _ptr(ri, ctypes.c_int32), int(source),
+                        _ptr(depth, ctypes.c_int32), _ptr(sigma, ctypes.c_double))
+    if rc != 0:
+        raise ValueError("oracle_bfs: invalid input")
+    return depth, sigma
+
+
+def delta(col_ptr, row_idx, source: int) -> np.ndarray:
+    """One-sided dependencies delta_s(v) (Eq. 2), unhalved; 0 at s and unreachable v."""
+    lib = _load()
+    cp, ri = _csc(col_ptr, row_idx)
+    n = cp.size - 1
+    out = np.empty(n, dtype=np.float64)
+    rc = lib.oracle_delta(n, _ptr(cp, ctypes.c_int64), _ptr(ri, ctypes.c_int32), int(source),
+                          _ptr(out, ctypes.c_double))
+    if rc != 0:
+        raise ValueError("oracle_delta: invalid input")
+    return out

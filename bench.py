@@ -1,0 +1,326 @@
+#!/usr/bin/env python
+"""bench.py -- TurboBC hot path on B200: GTEPS and sec/source, roofline, CPU-oracle baseline.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 3] [--impl ours|reference]
+    (N > 1: torchrun --nproc-per-node N ... bench.py --gpus N ...)
+
+A step = one full pass of the hot path (forward + backward for every source of the rank's
+source batch, then the one all-reduce of bc across ranks) -- PAPER.md Algorithm 1 over a
+source list.  Workload (BASELINE.json configs[2], the one the metric's 1/2/4/8-GPU figures
+are quoted on): Graph500 Kronecker scale 22, edgefactor 16, directed, CSC engine, 4096
+sources per GPU (weak scaling: rank r takes sources [r*4096, (r+1)*4096) of one seeded list).
+GTEPS = sources * m / t (paper convention: m = stored nnz, every source counted
+against all m).  The graph (523 MB of CSC+CSR) is larger than the 126 MB L2.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "BC GTEPS and sec/source at 1/2/4/8 B200; HBM GB/s fraction of peak"
+SOURCES_PER_GPU = {1: 1024, 2: 1024, 3: 4096, 4: 1024, 5: 1024}
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=3)
+    ap.add_argument("--sources", type=int, default=None, help="sources per GPU (default: the config's)")
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample", type=int, default=None, help="sources in the CPU-oracle sample")
+    ap.add_argument("--direction", type=int, default=0)
+    ap.add_argument("--alpha", type=float, default=1.0)
+    return ap.parse_args()
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled every 200 ms during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.idx = gpu_index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.idx}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm = [float(r[1]) for r in self.rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in self.rows:
+            if len(r) >= 9:
+                for nm, val in zip(names, r[5:9]):
+                    if val.strip().lower() == "active":
+                        reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def make_graph(cfg, device):
+    import graphgen as gg
+    t0 = time.time()
+    g, _ = gg.make_config(cfg, device=device)
+    return g, time.time() - t0
+
+
+def source_list(g, cfg, total):
+    import graphgen as gg
+    if cfg == 1:
+        return np.tile(np.arange(g.n, dtype=np.int32), (total + g.n - 1) // g.n)[:total]
+    return gg.sources(g, total, seed=gg.CONFIGS[cfg]["src_seed"])
+
+
+def cpu_baseline(g, sources, sample):
+    """The oracle as it stands on this host's cores, bounded sample of the same workload."""
+    import oracle
+    cores = os.cpu_count() or 1
+    k = sample or min(max(cores, 4), 64)
+    src = sources[:k]
+    _, secs = oracle.bc_timed(g.col_ptr, g.row_idx, g.directed, src, nthreads=min(cores, k))
+    return {"value": k * g.nnz / secs / 1e9, "unit": "GTEPS", "cores": min(cores, k), "kind": "oracle",
+            "sample": f"{k} sources of the same graph (first {k} of the rank-0 source list), "
+                      f"{secs:.2f} s of C Brandes oracle, one source per thread, graph build excluded",
+            "sec_per_source": secs / k}
+
+
+def run_reference(args):
+    """--impl reference: the oracle (this tier's reference arm) on the bench workload, rank 0 only."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    g, _ = make_graph(args.config, "cpu" if args.config in (1,) else _gen_device())
+    per_gpu = args.sources or SOURCES_PER_GPU[args.config]
+    srcs = source_list(g, args.config, per_gpu * args.gpus)
+    cores = os.cpu_count() or 1
+    k = args.cpu_sample or min(max(cores, 4), 64)
+    times = []
+    for i in range(args.warmup + args.steps):
+        sub = srcs[(i * k) % len(srcs):][:k]
+        _, secs = oracle.bc_timed(g.col_ptr, g.row_idx, g.directed, sub, nthreads=min(cores, k))
+        if i >= args.warmup:
+            times.append(secs / len(sub))
+    spp = statistics.mean(times)
+    val = g.nnz / spp / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "GTEPS", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": spp * k * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "sec_per_source": spp,
+            "config": {"workload": _workload_name(args.config), "n": g.n, "m": g.nnz,
+                       "sources_per_step": k},
+            "cpu_baseline": {"value": val, "unit": "GTEPS", "cores": min(cores, k), "kind": "oracle",
+                             "sample": f"{k} sources per step of the same workload"},
+            "e2e": {"value": val, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def _gen_device():
+    import torch
+    return "cuda" if torch.cuda.is_available() else "cpu"
+
+
+def _workload_name(cfg):
+    import graphgen as gg
+    return gg.CONFIGS[cfg]["name"]
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icppw_artiless21_b200 as tbc
+    from paper_conf_icppw_artiless21_b200 import dist as tdist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=dev)
+
+    g, gen_s = make_graph(args.config, "cuda")
+    per_gpu = args.sources or SOURCES_PER_GPU[args.config]
+    all_src = source_list(g, args.config, per_gpu * world)
+    lo, hi = rank * per_gpu, (rank + 1) * per_gpu
+    my_src = all_src[lo:hi]
+    t0 = time.time()
+    G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, device=local)
+    create_s = time.time() - t0
+    G.set_direction(args.direction)
+    G.set_alpha(args.alpha)
+    src_d = torch.from_numpy(my_src).to(dev)
+    bc = torch.zeros(g.n, dtype=torch.float64, device=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    def step():
+        bc.zero_()
+        G.bc_device(src_d, bc, stream)
+        if world > 1:
+            dist.all_reduce(bc, op=dist.ReduceOp.SUM)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    G.reset_stats()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for i in range(args.steps):
+            ev[i][0].record(stream)
+            bc.zero_()
+            kev[i][0].record(stream)
+            G.bc_device(src_d, bc, stream)
+            kev[i][1].record(stream)
+            if world > 1:
+                dist.all_reduce(bc, op=dist.ReduceOp.SUM)
+            ev[i][1].record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    kern_ms = [a.elapsed_time(b) for a, b in kev]
+    total_ms = sum(step_ms)
+    if world > 1:
+        t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    st = G.stats()
+    sources_total = per_gpu * world * args.steps
+    gteps = sources_total * g.nnz / (total_ms / 1e3) / 1e9
+    ms_per_step = total_ms / args.steps
+
+    # roofline of k_bc (the only kernel of the hot path): SURVEY 8(d) algorithmic bytes
+    # B_min = 8 B per out-edge of the reached set (4 B index read once per stage) + 80 B per
+    # reached vertex, summed over the launch's sources; / the kernel's event-timed duration.
+    alg_bytes_per_launch = (8.0 * st["reached_edges"] + 80.0 * st["reached"]) / args.steps
+    k_avg_s = statistics.mean(kern_ms) / 1e3
+    peak, peak_kind = peaks()
+    achieved = alg_bytes_per_launch / k_avg_s / 1e9
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", f"traffic_cfg{args.config}.json")
+    if os.path.exists(tpath):
+        try:
+            tj = json.load(open(tpath))
+            traffic = tj["dram_bytes_per_source"] * per_gpu
+        except Exception:
+            traffic = None
+
+    # end to end through the public host API: H2D sources, run, all-reduce, D2H bc
+    e2e_times = []
+    for i in range(max(2, min(args.steps, 3))):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t1 = time.perf_counter()
+        out = tdist.bc(G, all_src, None) if world > 1 else G.bc(my_src)
+        t2 = time.perf_counter()
+        e2e_times.append(t2 - t1)
+    e2e_s = statistics.median(e2e_times)
+    if world > 1:
+        t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_s = float(t.item())
+    e2e_gteps = per_gpu * world * g.nnz / e2e_s / 1e9
+
+    if rank == 0:
+        cpu = None
+        if not args.no_cpu_baseline and world == 1:
+            cpu = cpu_baseline(g, my_src, args.cpu_sample)
+        clocks = clk.summary()
+        line = {
+            "metric": METRIC, "value": gteps, "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "sec_per_source": total_ms / 1e3 / sources_total,
+            "config": {"workload": _workload_name(args.config), "n": g.n, "m": g.nnz,
+                       "directed": g.directed, "engine": "csc", "sources_per_gpu": per_gpu,
+                       "parallelism": f"source-partitioned x{world}, graph replicated, 1 NCCL all-reduce/step",
+                       "l2": "inputs larger than L2 (CSC+CSR %.0f MB vs 126 MB L2); no flush" %
+                             ((8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) / 1e6),
+                       "direction": args.direction, "alpha": args.alpha},
+            "clocks": clocks,
+            "gpu_launches": args.steps,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                         "kernel": "k_bc", "alg_bytes_per_launch": alg_bytes_per_launch,
+                         "kernel_ms": statistics.mean(kern_ms)},
+            "e2e": {"value": e2e_gteps, "unit": "GTEPS", "h2d_bytes_per_step": 4 * len(my_src),
+                    "d2h_bytes_per_step": 8 * g.n},
+            "cpu_baseline": cpu,
+            "traversal": {"reached_per_source": st["reached"] / max(st["sources"], 1),
+                          "reached_edges_per_source": st["reached_edges"] / max(st["sources"], 1),
+                          "fwd_edges_per_source": st["fwd_edges"] / max(st["sources"], 1),
+                          "bwd_edges_per_source": st["bwd_edges"] / max(st["sources"], 1),
+                          "levels_per_source": st["levels"] / max(st["sources"], 1),
+                          "pull_levels_per_source": st["pull_levels"] / max(st["sources"], 1),
+                          "traversed_gteps": (st["reached_edges"] / args.steps) * world * args.steps
+                          / (total_ms / 1e3) / 1e9},
+            "setup": {"generate_s": gen_s, "create_s": create_s, "device_bytes": G.device_bytes},
+        }
+        print(json.dumps(line), flush=True)
+    G.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

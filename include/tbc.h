@@ -1,0 +1,150 @@
+/*
+ * tbc.h -- C ABI of the B200-native TurboBC hot path (libturbobc.so).
+ *
+ * The method: Brandes betweenness centrality written as linear algebra, PAPER.md
+ * (Artiles & Saeed, "TurboBC", ICPP Workshops '21), cited as P:<line>:
+ *   Algorithm 1 BC-LA: per source s a forward BFS stage of masked SpMV
+ *   f_t = A^T f producing sigma (shortest-path counts) and S (depth)  (l.11-28), then a
+ *   backward stage over the levels in reverse with delta_u = (1+delta)/sigma, one SpMV
+ *   and delta += sigma * (SpMV result)  (l.29-42), then bc(v) += delta(v), v != s
+ *   (l.43-47), halved for undirected graphs.
+ *
+ * Conventions (all functions):
+ *   - vertex ids are int32_t, 0-based (the paper's CSC is 1-based); sizes int64_t.
+ *   - the graph is the boolean n x n adjacency matrix A: A(u,v) = 1 <=> edge u->v.
+ *     CSC column v lists the ROWS u with A(u,v)=1, i.e. the in-neighbours of v.
+ *     Duplicates collapse (A is boolean); self-loops are accepted and change nothing.
+ *   - depth(s) = 0, unreachable = -1 (the paper's S is max(depth,0), R3).
+ *   - sigma and bc are IEEE fp64.  sigma is exact while < 2^53.
+ *   - the backward SpMV uses A (out-neighbours); the printed A^T of Alg.1 l.37
+ *     is only right for undirected graphs (R1).
+ *   - no normalisation, no n/k extrapolation (Eq. 1-3); each occurrence of a
+ *     source in the list counts.
+ *
+ * Errors: every function returns a tbc_status; nothing crosses the ABI as an exception.
+ * On error the outputs are untouched (create: *out = NULL), nothing leaks, and
+ * tbc_last_error() holds a thread-local detail message.
+ *
+ * Threading: a tbc_graph is not re-entrant (it owns one workspace); distinct graphs may
+ * be used from distinct host threads.
+ */
+#ifndef TBC_H
+#define TBC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct tbc_graph tbc_graph; /* opaque; owns device memory on its device */
+
+typedef enum {
+    TBC_OK = 0,
+    TBC_ERR_INVALID = 1,     /* bad argument or malformed graph (see tbc_last_error) */
+    TBC_ERR_OOM = 2,         /* cudaMalloc failed */
+    TBC_ERR_CUDA = 3,        /* any other CUDA runtime error (message in tbc_last_error) */
+    TBC_ERR_UNSUPPORTED = 4  /* valid request this build does not implement */
+} tbc_status;
+
+/* engine: which SpMV formulation drives both stages */
+enum {
+    TBC_ENGINE_CSC = 0,  /* frontier-compacted push/pull over CSC (+CSR for directed graphs) */
+    TBC_ENGINE_COOT = 1  /* scCOOC: edge-parallel over the transposed-COO arrays every level
+                            (Alg. 2) */
+};
+
+/* create flags */
+enum {
+    TBC_FLAG_ONE_FORMAT = 1u << 0,  /* reserved (strict single-format directed mode, not yet built) */
+    TBC_FLAG_NO_VALIDATE = 1u << 1  /* skip host-side input validation (caller guarantees it) */
+};
+
+/* options for tbc_graph_set_option */
+enum {
+    TBC_OPT_DIRECTION = 1,  /* value: 0 auto (default), 1 push only, 2 pull whenever possible */
+    TBC_OPT_PULL_ALPHA = 2  /* auto mode: pull when alpha * pull_cost < push_cost (default 1.0) */
+};
+
+/* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since
+ * the last tbc_stats_reset; TEPS/roofline bookkeeping for the bench. */
+typedef struct {
+    int64_t sources;     /* sources processed */
+    int64_t reached;     /* sum over sources of reached vertices (s included) */
+    int64_t reached_edges; /* sum over sources of the out-edges of the reached vertices */
+    int64_t fwd_edges;   /* stored entries examined by forward levels (push: frontier
+                            out-edges, pull: candidate in-edges, coot: nnz per level) */
+    int64_t bwd_edges;   /* stored entries examined by backward levels */
+    int64_t levels;      /* forward levels run (incl. the final empty one) */
+    int64_t pull_levels; /* forward levels run as pull */
+    int64_t scans;       /* candidate scans (first pull level of a source) */
+    int64_t max_depth;   /* deepest BFS height seen */
+} tbc_stats;
+
+/* Create a graph from the CSC of A (CP_A = col_ptr, row_A = row_idx, here 0-based).
+ *   n       : number of vertices, 1 <= n < 2^31
+ *   nnz     : col_ptr[n]; entries in row_idx
+ *   col_ptr : host int64[n+1], col_ptr[0] = 0, non-decreasing, col_ptr[n] = nnz
+ *   row_idx : host int32[nnz], rows in [0, n); any order within a column; duplicates ok
+ *   directed: 0 = undirected (pattern must be symmetric; validated unless NO_VALIDATE;
+ *             bc halved per P:180), 1 = directed
+ *   engine  : TBC_ENGINE_CSC or TBC_ENGINE_COOT
+ *   device  : CUDA device ordinal
+ *   out     : receives the handle (NULL on error)
+ * The host arrays are copied; the caller may free them on return.  The graph is
+ * canonicalised on the device (sorted, deduplicated columns; CSR copy for directed graphs).
+ * Errors: TBC_ERR_INVALID (arguments/malformed/asymmetric), TBC_ERR_OOM, TBC_ERR_CUDA. */
+tbc_status tbc_graph_create_csc(int64_t n, int64_t nnz, const int64_t *col_ptr,
+                                const int32_t *row_idx, int directed, int engine,
+                                unsigned flags, int device, tbc_graph **out);
+
+/* Create a graph from an edge list: edge k is src[k] -> dst[k], i.e. A(src,dst) = 1,
+ * stored as row src[k] of column dst[k] (the COOC arrays row_A = src, col_A = dst).
+ * Arguments and errors as tbc_graph_create_csc; nnz >= 0 entries, ids in [0, n). */
+tbc_status tbc_graph_create_coo(int64_t n, int64_t nnz, const int32_t *src, const int32_t *dst,
+                                int directed, int engine, unsigned flags, int device,
+                                tbc_graph **out);
+
+/* Betweenness centrality over a source list (Alg.1 l.6 generalised to a list).
+ *   sources: host int32[k], each in [0, n) (validated; TBC_ERR_INVALID otherwise); k >= 0
+ *   bc_out : host double[n], OVERWRITTEN with bc(v) = sum_{s in list} delta_s(v)
+ *            (x 1/2 per source if undirected).  k = 0 gives all zeros.
+ * Synchronous. */
+tbc_status tbc_bc(tbc_graph *g, const int32_t *sources, int64_t k, double *bc_out);
+
+/* Device-pointer variant for framework integration (PyTorch tensors, multi-GPU ranks).
+ *   d_sources   : device int32[k] on the graph's device; out-of-range entries are skipped
+ *                 and counted (not validated on the host)
+ *   d_bc        : device double[n]; the result is ACCUMULATED into it (bc += ...)
+ *   cuda_stream : cudaStream_t to run on (NULL = legacy default stream)
+ * Asynchronous with respect to the host; errors of the launch itself are returned. */
+tbc_status tbc_bc_device(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc,
+                         void *cuda_stream);
+
+/* Forward stage only (Alg.1 l.11-28) from one source.
+ *   depth_out: host int32[n] or NULL; sigma_out: host double[n] or NULL.  Synchronous. */
+tbc_status tbc_bfs(tbc_graph *g, int32_t source, int32_t *depth_out, double *sigma_out);
+
+/* Graph properties after canonicalisation; any output pointer may be NULL.
+ *   nnz = stored entries of A after deduplication; device_bytes = device memory owned. */
+tbc_status tbc_graph_info(const tbc_graph *g, int64_t *n, int64_t *nnz, int *directed,
+                          size_t *device_bytes);
+
+/* Engine options (TBC_OPT_*); TBC_ERR_INVALID for an unknown key or value. */
+tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value);
+
+/* Read (synchronises the graph's device) / reset the accumulated counters. */
+tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out);
+tbc_status tbc_stats_reset(tbc_graph *g);
+
+/* Free everything the handle owns.  NULL is a no-op. */
+tbc_status tbc_destroy(tbc_graph *g);
+
+const char *tbc_status_string(tbc_status s);
+const char *tbc_last_error(void); /* thread-local; "" if none */
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TBC_H */

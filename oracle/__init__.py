@@ -45,6 +45,9 @@ def _load():
         P = ctypes.POINTER
         lib.oracle_bc.argtypes = [i64, P(i64), P(i32), ctypes.c_int, P(i32), i64, ctypes.c_int, P(dbl)]
         lib.oracle_bc.restype = ctypes.c_int
+        lib.oracle_bc_timed.argtypes = [i64, P(i64), P(i32), ctypes.c_int, P(i32), i64, ctypes.c_int, P(dbl),
+                                        P(dbl)]
+        lib.oracle_bc_timed.restype = ctypes.c_int
         lib.oracle_bfs.argtypes = [i64, P(i64), P(i32), i32, P(i32), P(dbl)]
         lib.oracle_bfs.restype = ctypes.c_int
         lib.oracle_delta.argtypes = [i64, P(i64), P(i32), i32, P(dbl)]
@@ -81,6 +84,22 @@ def bc(col_ptr, row_idx, directed: bool, sources, nthreads: int | None = None) -
     if rc != 0:
         raise ValueError("oracle_bc: invalid input")
     return out
+
+
+def bc_timed(col_ptr, row_idx, directed: bool, sources, nthreads: int):
+    """(bc, seconds of the source loop alone, graph build excluded) -- bench cpu_baseline hook."""
+    lib = _load()
+    cp, ri = _csc(col_ptr, row_idx)
+    n = cp.size - 1
+    src = np.ascontiguousarray(sources, dtype=np.int32)
+    out = np.zeros(n, dtype=np.float64)
+    secs = ctypes.c_double(0.0)
+    rc = lib.oracle_bc_timed(n, _ptr(cp, ctypes.c_int64), _ptr(ri, ctypes.c_int32), int(bool(directed)),
+                             _ptr(src, ctypes.c_int32), src.size, int(nthreads), _ptr(out, ctypes.c_double),
+                             ctypes.byref(secs))
+    if rc != 0:
+        raise ValueError("oracle_bc_timed: invalid input")
+    return out, secs.value
 
 
 def bfs(col_ptr, row_idx, source: int):

@@ -26,10 +26,12 @@
  * Parity status: every function here is pinned by tests/test_oracle.py against
  * brute-force Eq. 1 (exact rationals), closed forms, invariants and networkx.
  */
+#define _POSIX_C_SOURCE 199309L
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
 #include <pthread.h>
+#include <time.h>
 
 typedef struct {
     int64_t n;
@@ -201,8 +203,20 @@ static void *og_thread(void *arg) {
 /* bc over an explicit source list (Alg.1 l.6 generalised to a list), nthreads >= 1
  * threads over contiguous source ranges, partials reduced in thread order.
  * Returns 0, or -1 on bad input / allocation failure. */
+int oracle_bc_timed(int64_t n, const int64_t *col_ptr, const int32_t *row_idx, int directed,
+                    const int32_t *sources, int64_t k, int nthreads, double *bc_out,
+                    double *compute_seconds);
+
 int oracle_bc(int64_t n, const int64_t *col_ptr, const int32_t *row_idx, int directed,
               const int32_t *sources, int64_t k, int nthreads, double *bc_out) {
+    return oracle_bc_timed(n, col_ptr, row_idx, directed, sources, k, nthreads, bc_out, NULL);
+}
+
+/* Same as oracle_bc; if compute_seconds != NULL it receives the wall time of the source loop
+ * alone (graph build excluded) -- a measurement hook for bench.py's cpu_baseline. */
+int oracle_bc_timed(int64_t n, const int64_t *col_ptr, const int32_t *row_idx, int directed,
+                    const int32_t *sources, int64_t k, int nthreads, double *bc_out,
+                    double *compute_seconds) {
     if (n <= 0 || k < 0 || !bc_out) return -1;
     for (int64_t i = 0; i < k; ++i) if (sources[i] < 0 || sources[i] >= n) return -1;
     og_graph g;
@@ -218,10 +232,15 @@ int oracle_bc(int64_t n, const int64_t *col_ptr, const int32_t *row_idx, int dir
         tasks[t].bc = (double *)calloc((size_t)n, sizeof(double));
         if (!tasks[t].bc) rc = -1;
     }
+    struct timespec t0, t1;
+    clock_gettime(CLOCK_MONOTONIC, &t0);
     if (!rc) {
         for (int t = 0; t < nthreads; ++t) pthread_create(&th[t], NULL, og_thread, &tasks[t]);
         for (int t = 0; t < nthreads; ++t) { pthread_join(th[t], NULL); if (tasks[t].status) rc = -1; }
     }
+    clock_gettime(CLOCK_MONOTONIC, &t1);
+    if (compute_seconds)
+        *compute_seconds = (double)(t1.tv_sec - t0.tv_sec) + 1e-9 * (double)(t1.tv_nsec - t0.tv_nsec);
     if (!rc) {
         for (int64_t v = 0; v < n; ++v) bc_out[v] = 0.0;
         for (int t = 0; t < nthreads; ++t)

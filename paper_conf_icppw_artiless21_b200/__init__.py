@@ -1,0 +1,182 @@
+"""Python binding of libturbobc (include/tbc.h): argument marshalling only.
+
+Every step of the TurboBC hot path (Algorithm 1) runs in the CUDA
+kernels of ``csrc/``; this module converts numpy / torch arguments to the C ABI and raises
+on error.  There is no CPU fallback: if the extension cannot be loaded, import of the
+compute entry points raises.
+
+    g = Graph.from_csc(col_ptr, row_idx, directed=False)       # tbc_graph_create_csc
+    bc = g.bc(sources)                                          # tbc_bc  -> float64[n]
+    depth, sigma = g.bfs(s)                                     # tbc_bfs
+    g.bc_device(src_tensor, bc_tensor, stream)                  # tbc_bc_device (accumulates)
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+from . import build as _build
+
+__all__ = ["Graph", "TBCError", "lib", "ENGINE_CSC", "ENGINE_COOT", "DIR_AUTO", "DIR_PUSH", "DIR_PULL"]
+
+ENGINE_CSC, ENGINE_COOT = 0, 1
+FLAG_ONE_FORMAT, FLAG_NO_VALIDATE = 1, 2
+OPT_DIRECTION, OPT_PULL_ALPHA = 1, 2
+DIR_AUTO, DIR_PUSH, DIR_PULL = 0, 1, 2
+STATUS = {0: "TBC_OK", 1: "TBC_ERR_INVALID", 2: "TBC_ERR_OOM", 3: "TBC_ERR_CUDA", 4: "TBC_ERR_UNSUPPORTED"}
+
+# every symbol include/tbc.h declares (checked by tests/test_abi.py)
+SYMBOLS = ["tbc_graph_create_csc", "tbc_graph_create_coo", "tbc_bc", "tbc_bc_device", "tbc_bfs",
+           "tbc_graph_info", "tbc_graph_set_option", "tbc_stats_get", "tbc_stats_reset", "tbc_destroy",
+           "tbc_status_string", "tbc_last_error"]
+
+
+class TBCError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [(f, ctypes.c_int64) for f in
+                ("sources", "reached", "reached_edges", "fwd_edges", "bwd_edges", "levels", "pull_levels", "scans", "max_depth")]
+
+    def as_dict(self):
+        return {f: int(getattr(self, f)) for f, _ in self._fields_}
+
+
+_LIB = None
+
+
+def lib():
+    """Load libturbobc.so (building it in-tree first if the sources are newer)."""
+    global _LIB
+    if _LIB is None:
+        path = _build.build()
+        L = ctypes.CDLL(path)
+        i64, i32, P = ctypes.c_int64, ctypes.c_int32, ctypes.POINTER
+        vp = ctypes.c_void_p
+        L.tbc_graph_create_csc.argtypes = [i64, i64, P(i64), P(i32), ctypes.c_int, ctypes.c_int,
+                                           ctypes.c_uint, ctypes.c_int, P(vp)]
+        L.tbc_graph_create_coo.argtypes = [i64, i64, P(i32), P(i32), ctypes.c_int, ctypes.c_int,
+                                           ctypes.c_uint, ctypes.c_int, P(vp)]
+        L.tbc_bc.argtypes = [vp, P(i32), i64, P(ctypes.c_double)]
+        L.tbc_bc_device.argtypes = [vp, vp, i64, vp, vp]
+        L.tbc_bfs.argtypes = [vp, i32, P(i32), P(ctypes.c_double)]
+        L.tbc_graph_info.argtypes = [vp, P(i64), P(i64), P(ctypes.c_int), P(ctypes.c_size_t)]
+        L.tbc_graph_set_option.argtypes = [vp, ctypes.c_int, ctypes.c_double]
+        L.tbc_stats_get.argtypes = [vp, P(Stats)]
+        L.tbc_stats_reset.argtypes = [vp]
+        L.tbc_destroy.argtypes = [vp]
+        L.tbc_status_string.argtypes = [ctypes.c_int]
+        L.tbc_status_string.restype = ctypes.c_char_p
+        L.tbc_last_error.restype = ctypes.c_char_p
+        for name in SYMBOLS[:10]:
+            getattr(L, name).restype = ctypes.c_int
+        _LIB = L
+    return _LIB
+
+
+def _check(status):
+    if status != 0:
+        raise TBCError(status, lib().tbc_last_error().decode())
+
+
+def _p(a, ct):
+    return a.ctypes.data_as(ctypes.POINTER(ct))
+
+
+class Graph:
+    """A graph resident on one GPU (tbc_graph): CSC of A (+ CSR when directed), workspace."""
+
+    def __init__(self, handle, device):
+        self._h = ctypes.c_void_p(handle)
+        self.device = device
+        n, m, d, b = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int(), ctypes.c_size_t()
+        _check(lib().tbc_graph_info(self._h, ctypes.byref(n), ctypes.byref(m), ctypes.byref(d), ctypes.byref(b)))
+        self.n, self.nnz, self.directed, self.device_bytes = n.value, m.value, bool(d.value), b.value
+
+    @classmethod
+    def from_csc(cls, col_ptr, row_idx, directed: bool, engine: int = ENGINE_CSC, device: int = 0,
+                 validate: bool = True):
+        cp = np.ascontiguousarray(col_ptr, dtype=np.int64)
+        ri = np.ascontiguousarray(row_idx, dtype=np.int32)
+        n = cp.size - 1
+        h = ctypes.c_void_p()
+        flags = 0 if validate else FLAG_NO_VALIDATE
+        _check(lib().tbc_graph_create_csc(n, int(cp[-1]) if n >= 0 else 0, _p(cp, ctypes.c_int64),
+                                          _p(ri, ctypes.c_int32) if ri.size else None, int(directed),
+                                          engine, flags, device, ctypes.byref(h)))
+        return cls(h.value, device)
+
+    @classmethod
+    def from_coo(cls, n, src, dst, directed: bool, engine: int = ENGINE_CSC, device: int = 0,
+                 validate: bool = True):
+        s = np.ascontiguousarray(src, dtype=np.int32)
+        d = np.ascontiguousarray(dst, dtype=np.int32)
+        h = ctypes.c_void_p()
+        flags = 0 if validate else FLAG_NO_VALIDATE
+        _check(lib().tbc_graph_create_coo(int(n), s.size, _p(s, ctypes.c_int32) if s.size else None,
+                                          _p(d, ctypes.c_int32) if d.size else None, int(directed), engine,
+                                          flags, device, ctypes.byref(h)))
+        return cls(h.value, device)
+
+    # ------------------------------------------------------------------ compute
+    def bc(self, sources) -> np.ndarray:
+        """tbc_bc: host source list -> host float64[n] (overwritten, synchronous)."""
+        src = np.ascontiguousarray(sources, dtype=np.int32)
+        out = np.empty(self.n, dtype=np.float64)
+        _check(lib().tbc_bc(self._h, _p(src, ctypes.c_int32) if src.size else None, src.size,
+                            _p(out, ctypes.c_double)))
+        return out
+
+    def bc_device(self, sources, bc, stream=None):
+        """tbc_bc_device: torch int32 CUDA tensor of sources, ACCUMULATE into float64 CUDA tensor bc."""
+        import torch
+        assert sources.dtype == torch.int32 and sources.is_cuda and sources.is_contiguous()
+        assert bc.dtype == torch.float64 and bc.is_cuda and bc.numel() == self.n
+        if stream is None:
+            stream = torch.cuda.current_stream(sources.device)
+        _check(lib().tbc_bc_device(self._h, ctypes.c_void_p(sources.data_ptr()), sources.numel(),
+                                   ctypes.c_void_p(bc.data_ptr()), ctypes.c_void_p(stream.cuda_stream)))
+        return bc
+
+    def bfs(self, source: int):
+        """tbc_bfs: (depth int32[n], sigma float64[n]); depth(s)=0, unreachable -1."""
+        depth = np.empty(self.n, dtype=np.int32)
+        sigma = np.empty(self.n, dtype=np.float64)
+        _check(lib().tbc_bfs(self._h, int(source), _p(depth, ctypes.c_int32), _p(sigma, ctypes.c_double)))
+        return depth, sigma
+
+    def set_direction(self, mode: int):
+        _check(lib().tbc_graph_set_option(self._h, OPT_DIRECTION, float(mode)))
+
+    def set_alpha(self, alpha: float):
+        _check(lib().tbc_graph_set_option(self._h, OPT_PULL_ALPHA, float(alpha)))
+
+    def stats(self) -> dict:
+        st = Stats()
+        _check(lib().tbc_stats_get(self._h, ctypes.byref(st)))
+        return st.as_dict()
+
+    def reset_stats(self):
+        _check(lib().tbc_stats_reset(self._h))
+
+    def close(self):
+        if self._h is not None and self._h.value:
+            lib().tbc_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

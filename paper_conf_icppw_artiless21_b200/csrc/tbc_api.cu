@@ -1,0 +1,530 @@
+// tbc_api.cu -- the extern "C" boundary of libturbobc: graph creation (device-side
+// canonicalisation of the CSC / COOC input of P:95-97), the tbc_bc / tbc_bfs drivers,
+// options, statistics and error reporting.  Declarations and contracts: include/tbc.h.
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <vector>
+
+#include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_select.cuh>
+
+#include "tbc_internal.cuh"
+
+namespace tbc {
+
+static thread_local char g_err[512] = "";
+
+tbc_status set_error(tbc_status s, const char *fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof g_err, fmt, ap);
+    va_end(ap);
+    return s;
+}
+
+tbc_status cuda_error(cudaError_t e, const char *what) {
+    if (e == cudaErrorMemoryAllocation)
+        return set_error(TBC_ERR_OOM, "%s: %s", what, cudaGetErrorString(e));
+    return set_error(TBC_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+}  // namespace tbc
+
+using namespace tbc;
+
+#define TBC_CUDA(call)                                             \
+    do {                                                           \
+        cudaError_t e_ = (call);                                   \
+        if (e_ != cudaSuccess) { st = cuda_error(e_, #call); goto fail; } \
+    } while (0)
+
+namespace {
+
+// ----------------------------------------------------------------- canonicalisation kernels
+
+// key = (column << 32) | row for every stored entry of the caller's CSC (column-major order)
+__global__ void k_csc_to_keys(int64_t n, int64_t nnz, const int64_t *__restrict__ col_ptr,
+                              const int32_t *__restrict__ row, unsigned long long *keys) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t lo = 0, hi = n;  // largest c with col_ptr[c] <= i
+        while (hi - lo > 1) {
+            int64_t mid = (lo + hi) >> 1;
+            if (col_ptr[mid] <= i) lo = mid; else hi = mid;
+        }
+        keys[i] = ((unsigned long long)lo << 32) | (unsigned)row[i];
+    }
+}
+
+// key = (dst << 32) | src for an edge list src -> dst (A(src,dst) = 1, column dst)
+__global__ void k_coo_to_keys(int64_t nnz, const int32_t *__restrict__ src,
+                              const int32_t *__restrict__ dst, unsigned long long *keys) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz;
+         i += (int64_t)gridDim.x * blockDim.x)
+        keys[i] = ((unsigned long long)(unsigned)dst[i] << 32) | (unsigned)src[i];
+}
+
+// split sorted unique keys into (major ptr, minor idx); ptr[v] = first key with major >= v
+__global__ void k_keys_to_ptr(int64_t n, int64_t m, const unsigned long long *__restrict__ keys,
+                              int64_t *ptr, int32_t *idx, int32_t *major_out) {
+    int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += stride) {
+        idx[i] = (int32_t)(keys[i] & 0xffffffffull);
+        if (major_out) major_out[i] = (int32_t)(keys[i] >> 32);
+    }
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= n; v += stride) {
+        int64_t lo = 0, hi = m;  // lower_bound of major v
+        unsigned long long key = (unsigned long long)v << 32;
+        while (lo < hi) {
+            int64_t mid = (lo + hi) >> 1;
+            if (keys[mid] < key) lo = mid + 1; else hi = mid;
+        }
+        ptr[v] = lo;
+    }
+}
+
+__global__ void k_transpose_keys(int64_t m, const unsigned long long *__restrict__ in,
+                                 unsigned long long *out) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        unsigned long long k = in[i];
+        out[i] = (k << 32) | (k >> 32);
+    }
+}
+
+__global__ void k_count_mismatch(int64_t m, const unsigned long long *__restrict__ a,
+                                 const unsigned long long *__restrict__ b, unsigned long long *bad) {
+    unsigned long long local = 0;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+         i += (int64_t)gridDim.x * blockDim.x)
+        local += (a[i] != b[i]);
+    if (local) atomicAdd(bad, local);
+}
+
+__global__ void k_deg2(int64_t n, const int64_t *__restrict__ out_ptr,
+                       const int64_t *__restrict__ in_ptr, int2 *deg2) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+         v += (int64_t)gridDim.x * blockDim.x)
+        deg2[v] = make_int2((int)(out_ptr[v + 1] - out_ptr[v]), (int)(in_ptr[v + 1] - in_ptr[v]));
+}
+
+inline int grid_for(int64_t work) {
+    int64_t b = (work + 255) / 256;
+    if (b < 1) b = 1;
+    if (b > 148 * 16) b = 148 * 16;
+    return (int)b;
+}
+
+template <class T>
+cudaError_t dmalloc(tbc_graph *g, T **p, size_t count) {
+    size_t bytes = sizeof(T) * (count > 0 ? count : 1);
+    cudaError_t e = cudaMalloc((void **)p, bytes);
+    if (e == cudaSuccess) g->device_bytes += bytes;
+    return e;
+}
+
+void free_graph(tbc_graph *g) {
+    if (!g) return;
+    int cur = 0;
+    cudaGetDevice(&cur);
+    cudaSetDevice(g->device);
+    if (g->out_ptr != g->in_ptr) cudaFree(g->out_ptr);
+    if (g->out_idx != g->in_idx) cudaFree(g->out_idx);
+    cudaFree(g->in_ptr);
+    cudaFree(g->in_idx);
+    cudaFree(g->deg2);
+    cudaFree(g->coo_col);
+    cudaFree(g->depth);
+    cudaFree(g->sigma);
+    cudaFree(g->du);
+    cudaFree(g->gacc);
+    cudaFree(g->gcnt);
+    cudaFree(g->list_v);
+    cudaFree(g->list_pre);
+    cudaFree(g->tiles);
+    for (int b = 0; b < 2; ++b) {
+        cudaFree(g->cand_v[b]);
+        cudaFree(g->cand_pre[b]);
+        cudaFree(g->cand_tiles[b]);
+    }
+    cudaFree(g->lvl);
+    cudaFree(g->ctr);
+    cudaFree(g->bc_tmp);
+    cudaFree(g->src_tmp);
+    if (g->stream) cudaStreamDestroy(g->stream);
+    cudaSetDevice(cur);
+    delete g;
+}
+
+// Canonicalise entries given as keys (column << 32 | row) into the graph's CSC (+CSR/COO^T).
+// Consumes d_keys (device, nnz entries).  Runs on g->stream.
+tbc_status build_from_keys(tbc_graph *g, unsigned long long *d_keys, int64_t nnz) {
+    tbc_status st = TBC_OK;
+    cudaStream_t s = g->stream;
+    unsigned long long *alt = nullptr, *tkeys = nullptr, *d_bad = nullptr;
+    int64_t *d_num = nullptr;
+    void *temp = nullptr;
+    size_t temp_bytes = 0, need = 0;
+    int64_t m = 0;
+    unsigned long long bad = 0;
+    int end_bit = 32;
+    while ((1ll << (end_bit - 32)) < g->n) ++end_bit;
+    if (end_bit > 64) end_bit = 64;
+
+    TBC_CUDA(cudaMalloc(&alt, sizeof(unsigned long long) * (nnz > 0 ? nnz : 1)));
+    TBC_CUDA(cudaMalloc(&d_num, sizeof(int64_t)));
+    TBC_CUDA(cudaMalloc(&d_bad, sizeof(unsigned long long)));
+    if (nnz > 0) {
+        TBC_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, need, d_keys, alt, nnz, 0, end_bit, s));
+        temp_bytes = need;
+        TBC_CUDA(cub::DeviceSelect::Unique(nullptr, need, alt, d_keys, d_num, nnz, s));
+        if (need > temp_bytes) temp_bytes = need;
+        TBC_CUDA(cudaMalloc(&temp, temp_bytes));
+        TBC_CUDA(cub::DeviceRadixSort::SortKeys(temp, temp_bytes, d_keys, alt, nnz, 0, end_bit, s));
+        TBC_CUDA(cub::DeviceSelect::Unique(temp, temp_bytes, alt, d_keys, d_num, nnz, s));
+        TBC_CUDA(cudaMemcpyAsync(&m, d_num, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        TBC_CUDA(cudaStreamSynchronize(s));
+    }
+    g->m = m;
+    // CSC of A (in-neighbours)
+    TBC_CUDA(dmalloc(g, &g->in_ptr, g->n + 1));
+    TBC_CUDA(dmalloc(g, &g->in_idx, m));
+    if (g->engine == TBC_ENGINE_COOT) TBC_CUDA(dmalloc(g, &g->coo_col, m));
+    k_keys_to_ptr<<<grid_for(m > g->n ? m : g->n + 1), 256, 0, s>>>(g->n, m, d_keys, g->in_ptr,
+                                                                   g->in_idx, g->coo_col);
+    TBC_CUDA(cudaGetLastError());
+    if (!g->directed || g->engine == TBC_ENGINE_CSC) {
+        // transpose (row << 32 | col), sorted: the CSR of A; compared to the CSC when undirected
+        tkeys = alt;  // reuse: alt is free after Unique
+        alt = nullptr;
+        if (m > 0) {
+            TBC_CUDA(cudaMalloc(&alt, sizeof(unsigned long long) * m));
+            k_transpose_keys<<<grid_for(m), 256, 0, s>>>(m, d_keys, alt);
+            TBC_CUDA(cudaGetLastError());
+            need = 0;
+            TBC_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, need, alt, tkeys, m, 0, end_bit, s));
+            if (need > temp_bytes) {
+                cudaFree(temp);
+                temp = nullptr;
+                temp_bytes = need;
+                TBC_CUDA(cudaMalloc(&temp, temp_bytes));
+            }
+            TBC_CUDA(cub::DeviceRadixSort::SortKeys(temp, temp_bytes, alt, tkeys, m, 0, end_bit, s));
+        }
+        if (!g->directed) {
+            if (!(g->flags & TBC_FLAG_NO_VALIDATE) && m > 0) {
+                TBC_CUDA(cudaMemsetAsync(d_bad, 0, sizeof(unsigned long long), s));
+                k_count_mismatch<<<grid_for(m), 256, 0, s>>>(m, d_keys, tkeys, d_bad);
+                TBC_CUDA(cudaGetLastError());
+                TBC_CUDA(cudaMemcpyAsync(&bad, d_bad, sizeof bad, cudaMemcpyDeviceToHost, s));
+                TBC_CUDA(cudaStreamSynchronize(s));
+                if (bad) {
+                    st = set_error(TBC_ERR_INVALID,
+                                   "directed=0 but the pattern is not symmetric (%llu mismatches)", bad);
+                    goto fail;
+                }
+            }
+            g->out_ptr = g->in_ptr;
+            g->out_idx = g->in_idx;
+        } else {
+            TBC_CUDA(dmalloc(g, &g->out_ptr, g->n + 1));
+            TBC_CUDA(dmalloc(g, &g->out_idx, m));
+            k_keys_to_ptr<<<grid_for(m > g->n ? m : g->n + 1), 256, 0, s>>>(g->n, m, tkeys, g->out_ptr,
+                                                                           g->out_idx, nullptr);
+            TBC_CUDA(cudaGetLastError());
+        }
+    } else {
+        g->out_ptr = nullptr;  // COO^T directed: one format only
+        g->out_idx = nullptr;
+    }
+    TBC_CUDA(dmalloc(g, &g->deg2, g->n));
+    k_deg2<<<grid_for(g->n), 256, 0, s>>>(g->n, g->out_ptr ? g->out_ptr : g->in_ptr, g->in_ptr, g->deg2);
+    TBC_CUDA(cudaGetLastError());
+    TBC_CUDA(cudaStreamSynchronize(s));
+fail:
+    cudaFree(alt);
+    if (tkeys) cudaFree(tkeys);
+    cudaFree(temp);
+    cudaFree(d_num);
+    cudaFree(d_bad);
+    return st;
+}
+
+tbc_status create_common(int64_t n, int directed, int engine, unsigned flags, int device,
+                         tbc_graph **gout) {
+    if (n <= 0 || n >= (1ll << 31)) return set_error(TBC_ERR_INVALID, "n=%lld out of [1, 2^31)", (long long)n);
+    if (engine != TBC_ENGINE_CSC && engine != TBC_ENGINE_COOT)
+        return set_error(TBC_ERR_INVALID, "unknown engine %d", engine);
+    if (flags & TBC_FLAG_ONE_FORMAT)
+        return set_error(TBC_ERR_UNSUPPORTED, "TBC_FLAG_ONE_FORMAT is not implemented in this build");
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess) return cuda_error(e, "cudaGetDeviceCount");
+    if (device < 0 || device >= ndev) return set_error(TBC_ERR_INVALID, "device %d of %d", device, ndev);
+    e = cudaSetDevice(device);
+    if (e != cudaSuccess) return cuda_error(e, "cudaSetDevice");
+    tbc_graph *g = new tbc_graph();
+    g->device = device;
+    g->n = n;
+    g->directed = directed ? 1 : 0;
+    g->engine = engine;
+    g->flags = flags;
+    e = cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking);
+    if (e != cudaSuccess) {
+        delete g;
+        return cuda_error(e, "cudaStreamCreate");
+    }
+    *gout = g;
+    return TBC_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *tbc_status_string(tbc_status s) {
+    switch (s) {
+        case TBC_OK: return "TBC_OK";
+        case TBC_ERR_INVALID: return "TBC_ERR_INVALID";
+        case TBC_ERR_OOM: return "TBC_ERR_OOM";
+        case TBC_ERR_CUDA: return "TBC_ERR_CUDA";
+        case TBC_ERR_UNSUPPORTED: return "TBC_ERR_UNSUPPORTED";
+    }
+    return "TBC_ERR_UNKNOWN";
+}
+
+const char *tbc_last_error(void) { return g_err; }
+
+tbc_status tbc_graph_create_csc(int64_t n, int64_t nnz, const int64_t *col_ptr, const int32_t *row_idx,
+                                int directed, int engine, unsigned flags, int device, tbc_graph **out) {
+    g_err[0] = 0;
+    if (!out) return set_error(TBC_ERR_INVALID, "out is NULL");
+    *out = nullptr;
+    if (nnz < 0) return set_error(TBC_ERR_INVALID, "nnz < 0");
+    if (!col_ptr || (nnz > 0 && !row_idx)) return set_error(TBC_ERR_INVALID, "NULL array");
+    if (n > 0 && n < (1ll << 31) && !(flags & TBC_FLAG_NO_VALIDATE)) {
+        if (col_ptr[0] != 0) return set_error(TBC_ERR_INVALID, "col_ptr[0] = %lld != 0", (long long)col_ptr[0]);
+        if (col_ptr[n] != nnz) return set_error(TBC_ERR_INVALID, "col_ptr[n] != nnz");
+        for (int64_t v = 0; v < n; ++v)
+            if (col_ptr[v + 1] < col_ptr[v]) return set_error(TBC_ERR_INVALID, "col_ptr not monotone at %lld", (long long)v);
+        for (int64_t i = 0; i < nnz; ++i)
+            if (row_idx[i] < 0 || row_idx[i] >= n)
+                return set_error(TBC_ERR_INVALID, "row_idx[%lld] = %d out of range", (long long)i, row_idx[i]);
+    }
+    tbc_graph *g = nullptr;
+    tbc_status st = create_common(n, directed, engine, flags, device, &g);
+    if (st != TBC_OK) return st;
+    int64_t *d_cp = nullptr;
+    int32_t *d_row = nullptr;
+    unsigned long long *keys = nullptr;
+    TBC_CUDA(cudaMalloc(&d_cp, sizeof(int64_t) * (n + 1)));
+    TBC_CUDA(cudaMalloc(&d_row, sizeof(int32_t) * (nnz > 0 ? nnz : 1)));
+    TBC_CUDA(cudaMalloc(&keys, sizeof(unsigned long long) * (nnz > 0 ? nnz : 1)));
+    TBC_CUDA(cudaMemcpyAsync(d_cp, col_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, g->stream));
+    if (nnz > 0) {
+        TBC_CUDA(cudaMemcpyAsync(d_row, row_idx, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, g->stream));
+        k_csc_to_keys<<<grid_for(nnz), 256, 0, g->stream>>>(n, nnz, d_cp, d_row, keys);
+        TBC_CUDA(cudaGetLastError());
+    }
+    TBC_CUDA(cudaStreamSynchronize(g->stream));
+    cudaFree(d_cp);
+    d_cp = nullptr;
+    cudaFree(d_row);
+    d_row = nullptr;
+    st = build_from_keys(g, keys, nnz);
+    if (st != TBC_OK) goto fail;
+    cudaFree(keys);
+    keys = nullptr;
+    st = engine_setup(g);
+    if (st != TBC_OK) goto fail;
+    *out = g;
+    return TBC_OK;
+fail:
+    cudaFree(d_cp);
+    cudaFree(d_row);
+    cudaFree(keys);
+    free_graph(g);
+    return st;
+}
+
+tbc_status tbc_graph_create_coo(int64_t n, int64_t nnz, const int32_t *src, const int32_t *dst,
+                                int directed, int engine, unsigned flags, int device, tbc_graph **out) {
+    g_err[0] = 0;
+    if (!out) return set_error(TBC_ERR_INVALID, "out is NULL");
+    *out = nullptr;
+    if (nnz < 0) return set_error(TBC_ERR_INVALID, "nnz < 0");
+    if (nnz > 0 && (!src || !dst)) return set_error(TBC_ERR_INVALID, "NULL array");
+    if (n > 0 && n < (1ll << 31) && !(flags & TBC_FLAG_NO_VALIDATE)) {
+        for (int64_t i = 0; i < nnz; ++i)
+            if (src[i] < 0 || src[i] >= n || dst[i] < 0 || dst[i] >= n)
+                return set_error(TBC_ERR_INVALID, "edge %lld (%d -> %d) out of range", (long long)i, src[i], dst[i]);
+    }
+    tbc_graph *g = nullptr;
+    tbc_status st = create_common(n, directed, engine, flags, device, &g);
+    if (st != TBC_OK) return st;
+    int32_t *d_s = nullptr, *d_d = nullptr;
+    unsigned long long *keys = nullptr;
+    TBC_CUDA(cudaMalloc(&d_s, sizeof(int32_t) * (nnz > 0 ? nnz : 1)));
+    TBC_CUDA(cudaMalloc(&d_d, sizeof(int32_t) * (nnz > 0 ? nnz : 1)));
+    TBC_CUDA(cudaMalloc(&keys, sizeof(unsigned long long) * (nnz > 0 ? nnz : 1)));
+    if (nnz > 0) {
+        TBC_CUDA(cudaMemcpyAsync(d_s, src, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, g->stream));
+        TBC_CUDA(cudaMemcpyAsync(d_d, dst, sizeof(int32_t) * nnz, cudaMemcpyHostToDevice, g->stream));
+        k_coo_to_keys<<<grid_for(nnz), 256, 0, g->stream>>>(nnz, d_s, d_d, keys);
+        TBC_CUDA(cudaGetLastError());
+    }
+    TBC_CUDA(cudaStreamSynchronize(g->stream));
+    cudaFree(d_s);
+    d_s = nullptr;
+    cudaFree(d_d);
+    d_d = nullptr;
+    st = build_from_keys(g, keys, nnz);
+    if (st != TBC_OK) goto fail;
+    cudaFree(keys);
+    keys = nullptr;
+    st = engine_setup(g);
+    if (st != TBC_OK) goto fail;
+    *out = g;
+    return TBC_OK;
+fail:
+    cudaFree(d_s);
+    cudaFree(d_d);
+    cudaFree(keys);
+    free_graph(g);
+    return st;
+}
+
+tbc_status tbc_destroy(tbc_graph *g) {
+    g_err[0] = 0;
+    if (!g) return TBC_OK;
+    free_graph(g);
+    return TBC_OK;
+}
+
+tbc_status tbc_graph_info(const tbc_graph *g, int64_t *n, int64_t *nnz, int *directed, size_t *device_bytes) {
+    if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
+    if (n) *n = g->n;
+    if (nnz) *nnz = g->m;
+    if (directed) *directed = g->directed;
+    if (device_bytes) *device_bytes = g->device_bytes;
+    return TBC_OK;
+}
+
+tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
+    if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
+    if (key == TBC_OPT_DIRECTION) {
+        int v = (int)value;
+        if (v < 0 || v > 2 || (double)v != value) return set_error(TBC_ERR_INVALID, "direction %g", value);
+        g->dir_mode = v;
+        return TBC_OK;
+    }
+    if (key == TBC_OPT_PULL_ALPHA) {
+        if (!(value > 0)) return set_error(TBC_ERR_INVALID, "alpha %g", value);
+        g->alpha = value;
+        return TBC_OK;
+    }
+    return set_error(TBC_ERR_INVALID, "unknown option %d", key);
+}
+
+tbc_status tbc_bc_device(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, void *cuda_stream) {
+    g_err[0] = 0;
+    if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
+    if (k < 0) return set_error(TBC_ERR_INVALID, "k < 0");
+    if (k > 0 && (!d_sources || !d_bc)) return set_error(TBC_ERR_INVALID, "NULL device pointer");
+    if (k == 0) return TBC_OK;
+    cudaError_t e = cudaSetDevice(g->device);
+    if (e != cudaSuccess) return cuda_error(e, "cudaSetDevice");
+    return engine_run(g, d_sources, k, d_bc, (cudaStream_t)cuda_stream, 0);
+}
+
+tbc_status tbc_bc(tbc_graph *g, const int32_t *sources, int64_t k, double *bc_out) {
+    g_err[0] = 0;
+    if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
+    if (k < 0) return set_error(TBC_ERR_INVALID, "k < 0");
+    if (!bc_out || (k > 0 && !sources)) return set_error(TBC_ERR_INVALID, "NULL pointer");
+    for (int64_t i = 0; i < k; ++i)
+        if (sources[i] < 0 || sources[i] >= g->n)
+            return set_error(TBC_ERR_INVALID, "sources[%lld] = %d out of range", (long long)i, sources[i]);
+    tbc_status st = TBC_OK;
+    TBC_CUDA(cudaSetDevice(g->device));
+    if (!g->bc_tmp) TBC_CUDA(dmalloc(g, &g->bc_tmp, g->n));
+    if (k > g->src_cap) {
+        cudaFree(g->src_tmp);
+        g->src_tmp = nullptr;
+        g->src_cap = 0;
+        TBC_CUDA(cudaMalloc(&g->src_tmp, sizeof(int32_t) * k));
+        g->src_cap = k;
+    }
+    TBC_CUDA(cudaMemsetAsync(g->bc_tmp, 0, sizeof(double) * g->n, g->stream));
+    if (k > 0) {
+        TBC_CUDA(cudaMemcpyAsync(g->src_tmp, sources, sizeof(int32_t) * k, cudaMemcpyHostToDevice, g->stream));
+        st = engine_run(g, g->src_tmp, k, g->bc_tmp, g->stream, 0);
+        if (st != TBC_OK) return st;
+    }
+    TBC_CUDA(cudaMemcpyAsync(bc_out, g->bc_tmp, sizeof(double) * g->n, cudaMemcpyDeviceToHost, g->stream));
+    TBC_CUDA(cudaStreamSynchronize(g->stream));
+    return TBC_OK;
+fail:
+    return st;
+}
+
+tbc_status tbc_bfs(tbc_graph *g, int32_t source, int32_t *depth_out, double *sigma_out) {
+    g_err[0] = 0;
+    if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
+    if (source < 0 || source >= g->n) return set_error(TBC_ERR_INVALID, "source %d out of range", source);
+    tbc_status st = TBC_OK;
+    TBC_CUDA(cudaSetDevice(g->device));
+    if (g->src_cap < 1) {
+        TBC_CUDA(cudaMalloc(&g->src_tmp, sizeof(int32_t)));
+        g->src_cap = 1;
+    }
+    TBC_CUDA(cudaMemcpyAsync(g->src_tmp, &source, sizeof(int32_t), cudaMemcpyHostToDevice, g->stream));
+    st = engine_run(g, g->src_tmp, 1, nullptr, g->stream, 1);
+    if (st != TBC_OK) return st;
+    if (depth_out)
+        TBC_CUDA(cudaMemcpyAsync(depth_out, g->depth, sizeof(int32_t) * g->n, cudaMemcpyDeviceToHost, g->stream));
+    if (sigma_out)
+        TBC_CUDA(cudaMemcpyAsync(sigma_out, g->sigma, sizeof(double) * g->n, cudaMemcpyDeviceToHost, g->stream));
+    // forward-only runs leave depth/sigma set: restore the all-unvisited workspace invariant
+    TBC_CUDA(cudaMemsetAsync(g->depth, 0xff, sizeof(int32_t) * g->n, g->stream));
+    TBC_CUDA(cudaMemsetAsync(g->sigma, 0, sizeof(double) * g->n, g->stream));
+    TBC_CUDA(cudaStreamSynchronize(g->stream));
+    return TBC_OK;
+fail:
+    return st;
+}
+
+tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
+    if (!g || !out) return set_error(TBC_ERR_INVALID, "NULL pointer");
+    tbc_status st = TBC_OK;
+    Ctrs c;
+    TBC_CUDA(cudaSetDevice(g->device));
+    TBC_CUDA(cudaDeviceSynchronize());
+    TBC_CUDA(cudaMemcpy(&c, g->ctr, sizeof c, cudaMemcpyDeviceToHost));
+    out->sources = c.st_sources;
+    out->reached = c.st_reached;
+    out->reached_edges = c.st_reached_edges;
+    out->fwd_edges = c.st_fwd_edges;
+    out->bwd_edges = c.st_bwd_edges;
+    out->levels = c.st_levels;
+    out->pull_levels = c.st_pull_levels;
+    out->scans = c.st_scans;
+    out->max_depth = c.st_max_depth;
+    return TBC_OK;
+fail:
+    return st;
+}
+
+tbc_status tbc_stats_reset(tbc_graph *g) {
+    if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
+    tbc_status st = TBC_OK;
+    TBC_CUDA(cudaSetDevice(g->device));
+    TBC_CUDA(cudaDeviceSynchronize());
+    TBC_CUDA(cudaMemset(&g->ctr->st_sources, 0, sizeof(long long) * 9));
+    return TBC_OK;
+fail:
+    return st;
+}
+
+}  // extern "C"

@@ -1,0 +1,106 @@
+// tbc_internal.cuh -- shared definitions of libturbobc (graph object, workspace, params).
+// Product code: shares nothing with oracle/.
+#pragma once
+#include <cstdint>
+#include <cstddef>
+#include <cuda_runtime.h>
+#include "tbc.h"
+
+namespace tbc {
+
+constexpr int kBlock = 256;  // threads per CTA of the persistent kernel
+
+// Device-side counters of one graph; all fields are touched by the persistent kernel only.
+struct Ctrs {
+    unsigned long long list;      // packed (count << ebits) | edge_sum of the BFS-order list
+    unsigned long long indeg_vis; // sum of in-degrees of visited vertices (pull heuristic)
+    unsigned long long cand[2];   // packed counters of the two pull-candidate buffers
+    unsigned int bar_count;       // grid barrier arrival counter
+    unsigned int bar_gen;         // grid barrier generation
+    unsigned long long bad_sources;
+    // accumulated statistics (tbc_stats)
+    long long st_sources, st_reached, st_reached_edges, st_fwd_edges, st_bwd_edges, st_levels, st_pull_levels,
+        st_scans, st_max_depth;
+};
+
+struct Params {
+    int64_t n, m;
+    const int64_t *__restrict__ in_ptr;   // CSC: in-neighbours (column v = rows u with u->v)
+    const int32_t *__restrict__ in_idx;
+    const int64_t *__restrict__ out_ptr;  // CSR: out-neighbours (== in_* when undirected)
+    const int32_t *__restrict__ out_idx;
+    const int2 *__restrict__ deg2;        // {out-degree, in-degree}
+    int32_t *depth;                       // -1 unvisited
+    double *sigma;                        // path counts, 0 when not on the current BFS
+    double *du;                           // signed delta_u, sign = parity of the level
+    double *gacc;                         // split-owner partial sums (self-resetting)
+    int32_t *gcnt;                        // split-owner item counters (self-resetting)
+    int32_t *list_v;                      // BFS-order vertex list (levels concatenated)
+    int64_t *list_pre;                    // exclusive out-degree prefix along list_v
+    int32_t *tiles;                       // per level: owner index starting each tile
+    int32_t *cand_v[2];                   // pull candidate buffers
+    int64_t *cand_pre[2];
+    int32_t *cand_tiles[2];
+    int64_t *lvl;                         // per level: p0, N, e0, E, tile_base
+    Ctrs *ctr;
+    double *bc;
+    const int32_t *sources;
+    int64_t k;
+    double bc_scale;                      // 0.5 undirected, 1 directed
+    int ebits;                            // low bits of packed counters hold edge sums
+    int bfs_only;                         // forward stage only (tbc_bfs)
+    int dir_mode;                         // 0 auto, 1 push, 2 pull
+    double alpha;                         // pull when alpha*pull_cost < push_cost
+    // COO^T engine
+    const int32_t *coo_row;               // column-major (row, col) pairs = A's COOC arrays
+    const int32_t *coo_col;
+};
+
+}  // namespace tbc
+
+struct tbc_graph {
+    int device = 0;
+    int64_t n = 0, m = 0;
+    int directed = 0;
+    int engine = 0;
+    unsigned flags = 0;
+    // graph (device)
+    int64_t *in_ptr = nullptr;
+    int32_t *in_idx = nullptr;
+    int64_t *out_ptr = nullptr;  // aliases in_ptr when undirected
+    int32_t *out_idx = nullptr;
+    int2 *deg2 = nullptr;
+    int32_t *coo_col = nullptr;  // COO^T engine: column of each stored entry (rows = in_idx)
+    // workspace (device)
+    int32_t *depth = nullptr;
+    double *sigma = nullptr, *du = nullptr, *gacc = nullptr;
+    int32_t *gcnt = nullptr;
+    int32_t *list_v = nullptr;
+    int64_t *list_pre = nullptr;
+    int32_t *tiles = nullptr;
+    int32_t *cand_v[2] = {nullptr, nullptr};
+    int64_t *cand_pre[2] = {nullptr, nullptr};
+    int32_t *cand_tiles[2] = {nullptr, nullptr};
+    int64_t *lvl = nullptr;
+    tbc::Ctrs *ctr = nullptr;
+    double *bc_tmp = nullptr;
+    int32_t *src_tmp = nullptr;
+    int64_t src_cap = 0;
+    // launch
+    int grid = 0;
+    int ebits = 38;
+    int dir_mode = 0;
+    double alpha = 1.0;
+    cudaStream_t stream = nullptr;  // internal stream for the synchronous host API
+    size_t device_bytes = 0;
+};
+
+namespace tbc {
+// error plumbing (tbc_api.cu)
+tbc_status set_error(tbc_status s, const char *fmt, ...);
+tbc_status cuda_error(cudaError_t e, const char *what);
+// engine entry points (tbc_engine.cu)
+tbc_status engine_setup(tbc_graph *g);
+tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc,
+                      cudaStream_t stream, int bfs_only);
+}  // namespace tbc

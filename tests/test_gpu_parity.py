@@ -1,0 +1,221 @@
+"""CUDA path (through the C ABI) vs the CPU oracle, element by element.  Needs a B200.
+
+Bars (BASELINE.json north star):
+  depth  bit-exact;  sigma bit-exact while < 2^53 (relative 1e-12 above);
+  bc     |gpu - ora| <= 1e-9 |ora|, and ora == 0  =>  gpu == 0 exactly.
+"""
+import numpy as np
+import pytest
+
+import graphgen as gg
+import oracle
+import paper_conf_icppw_artiless21_b200 as tbc
+
+pytestmark = pytest.mark.gpu
+
+MODES = [tbc.DIR_AUTO, tbc.DIR_PUSH, tbc.DIR_PULL]
+
+
+def assert_bc(got, want, rel=1e-9):
+    got = np.asarray(got)
+    want = np.asarray(want)
+    zero = want == 0
+    assert np.all(got[zero] == 0.0), np.nonzero(got[zero])[0][:10]
+    err = np.abs(got[~zero] - want[~zero]) / np.abs(want[~zero])
+    assert err.size == 0 or err.max() <= rel, (err.max(), np.argmax(err))
+
+
+def assert_bfs(g, G, s):
+    d_gpu, s_gpu = G.bfs(int(s))
+    d_ora, s_ora = oracle.bfs(g.col_ptr, g.row_idx, int(s))
+    np.testing.assert_array_equal(d_gpu, d_ora)
+    exact = s_ora < 2.0 ** 53
+    np.testing.assert_array_equal(s_gpu[exact], s_ora[exact])
+    if (~exact).any():
+        np.testing.assert_allclose(s_gpu[~exact], s_ora[~exact], rtol=1e-12)
+
+
+def gpu_graph(g, **kw):
+    return tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, **kw)
+
+
+# ------------------------------------------------------------------ closed forms / small graphs
+
+SMALL = [gg.star(7), gg.star(7, directed_both=True), gg.path(7), gg.path(7, directed=True), gg.cycle(8),
+         gg.cycle(9), gg.complete(6), gg.complete_bipartite(3, 5), gg.grid(6, 7), gg.random_tree(50, 1),
+         gg.mycielski(6), gg.from_edges("one", 1, [], False), gg.from_edges("iso", 4, [(1, 2), (2, 3)], False)]
+
+
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("g", SMALL, ids=lambda g: g.name)
+def test_small_graphs_all_sources(g, mode):
+    with gpu_graph(g) as G:
+        G.set_direction(mode)
+        src = np.arange(g.n, dtype=np.int32)
+        assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, g.directed, src))
+        for s in range(min(g.n, 5)):
+            assert_bfs(g, G, s)
+
+
+@pytest.mark.parametrize("directed", [False, True])
+def test_random_small_graphs_many(directed):
+    rng = np.random.default_rng(5)
+    for t in range(40):
+        n = int(rng.integers(2, 60))
+        p = float(rng.choice([0.02, 0.08, 0.3]))
+        A = rng.random((n, n)) < p
+        np.fill_diagonal(A, False)
+        if not directed:
+            A = A | A.T
+        u, v = np.nonzero(A)
+        g = gg.from_edges("r", n, np.stack([u, v], 1), directed)
+        src = rng.integers(0, n, size=int(rng.integers(0, 2 * n))).astype(np.int32)
+        with gpu_graph(g) as G:
+            for mode in MODES:
+                G.set_direction(mode)
+                assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, directed, src))
+
+
+def test_grid_sigma_crosses_2_53():
+    g = gg.grid(40, 40)
+    with gpu_graph(g) as G:
+        for mode in MODES:
+            G.set_direction(mode)
+            assert_bfs(g, G, 0)
+            assert_bfs(g, G, 820)
+
+
+# ------------------------------------------------------------------ tile / hub edge cases
+
+@pytest.mark.parametrize("leaves", [1023, 1024, 1025, 5000, 70000])
+def test_hub_spans_many_tiles(leaves):
+    """A star centre owns one column spanning many merge-path tiles (split-owner protocol)."""
+    g = gg.star(leaves + 1)
+    with gpu_graph(g) as G:
+        for mode in MODES:
+            G.set_direction(mode)
+            src = np.array([0, 1, 2, leaves], dtype=np.int32)
+            assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, False, src))
+
+
+def test_double_star_and_directed_hubs():
+    # two hubs joined, leaves on both: split owners in push, pull and backward
+    e = [(0, 1)] + [(0, i) for i in range(2, 3000)] + [(1, i) for i in range(3000, 7000)]
+    g = gg.from_edges("dstar", 7000, e, False)
+    h = gg.from_edges("dstar_d", 7000, e + [(i, 1) for i in range(2, 3000)], True)
+    for gr in (g, h):
+        with gpu_graph(gr) as G:
+            for mode in MODES:
+                G.set_direction(mode)
+                src = np.array([0, 1, 2, 3001, 6999], dtype=np.int32)
+                assert_bc(G.bc(src), oracle.bc(gr.col_ptr, gr.row_idx, gr.directed, src))
+                assert_bfs(gr, G, 2)
+
+
+def test_duplicates_self_loops_and_coo_input():
+    rng = np.random.default_rng(1)
+    n = 300
+    u = rng.integers(0, n, 3000)
+    v = rng.integers(0, n, 3000)
+    u = np.concatenate([u, u[:500], np.arange(50)])    # duplicates and self-loops
+    v = np.concatenate([v, v[:500], np.arange(50)])
+    clean = gg.from_edges("clean", n, np.stack([u, v], 1), True)
+    src = np.arange(0, n, 7, dtype=np.int32)
+    want = oracle.bc(clean.col_ptr, clean.row_idx, True, src)
+    with tbc.Graph.from_coo(n, u, v, directed=True) as G:
+        # self-loops are kept in storage (they never join consecutive levels), duplicates collapse
+        assert G.nnz == clean.nnz + len(set(int(a) for a, b in zip(u, v) if a == b))
+        assert_bc(G.bc(src), want)
+    # raw CSC with unsorted rows, duplicates and self-loops
+    order = np.lexsort((rng.random(u.size), v))
+    cp = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(np.bincount(v, minlength=n), out=cp[1:])
+    with tbc.Graph.from_csc(cp, u[order], directed=True) as G:
+        assert_bc(G.bc(src), want)
+
+
+def test_errors_and_semantics():
+    g = gg.path(5)
+    with gpu_graph(g) as G:
+        with pytest.raises(tbc.TBCError):
+            G.bc([0, 9])
+        assert np.all(G.bc([]) == 0)
+        one = G.bc([2])
+        np.testing.assert_array_equal(G.bc([2, 2, 2]), 3 * one)
+    asym = gg.path(5, directed=True)
+    with pytest.raises(tbc.TBCError) as e:
+        tbc.Graph.from_csc(asym.col_ptr, asym.row_idx, directed=False)
+    assert e.value.status == 1
+
+
+def test_bc_device_accumulates():
+    import torch
+    g = gg.kronecker(10, 8, seed=3, directed=False)
+    src = gg.sources(g, 32, seed=1)
+    with gpu_graph(g) as G:
+        s = torch.from_numpy(src).cuda()
+        acc = torch.ones(g.n, dtype=torch.float64, device="cuda")
+        G.bc_device(s[:10], acc)
+        G.bc_device(s[10:], acc)
+        torch.cuda.synchronize()
+        assert_bc(acc.cpu().numpy() - 1.0, oracle.bc(g.col_ptr, g.row_idx, False, src), rel=1e-9)
+
+
+# ------------------------------------------------------------------ the configs
+
+def test_cfg1_exact_bc_all_sources():
+    """Config 1 (BASELINE.json configs[0]): ER n=1024, M=4096, all 1024 sources."""
+    g, src = gg.make_config(1)
+    want = oracle.bc(g.col_ptr, g.row_idx, False, src)
+    with gpu_graph(g) as G:
+        for mode in MODES:
+            G.set_direction(mode)
+            assert_bc(G.bc(src), want)
+        for s in (0, 17, 1023):
+            assert_bfs(g, G, s)
+
+
+@pytest.mark.parametrize("scale,directed", [(14, False), (15, True)])
+def test_kronecker_reduced_scale_full_oracle(scale, directed):
+    g = gg.kronecker(scale, 16, seed=2, directed=directed, device="cuda")
+    src = gg.sources(g, 256, seed=12)
+    want = oracle.bc(g.col_ptr, g.row_idx, directed, src)
+    with gpu_graph(g) as G:
+        for mode in MODES:
+            G.set_direction(mode)
+            assert_bc(G.bc(src), want)
+        for s in src[:3]:
+            assert_bfs(g, G, s)
+
+
+def test_cfg2_rmat18_sample():
+    """Config 2 at full size: 64 of its 1024 sources against the oracle (all cores)."""
+    g, src = gg.make_config(2, device="cuda")
+    src = src[:64]
+    with gpu_graph(g) as G:
+        assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, False, src))
+        for s in src[:2]:
+            assert_bfs(g, G, s)
+
+
+def test_cfg3_kron22_directed_sample_in_bench_launch_config():
+    """Config 3 at full size (the bench workload), sampled sources, auto direction."""
+    g, src = gg.make_config(3, device="cuda")
+    sample = src[:8]
+    with gpu_graph(g) as G:
+        assert_bc(G.bc(sample), oracle.bc(g.col_ptr, g.row_idx, True, sample))
+        for s in sample[:2]:
+            assert_bfs(g, G, s)
+        # per-source invariant at any size: sum_v bc_s(v) = sum_t (depth_s(t) - 1)
+        s = int(src[100])
+        depth, _ = G.bfs(s)
+        assert abs(G.bc([s]).sum() - float(np.sum(depth[depth > 0] - 1))) <= 1e-9 * max(1.0, depth.sum())
+
+
+@pytest.mark.parametrize("side", [256, 1024])
+def test_road_lattice(side):
+    g = gg.road_lattice(side, 0.10, seed=4)
+    src = gg.sources(g, 8, seed=14)
+    with gpu_graph(g) as G:
+        assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, False, src))
+        assert_bfs(g, G, src[0])

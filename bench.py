@@ -43,7 +43,10 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=None, help="sources in the CPU-oracle sample")
     ap.add_argument("--direction", type=int, default=0)
-    ap.add_argument("--alpha", type=float, default=1.0)
+    ap.add_argument("--format", type=int, default=0, help="0 auto, 1 list passes, 2 edge streams")
+    ap.add_argument("--engine", choices=["csc", "coot"], default="csc")
+    ap.add_argument("--cost", default="", help="cost model overrides, e.g. list=10,stream=2")
+    ap.add_argument("--trace", type=int, default=-1, help="print the per-level timeline of this source to stderr")
     return ap.parse_args()
 
 
@@ -200,10 +203,13 @@ def main():
     lo, hi = rank * per_gpu, (rank + 1) * per_gpu
     my_src = all_src[lo:hi]
     t0 = time.time()
-    G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, device=local)
+    engine = tbc.ENGINE_COOT if args.engine == "coot" else tbc.ENGINE_CSC
+    G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, engine=engine, device=local)
     create_s = time.time() - t0
     G.set_direction(args.direction)
-    G.set_alpha(args.alpha)
+    G.set_format(args.format)
+    if args.cost:
+        G.set_cost(**{k: float(v) for k, v in (kv.split("=") for kv in args.cost.split(","))})
     src_d = torch.from_numpy(my_src).to(dev)
     bc = torch.zeros(g.n, dtype=torch.float64, device=dev)
     stream = torch.cuda.current_stream(dev)
@@ -292,11 +298,12 @@ def main():
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "sec_per_source": total_ms / 1e3 / sources_total,
             "config": {"workload": _workload_name(args.config), "n": g.n, "m": g.nnz,
-                       "directed": g.directed, "engine": "csc", "sources_per_gpu": per_gpu,
+                       "directed": g.directed, "engine": args.engine, "sources_per_gpu": per_gpu,
                        "parallelism": f"source-partitioned x{world}, graph replicated, 1 NCCL all-reduce/step",
                        "l2": "inputs larger than L2 (CSC+CSR %.0f MB vs 126 MB L2); no flush" %
                              ((8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) / 1e6),
-                       "direction": args.direction, "alpha": args.alpha},
+                       "direction": args.direction, "format": args.format, "engine_kind": args.engine,
+                       "cost": args.cost},
             "clocks": clocks,
             "gpu_launches": args.steps,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -317,6 +324,12 @@ def main():
             "setup": {"generate_s": gen_s, "create_s": create_s, "device_bytes": G.device_bytes},
         }
         print(json.dumps(line), flush=True)
+    if args.trace >= 0 and rank == 0:
+        G.set_trace(args.trace)
+        G.bc(my_src[: args.trace + 1])
+        for r in G.trace():
+            print("TRACE " + json.dumps(r), file=sys.stderr)
+        G.set_trace(-1)
     G.close()
     if world > 1:
         dist.destroy_process_group()

@@ -61,10 +61,21 @@ enum {
     TBC_FLAG_NO_VALIDATE = 1u << 1  /* skip host-side input validation (caller guarantees it) */
 };
 
-/* options for tbc_graph_set_option */
+/* options for tbc_graph_set_option.  Every forward level is run as one of four passes, chosen
+ * by a per-item cost model: push over the frontier list,
+ * push over all stored entries (edge stream, the scCOOC form of Alg. 2), pull over the
+ * survivors of the previous pull, pull over all stored entries; every backward level as a
+ * list pass or an edge stream.  The options restrict or re-weight that choice. */
 enum {
-    TBC_OPT_DIRECTION = 1,  /* value: 0 auto (default), 1 push only, 2 pull whenever possible */
-    TBC_OPT_PULL_ALPHA = 2  /* auto mode: pull when alpha * pull_cost < push_cost (default 1.0) */
+    TBC_OPT_DIRECTION = 1,   /* 0 auto (default), 1 push only, 2 pull whenever possible (level >= 2) */
+    TBC_OPT_TRACE = 3,       /* index in the next calls' source lists whose per-level timeline is
+                                recorded (-1 = off, default) */
+    TBC_OPT_FORMAT = 4,      /* 0 auto (default), 1 list passes only, 2 edge streams only
+                                (TBC_ENGINE_COOT always streams) */
+    TBC_OPT_COST_LIST = 5,   /* cost model, picoseconds per item: list-pass item (default 10) */
+    TBC_OPT_COST_STREAM = 6, /*   stream-pass stored entry (default 2) */
+    TBC_OPT_COST_ATOMIC = 7, /*   push contribution (fp64 atomic) (default 20) */
+    TBC_OPT_COST_VERTEX = 8  /*   vertex of a whole-graph owner pass (default 1) */
 };
 
 /* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since
@@ -137,6 +148,16 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value);
 /* Read (synchronises the graph's device) / reset the accumulated counters. */
 tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out);
 tbc_status tbc_stats_reset(tbc_graph *g);
+
+/* Per-level timeline of the traced source (TBC_OPT_TRACE) of the last call that reached it:
+ *   out  : host int64[8 * cap]; entry i = {globaltimer ns, kind, level, N, E, a, b, 0} with
+ *          kind 0 init, 1 candidate scan, 2 push level, 3 pull edge pass, 4 backward edge pass,
+ *          5 owner pass (pull mask / backward delta); N/E = list size / out-edges produced
+ *          (fwd) or processed (bwd),
+ *          a/b = owners / edges the level traversed.  Timestamps are taken after each grid
+ *          barrier, so consecutive differences are level durations.
+ *   count: receives the number of entries recorded (<= 65536).  Synchronises the device. */
+tbc_status tbc_trace_get(tbc_graph *g, int64_t *out, int64_t cap, int64_t *count);
 
 /* Free everything the handle owns.  NULL is a no-op. */
 tbc_status tbc_destroy(tbc_graph *g);

@@ -19,18 +19,21 @@ import numpy as np
 
 from . import build as _build
 
-__all__ = ["Graph", "TBCError", "lib", "ENGINE_CSC", "ENGINE_COOT", "DIR_AUTO", "DIR_PUSH", "DIR_PULL"]
+__all__ = ["Graph", "TBCError", "lib", "ENGINE_CSC", "ENGINE_COOT", "DIR_AUTO", "DIR_PUSH", "DIR_PULL",
+           "FMT_AUTO", "FMT_LIST", "FMT_STREAM"]
 
 ENGINE_CSC, ENGINE_COOT = 0, 1
 FLAG_ONE_FORMAT, FLAG_NO_VALIDATE = 1, 2
-OPT_DIRECTION, OPT_PULL_ALPHA = 1, 2
+OPT_DIRECTION, OPT_TRACE, OPT_FORMAT = 1, 3, 4
+OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8}
+FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
 DIR_AUTO, DIR_PUSH, DIR_PULL = 0, 1, 2
 STATUS = {0: "TBC_OK", 1: "TBC_ERR_INVALID", 2: "TBC_ERR_OOM", 3: "TBC_ERR_CUDA", 4: "TBC_ERR_UNSUPPORTED"}
 
 # every symbol include/tbc.h declares (checked by tests/test_abi.py)
 SYMBOLS = ["tbc_graph_create_csc", "tbc_graph_create_coo", "tbc_bc", "tbc_bc_device", "tbc_bfs",
-           "tbc_graph_info", "tbc_graph_set_option", "tbc_stats_get", "tbc_stats_reset", "tbc_destroy",
-           "tbc_status_string", "tbc_last_error"]
+           "tbc_graph_info", "tbc_graph_set_option", "tbc_stats_get", "tbc_stats_reset", "tbc_trace_get",
+           "tbc_destroy", "tbc_status_string", "tbc_last_error"]
 
 
 class TBCError(RuntimeError):
@@ -69,11 +72,12 @@ def lib():
         L.tbc_graph_set_option.argtypes = [vp, ctypes.c_int, ctypes.c_double]
         L.tbc_stats_get.argtypes = [vp, P(Stats)]
         L.tbc_stats_reset.argtypes = [vp]
+        L.tbc_trace_get.argtypes = [vp, P(i64), i64, P(i64)]
         L.tbc_destroy.argtypes = [vp]
         L.tbc_status_string.argtypes = [ctypes.c_int]
         L.tbc_status_string.restype = ctypes.c_char_p
         L.tbc_last_error.restype = ctypes.c_char_p
-        for name in SYMBOLS[:10]:
+        for name in SYMBOLS[:11]:
             getattr(L, name).restype = ctypes.c_int
         _LIB = L
     return _LIB
@@ -153,8 +157,33 @@ class Graph:
     def set_direction(self, mode: int):
         _check(lib().tbc_graph_set_option(self._h, OPT_DIRECTION, float(mode)))
 
-    def set_alpha(self, alpha: float):
-        _check(lib().tbc_graph_set_option(self._h, OPT_PULL_ALPHA, float(alpha)))
+    def set_format(self, mode: int):
+        """0 auto, 1 list passes only, 2 edge-stream passes only."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_FORMAT, float(mode)))
+
+    def set_cost(self, **costs):
+        """Per-item cost model in ps: list=, stream=, atomic=, vertex=."""
+        for k, v in costs.items():
+            _check(lib().tbc_graph_set_option(self._h, OPT_COST[k], float(v)))
+
+    def set_trace(self, source_index: int):
+        """Record the per-level timeline of source_index of the next call(s) (-1 = off)."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_TRACE, float(source_index)))
+
+    def trace(self):
+        """List of per-level records of the traced source (see tbc_trace_get)."""
+        cap = 65536
+        buf = np.zeros(8 * cap, dtype=np.int64)
+        cnt = ctypes.c_int64()
+        _check(lib().tbc_trace_get(self._h, _p(buf, ctypes.c_int64), cap, ctypes.byref(cnt)))
+        names = ["init", "scan", "push", "pull_edges", "bwd_edges", "owner"]
+        rec = buf[: 8 * cnt.value].reshape(-1, 8)
+        out = []
+        for i, r in enumerate(rec):
+            dt = int(r[0] - rec[i - 1][0]) if i > 0 else 0
+            out.append({"kind": names[int(r[1])], "level": int(r[2]), "N": int(r[3]), "E": int(r[4]),
+                        "a": int(r[5]), "b": int(r[6]), "dt_us": dt / 1e3})
+        return out
 
     def stats(self) -> dict:
         st = Stats()

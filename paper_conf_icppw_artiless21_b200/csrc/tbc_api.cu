@@ -109,6 +109,18 @@ __global__ void k_deg2(int64_t n, const int64_t *__restrict__ out_ptr,
         deg2[v] = make_int2((int)(out_ptr[v + 1] - out_ptr[v]), (int)(in_ptr[v + 1] - in_ptr[v]));
 }
 
+// out-degrees from the rows of the CSC (one-format COO^T directed graphs have no CSR):
+// zero them, then count every stored row
+__global__ void k_out_degree(int64_t n, int64_t m, const int32_t *__restrict__ rows, int2 *deg2) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        deg2[v].x = 0;
+}
+
+__global__ void k_count_rows(int64_t m, const int32_t *__restrict__ rows, int2 *deg2) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(&deg2[rows[i]].x, 1);
+}
+
 inline int grid_for(int64_t work) {
     int64_t b = (work + 255) / 256;
     if (b < 1) b = 1;
@@ -134,22 +146,27 @@ void free_graph(tbc_graph *g) {
     cudaFree(g->in_ptr);
     cudaFree(g->in_idx);
     cudaFree(g->deg2);
-    cudaFree(g->coo_col);
+    cudaFree(g->in_col);
+    if (g->out_row != g->in_col) cudaFree(g->out_row);
     cudaFree(g->depth);
     cudaFree(g->sigma);
     cudaFree(g->du);
     cudaFree(g->gacc);
-    cudaFree(g->gcnt);
     cudaFree(g->list_v);
     cudaFree(g->list_pre);
+    cudaFree(g->list_beg);
     cudaFree(g->tiles);
     for (int b = 0; b < 2; ++b) {
+        cudaFree(g->fbm[b]);
+        cudaFree(g->bbm[b]);
         cudaFree(g->cand_v[b]);
         cudaFree(g->cand_pre[b]);
+        cudaFree(g->cand_beg[b]);
         cudaFree(g->cand_tiles[b]);
     }
     cudaFree(g->lvl);
     cudaFree(g->ctr);
+    cudaFree(g->trace);
     cudaFree(g->bc_tmp);
     cudaFree(g->src_tmp);
     if (g->stream) cudaStreamDestroy(g->stream);
@@ -190,9 +207,9 @@ tbc_status build_from_keys(tbc_graph *g, unsigned long long *d_keys, int64_t nnz
     // CSC of A (in-neighbours)
     TBC_CUDA(dmalloc(g, &g->in_ptr, g->n + 1));
     TBC_CUDA(dmalloc(g, &g->in_idx, m));
-    if (g->engine == TBC_ENGINE_COOT) TBC_CUDA(dmalloc(g, &g->coo_col, m));
+    TBC_CUDA(dmalloc(g, &g->in_col, m));  // column (owner) of every CSC entry: the COOC col_A
     k_keys_to_ptr<<<grid_for(m > g->n ? m : g->n + 1), 256, 0, s>>>(g->n, m, d_keys, g->in_ptr,
-                                                                   g->in_idx, g->coo_col);
+                                                                   g->in_idx, g->in_col);
     TBC_CUDA(cudaGetLastError());
     if (!g->directed || g->engine == TBC_ENGINE_CSC) {
         // transpose (row << 32 | col), sorted: the CSR of A; compared to the CSC when undirected
@@ -227,19 +244,30 @@ tbc_status build_from_keys(tbc_graph *g, unsigned long long *d_keys, int64_t nnz
             }
             g->out_ptr = g->in_ptr;
             g->out_idx = g->in_idx;
+            g->out_row = g->in_col;
         } else {
             TBC_CUDA(dmalloc(g, &g->out_ptr, g->n + 1));
             TBC_CUDA(dmalloc(g, &g->out_idx, m));
+            TBC_CUDA(dmalloc(g, &g->out_row, m));
             k_keys_to_ptr<<<grid_for(m > g->n ? m : g->n + 1), 256, 0, s>>>(g->n, m, tkeys, g->out_ptr,
-                                                                           g->out_idx, nullptr);
+                                                                           g->out_idx, g->out_row);
             TBC_CUDA(cudaGetLastError());
         }
     } else {
         g->out_ptr = nullptr;  // COO^T directed: one format only
         g->out_idx = nullptr;
+        g->out_row = nullptr;
     }
     TBC_CUDA(dmalloc(g, &g->deg2, g->n));
-    k_deg2<<<grid_for(g->n), 256, 0, s>>>(g->n, g->out_ptr ? g->out_ptr : g->in_ptr, g->in_ptr, g->deg2);
+    if (g->out_ptr) {
+        k_deg2<<<grid_for(g->n), 256, 0, s>>>(g->n, g->out_ptr, g->in_ptr, g->deg2);
+    } else {
+        k_deg2<<<grid_for(g->n), 256, 0, s>>>(g->n, g->in_ptr, g->in_ptr, g->deg2);
+        TBC_CUDA(cudaGetLastError());
+        k_out_degree<<<grid_for(g->n), 256, 0, s>>>(g->n, m, g->in_idx, g->deg2);
+        TBC_CUDA(cudaGetLastError());
+        if (m > 0) k_count_rows<<<grid_for(m), 256, 0, s>>>(m, g->in_idx, g->deg2);
+    }
     TBC_CUDA(cudaGetLastError());
     TBC_CUDA(cudaStreamSynchronize(s));
 fail:
@@ -419,9 +447,21 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->dir_mode = v;
         return TBC_OK;
     }
-    if (key == TBC_OPT_PULL_ALPHA) {
-        if (!(value > 0)) return set_error(TBC_ERR_INVALID, "alpha %g", value);
-        g->alpha = value;
+    if (key == TBC_OPT_TRACE) {
+        if (value < -1 || (double)(int64_t)value != value) return set_error(TBC_ERR_INVALID, "trace %g", value);
+        g->trace_src = (int64_t)value;
+        return TBC_OK;
+    }
+    if (key == TBC_OPT_FORMAT) {
+        int v = (int)value;
+        if (v < 0 || v > 2 || (double)v != value) return set_error(TBC_ERR_INVALID, "format %g", value);
+        g->fmt_mode = v;
+        return TBC_OK;
+    }
+    if (key >= TBC_OPT_COST_LIST && key <= TBC_OPT_COST_VERTEX) {
+        if (!(value >= 0)) return set_error(TBC_ERR_INVALID, "cost %g", value);
+        double *c[] = {&g->c_list, &g->c_stream, &g->c_atom, &g->c_vert};
+        *c[key - TBC_OPT_COST_LIST] = value;
         return TBC_OK;
     }
     return set_error(TBC_ERR_INVALID, "unknown option %d", key);
@@ -511,6 +551,24 @@ tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
     out->pull_levels = c.st_pull_levels;
     out->scans = c.st_scans;
     out->max_depth = c.st_max_depth;
+    return TBC_OK;
+fail:
+    return st;
+}
+
+tbc_status tbc_trace_get(tbc_graph *g, int64_t *out, int64_t cap, int64_t *count) {
+    if (!g || !count || (cap > 0 && !out)) return set_error(TBC_ERR_INVALID, "NULL pointer");
+    tbc_status st = TBC_OK;
+    Ctrs c;
+    int64_t nrec = 0;
+    TBC_CUDA(cudaSetDevice(g->device));
+    TBC_CUDA(cudaDeviceSynchronize());
+    TBC_CUDA(cudaMemcpy(&c, g->ctr, sizeof c, cudaMemcpyDeviceToHost));
+    nrec = (int64_t)c.trace_n;
+    if (nrec > kTraceCap) nrec = kTraceCap;
+    *count = nrec;
+    if (cap > 0 && nrec > 0)
+        TBC_CUDA(cudaMemcpy(out, g->trace, sizeof(int64_t) * 8 * (nrec < cap ? nrec : cap), cudaMemcpyDeviceToHost));
     return TBC_OK;
 fail:
     return st;

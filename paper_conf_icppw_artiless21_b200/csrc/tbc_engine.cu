@@ -1,23 +1,25 @@
 // tbc_engine.cu -- the per-source hot path of TurboBC (Algorithm 1) as one
-// persistent, cooperative sm_100a kernel per tbc_bc call.
+// persistent, cooperative sm_100a kernel per tbc_bc call (all sources, all levels).
 //
-//   forward  (Alg.1 l.11-28):  level-synchronous masked SpMV.  Each level is either
-//            PUSH  -- frontier (level d-1 list) scatters sigma along out-edges (CSR), claiming
-//                     undiscovered targets with a CAS on depth (K1' + K2 of DESIGN.md), or
-//            PULL  -- every still-undiscovered candidate sums sigma over in-edges (CSC) from
-//                     the frontier: exactly the masked f_t = A^T f of l.19-22 / Alg.3.
-//            Direction is chosen per level from frontier out-edges vs candidate in-edges.
-//   backward (Alg.1 l.29-47): for L = D..1, owners on level L sum delta_u of their
-//            out-neighbours on level L+1 (A delta_u, reading R1), delta = sigma * sum,
-//            bc += delta (x 1/2 undirected), delta_u = (1+delta)/sigma (l.35).
+//   forward  (Alg.1 l.11-28): level-synchronous masked SpMV.  Each level is either
+//            PUSH  -- the frontier (level d-1 list) scatters sigma along its out-edges (CSR);
+//                     the fp64 atomic that lifts sigma(x) from 0 claims x for level d, or
+//            PULL  -- every still-undiscovered candidate sums sigma over its in-edges (CSC)
+//                     from the frontier: the masked f_t = A^T f of l.19-22 / Alg.3,
+//                     then an owner pass applies the mask of l.20-25 (discovered iff sum > 0).
+//            Direction per level: frontier out-edges vs candidate in-edges.
+//   backward (Alg.1 l.29-47): for L = D..1 an edge pass sums delta_u of the
+//            out-neighbours on level L+1 (A delta_u, reading R1) into acc(v), then an owner
+//            pass sets delta = sigma * acc, bc += delta (x 1/2 undirected) and
+//            delta_u = (1+delta)/sigma (l.35), and resets the vertex for the next source.
 //
-// Every level is one merge-path pass over (owner list, out/in-edges): the diagonal of
-// (owner end items + edges) is cut into warp tiles of kWT items, so a 600k-edge hub and a million
-// degree-1 vertices cost the same per tile.  Tile start owners are written by the producers
-// of the list at append time (warp-aggregated append, see warp_append), so no search is
-// needed.  Levels are separated by a grid barrier inside the kernel: no host round trip per
-// level (the paper's per-level host loop), one launch per call for all sources.
-#include <cooperative_groups.h>
+// Edge passes are merge-path passes over (owner list, adjacency): the diagonal of (owner end
+// items + edges) is cut into warp tiles of kWT items, so a 600k-edge hub and a million
+// degree-1 vertices cost the same per tile.  The producer of a list writes the start owner of
+// every tile while appending (warp_flush), so no search is needed, and tiles are dealt to
+// warps round-robin (equal items per tile => balanced).  Phases are separated by a grid
+// barrier inside the kernel: no host round trip per level (cf. the paper's per-level kernels
+// and host loop).
 #include <cstdio>
 
 #include "tbc_internal.cuh"
@@ -28,19 +30,18 @@ namespace {
 constexpr unsigned FULL = 0xffffffffu;
 enum { MODE_PUSH = 0, MODE_PULL = 1, MODE_BWD = 2 };
 
-constexpr int kLaneItems = 8;              // items per lane per warp tile
-constexpr int kWT = 32 * kLaneItems;        // diagonal items per warp tile
+constexpr int kLaneItems = 8;          // items per lane per warp tile
+constexpr int kWT = 32 * kLaneItems;   // diagonal items per warp tile
 constexpr int kWarpsPerBlock = kBlock / 32;
 
+// per-warp slice of shared memory (owner window of one tile; reused as append buffers)
 struct __align__(16) WarpSmem {
-    int64_t beg[kWT + 1];    // adjacency position of the owner's first in-tile edge
-    double val[kWT + 1];     // PUSH: owner sigma; PULL/BWD: owner partial sum
+    int64_t beg[kWT + 2];    // adjacency position of the owner's first in-tile edge
+    double val[kWT + 2];     // PUSH: owner sigma; PULL/BWD: owner partial sum
     int32_t first[kWT + 2];  // slot of the owner's first in-tile edge (+ sentinel = ne)
-    int32_t deg[kWT + 1];    // owner degree in the traversed direction
-    int32_t own[kWT];        // owner (window index) of each edge slot
-    int32_t start0;          // owner 0 begins inside the tile
+    int32_t own[kWT + 2];    // owner (window index) of each edge slot
+    int32_t v[kWT + 2];      // owner vertex id
 };
-
 constexpr size_t kSmemBytes = sizeof(WarpSmem) * kWarpsPerBlock;
 
 // ------------------------------------------------------------------ memory-model helpers
@@ -50,6 +51,8 @@ __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
     asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
+
+__device__ __forceinline__ void fence_acq_rel() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 
 __device__ __forceinline__ uint64_t policy_evict_first() {
     uint64_t p;
@@ -64,7 +67,13 @@ __device__ __forceinline__ int ld_stream(const int32_t *ptr, uint64_t pol) {
     return v;
 }
 
-__device__ __forceinline__ void fence_acq_rel() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+// 16-byte streaming read of graph arrays (read-only for the whole kernel), L2 evict-first
+__device__ __forceinline__ int4 ld_stream4(const int32_t *ptr, uint64_t pol) {
+    int4 v;
+    asm volatile("ld.global.nc.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(ptr), "l"(pol));
+    return v;
+}
 
 __device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned long long *p) {
     return *(volatile const unsigned long long *)p;
@@ -78,71 +87,90 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 
 constexpr unsigned long long kWatchdogNs = 20ull * 1000 * 1000 * 1000;  // 20 s at one barrier
 
-// Grid-wide barrier for a cooperative (co-resident) grid.  Sense by generation counter.
+// Grid-wide barrier of the cooperative (co-resident) grid: release fence + arrival atomic,
+// the last arriver bumps the generation; waiters acquire it.  The acquire-side gpu fence also
+// invalidates this SM's L1, so plain loads after the barrier see other CTAs' writes.
 __device__ __forceinline__ void grid_sync(Ctrs *c, unsigned &gen) {
     __syncthreads();
     if (threadIdx.x == 0) {
-        unsigned g0 = gen;
-        __threadfence();
-        unsigned arrived = atomicAdd(&c->bar_count, 1u);
+        const unsigned g0 = gen;
+        fence_acq_rel();
+        const unsigned arrived = atomicAdd(&c->bar_count, 1u);
         if (arrived == gridDim.x - 1) {
             c->bar_count = 0;
-            __threadfence();
+            fence_acq_rel();
             atomicExch(&c->bar_gen, g0 + 1);
         } else {
             const unsigned long long t0 = globaltimer_ns();
             while (ld_acquire(&c->bar_gen) == g0) {
-                __nanosleep(32);
+                __nanosleep(20);
                 if (globaltimer_ns() - t0 > kWatchdogNs) __trap();  // never hang the GPU
             }
         }
-        __threadfence();  // acquire side; also invalidates this SM's L1 (CCTL.IVALL)
+        fence_acq_rel();
     }
     gen += 1;
     __syncthreads();
 }
 
+// ------------------------------------------------------------------ level bitmaps
+// fbm[d&1]: vertices discovered on level d (forward); bbm[L&1]: vertices of level L whose
+// delta_u is final (backward).  Cleared per source.  Within a source they are exact filters:
+// the in-neighbours of a still-undiscovered vertex lie on level d-1 or are undiscovered, and
+// the out-neighbours of a level-L vertex lie on levels <= L+1, so the same-parity levels that
+// share a bitmap never meet the test.  A 0.5 MB bitmap (scale 22) stays in L2, so the 8 B
+// gathers of sigma / delta_u from the 33 MB arrays happen only for real contributions.
+
+__device__ __forceinline__ bool bit_test(const uint32_t *bm, int32_t x) { return (bm[x >> 5] >> (x & 31)) & 1u; }
+__device__ __forceinline__ void bit_set(uint32_t *bm, int32_t x) { atomicOr(&bm[x >> 5], 1u << (x & 31)); }
+
 // ------------------------------------------------------------------ warp-aggregated append
 
-// Append the lanes with pred to a list (v, exclusive degree prefix) through ONE packed 64-bit
-// atomic per warp: (count << ebits) | degree_sum.  Because count and prefix are reserved
-// together, list order and prefix order agree, and each appended owner knows its merge-path
-// diagonal span [k0, k0+deg] inside its level, so it writes the start owner of every tile
-// whose first diagonal lies in that span.  All 32 lanes must call this.
-__device__ __forceinline__ void warp_append(bool pred, int32_t v, int64_t deg, unsigned long long *ctr,
-                                            int ebits, int32_t *lv, int64_t *lpre, int32_t *tiles,
-                                            int64_t p0, int64_t e0) {
-    unsigned mask = __ballot_sync(FULL, pred);
-    if (!mask) return;
-    const int lane = threadIdx.x & 31;
-    int64_t dg = pred ? deg : 0;
-    int64_t inc = dg;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        int64_t t = __shfl_up_sync(FULL, inc, o);
-        if (lane >= o) inc += t;
-    }
-    int64_t tot = __shfl_sync(FULL, inc, 31);
-    unsigned long long old = 0;
-    if (lane == 0)
-        old = atomicAdd(ctr, ((unsigned long long)__popc(mask) << ebits) + (unsigned long long)tot);
-    old = __shfl_sync(FULL, old, 0);
-    if (pred) {
-        int64_t p = (int64_t)(old >> ebits) + __popc(mask & ((1u << lane) - 1u));
-        int64_t e = (int64_t)(old & ((1ull << ebits) - 1ull)) + inc - dg;
-        lv[p] = v;
-        lpre[p] = e;
-        int64_t k0 = (e - e0) + (p - p0);
-        int64_t k1 = k0 + dg;
-        for (int64_t i = (k0 + kWT - 1) / kWT; i <= k1 / kWT; ++i) tiles[i] = (int32_t)(p - p0);
-    }
-}
+// Append c buffered entries (vertex bv[i], degree bd[i], adjacency begin bb[i]) with ONE packed
+// 64-bit atomic for the whole warp: (count << ebits) | degree_sum.  Count and prefix are
+// reserved together, so list order and prefix order agree and each owner knows its merge-path
+// span [k0, k0+deg] inside its level: it writes the start owner of every tile whose first
+// diagonal lies in that span.  Lane l takes entries [l*q, l*q+q); a warp scan of the lanes'
+// degree sums gives the prefixes.  c must be warp-uniform; all 32 lanes call this.
+struct ListOut {
+    unsigned long long *ctr;
+    int32_t *v;
+    int64_t *pre;
+    int64_t *beg;
+    int32_t *tiles;  // already offset to this level's tile base
+    int64_t p0, e0;  // level start within the list (list position, edge prefix)
+};
 
-// Warp-aggregated counter add (one atomic per warp); all 32 lanes must call this.
-__device__ __forceinline__ void warp_add(unsigned long long val, unsigned long long *ctr) {
+__device__ __forceinline__ void warp_flush(int c, const int32_t *bv, const int32_t *bd, const int64_t *bb,
+                                           const ListOut &o, int ebits) {
+    if (c == 0) return;
+    const int lane = threadIdx.x & 31;
+    const int q = (c + 31) >> 5;
+    const int lo = min(lane * q, c), hi = min(lo + q, c);
+    int64_t sum = 0;
+    for (int i = lo; i < hi; ++i) sum += bd[i];
+    int64_t inc = sum;
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) val += __shfl_xor_sync(FULL, val, o);
-    if ((threadIdx.x & 31) == 0 && val) atomicAdd(ctr, val);
+    for (int k = 1; k < 32; k <<= 1) {
+        const int64_t t = __shfl_up_sync(FULL, inc, k);
+        if (lane >= k) inc += t;
+    }
+    const int64_t tot = __shfl_sync(FULL, inc, 31);
+    unsigned long long old = 0;
+    if (lane == 0) old = atomicAdd(o.ctr, ((unsigned long long)c << ebits) + (unsigned long long)tot);
+    old = __shfl_sync(FULL, old, 0);
+    int64_t p = (int64_t)(old >> ebits) + lo;
+    int64_t e = (int64_t)(old & ((1ull << ebits) - 1ull)) + inc - sum;
+    for (int i = lo; i < hi; ++i, ++p) {
+        const int64_t dg = bd[i];
+        o.v[p] = bv[i];
+        o.pre[p] = e;
+        o.beg[p] = bb[i];
+        const int64_t k0 = (e - o.e0) + (p - o.p0);
+        const int64_t k1 = k0 + dg;
+        for (int64_t t = (k0 + kWT - 1) / kWT; t <= k1 / kWT; ++t) o.tiles[t] = (int32_t)(p - o.p0);
+        e += dg;
+    }
 }
 
 // ------------------------------------------------------------------ level descriptors
@@ -151,40 +179,30 @@ struct Level {
     int64_t p0, N, e0, E, tbase;
 };
 
-struct AppendTarget {
-    unsigned long long *ctr;
-    int32_t *v;
-    int64_t *pre;
-    int32_t *tiles;  // already offset to this level's tile base
-    int64_t p0, e0;  // level start within the list (list position, edge prefix)
-};
-
 __device__ __forceinline__ int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
-__device__ __forceinline__ double atomic_exch_d(double *p, double v) {
-    unsigned long long r = atomicExch((unsigned long long *)p, __double_as_longlong(v));
-    return __longlong_as_double(r);
-}
-
-// ------------------------------------------------------------------ merge-path level pass
+// ------------------------------------------------------------------ merge-path edge pass
 //
-// One WARP processes one tile of kWT diagonal items (owner end items + edges) with no block
-// barrier: tiles are assigned round-robin to the grid's warps (every tile holds the same number
-// of items, so the static assignment is balanced), the owner window lives in the warp's slice
-// of shared memory, each lane keeps kLaneItems index loads and kLaneItems gathers in flight.
-//
-// Owners: ov[0..N) with exclusive degree prefix opre[] (minus e0), tile starts otiles[].
-// adj_ptr/adj_idx: the traversed adjacency (CSR out-edges for PUSH/BWD, CSC in-edges for PULL).
-// d: the level being discovered (push/pull), or the owners' level L (bwd).
-// NOTE: ov/opre/otiles are written earlier in this same kernel (previous phases): they must
-// NOT be declared __restrict__ const, or the compiler may read them through the
+// One WARP processes one tile of kWT diagonal items with no block barrier.  Lane l owns the
+// kLaneItems CONSECUTIVE edge slots [l*kLaneItems, +kLaneItems) of the tile, so its owners come
+// out of the owner scan in registers and its per-owner sums are local runs; a single segmented
+// warp scan over the lanes' trailing runs joins owners that straddle lanes.  Each lane keeps
+// kLaneItems index loads and then kLaneItems gathers / atomics in flight.
+// Owners: ov[0..N) with exclusive degree prefix opre[] (minus e0), adjacency begin obeg[],
+// tile starts otiles[].  adj_idx: the traversed adjacency (CSR out-edges for PUSH/BWD, CSC
+// in-edges for PULL).  d: the level being discovered (PUSH/PULL) or the owners' level (BWD).
+// PULL/BWD hand each owner's sum to gacc[v]: a plain store when the whole owner lies in the
+// tile, an fp64 atomic add for the (at most two) owners cut by the tile's ends.  The owner
+// pass after the next barrier consumes and re-zeroes gacc.
+// NOTE: ov/opre/obeg/otiles are written earlier in this same kernel (previous phases): they
+// must NOT be declared __restrict__ const, or the compiler may read them through the
 // non-coherent (ld.global.nc) path and see stale lines.
 template <int MODE>
-__device__ __forceinline__ void level_pass(const Params &P, WarpSmem &ws, const int32_t *ov,
-                                           const int64_t *opre, const int32_t *otiles, int64_t N, int64_t E,
-                                           int64_t e0, const int64_t *__restrict__ adj_ptr,
-                                           const int32_t *__restrict__ adj_idx, int d, int64_t gwarp,
-                                           int64_t nwarps, AppendTarget lvl_out, AppendTarget cand_out) {
+__device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const int32_t *ov, const int64_t *opre,
+                                          const int64_t *obeg, const int32_t *otiles, int64_t N, int64_t E,
+                                          int64_t e0, const int64_t *__restrict__ adj_ptr,
+                                          const int32_t *__restrict__ adj_idx, int d, int64_t gwarp, int64_t nwarps,
+                                          ListOut out) {
     const int lane = threadIdx.x & 31;
     const int64_t K = N + E;
     const int64_t ntiles = ceil_div(K, kWT);
@@ -198,53 +216,56 @@ __device__ __forceinline__ void level_pass(const Params &P, WarpSmem &ws, const 
         const int nwin = (int)(min(pe, N - 1) - ps + 1);
         const int ne = (int)(ee - es);
 
-        // ---- owner window: slot of the first in-tile edge, adjacency position of that edge
+        // ---- owner window (three coalesced list reads): first in-tile slot, its adjacency position
+        bool start0 = true;
         for (int j = lane; j < nwin; j += 32) {
-            const int32_t v = ov[ps + j];
             const int64_t pre = opre[ps + j] - e0;
-            const int64_t b = adj_ptr[v];
-            const int64_t deg = adj_ptr[v + 1] - b;
             const int64_t f = max(pre, es);
+            const int32_t v = ov[ps + j];
             ws.first[j] = (int32_t)(f - es);
-            ws.beg[j] = b + (f - pre);
-            ws.deg[j] = (int32_t)deg;
+            ws.beg[j] = obeg[ps + j] + (f - pre);
+            ws.v[j] = v;
+            ws.own[j] = -1;
             if (MODE == MODE_PUSH) ws.val[j] = P.sigma[v];
             else ws.val[j] = 0.0;
-            if (j == 0) ws.start0 = (pre >= es) ? 1 : 0;  // owner 0 begins inside this tile
+            if (j == 0) start0 = pre >= es;  // owner 0 begins inside this tile
+
         }
+        start0 = __shfl_sync(FULL, start0, 0);
+        for (int sl = nwin + lane; sl < ne; sl += 32) ws.own[sl] = -1;
         if (lane == 0) ws.first[nwin] = ne;
-        for (int sl = lane; sl < ne; sl += 32) ws.own[sl] = -1;
         __syncwarp();
         for (int j = lane; j < nwin; j += 32)
             if (ws.first[j] < ws.first[j + 1]) ws.own[ws.first[j]] = j;
         __syncwarp();
-        // inclusive running max over own[0..ne): lane l scans slots [l*kLaneItems, +kLaneItems)
+        // owners of this lane's slots [l*kLaneItems, +kLaneItems): running max of the head marks
+        int o[kLaneItems];
         {
-            int loc[kLaneItems];
             int run = -1;
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
                 const int sl = lane * kLaneItems + i;
                 run = max(run, sl < ne ? ws.own[sl] : -1);
-                loc[i] = run;
+                o[i] = run;
             }
             int incl = run;
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const int t = __shfl_up_sync(FULL, incl, o);
-                if (lane >= o) incl = max(incl, t);
+            for (int k = 1; k < 32; k <<= 1) {
+                const int t = __shfl_up_sync(FULL, incl, k);
+                if (lane >= k) incl = max(incl, t);
             }
             int prev = __shfl_up_sync(FULL, incl, 1);
             if (lane == 0) prev = -1;
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
                 const int sl = lane * kLaneItems + i;
-                if (sl < ne) ws.own[sl] = max(prev, loc[i]);
+                o[i] = sl < ne ? max(prev, o[i]) : -1;
+                if (sl < ne) ws.own[sl] = o[i];
             }
         }
         __syncwarp();
 
-        // ---- edges: slot = i*32 + lane (consecutive lanes -> consecutive adjacency entries)
+        // ---- edges in coalesced order: slot = i*32 + lane (consecutive lanes -> consecutive entries)
         int xs[kLaneItems];
         int js[kLaneItems];
 #pragma unroll
@@ -259,132 +280,404 @@ __device__ __forceinline__ void level_pass(const Params &P, WarpSmem &ws, const 
             }
         }
         if (MODE == MODE_PUSH) {
-            // masked scatter f_t(x) += f(u) for undiscovered x (Alg.1 l.19-25 as a push)
+            // masked scatter f_t(x) += f(u) for x on levels {-1, d} (Alg.1 l.19-25 as a push).
+            // sigma is 0 off the current BFS, so the atomic that lifts sigma(x) from 0 is the
+            // unique claim of x.  All kLaneItems atomics are issued before any result is used.
             int dxs[kLaneItems];
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) dxs[i] = js[i] >= 0 ? P.depth[xs[i]] : -2;
+            double olds[kLaneItems];
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
-                bool claim = false;
-                if (dxs[i] == -1) {
-                    const int old = atomicCAS(&P.depth[xs[i]], -1, d);
-                    claim = (old == -1);
-                    dxs[i] = claim ? d : old;
-                }
-                if (dxs[i] == d) atomicAdd(&P.sigma[xs[i]], ws.val[js[i]]);
-                if (__any_sync(FULL, claim)) {
-                    int2 dg = make_int2(0, 0);
-                    if (claim) {
-                        P.du[xs[i]] = 0.0;
-                        dg = P.deg2[xs[i]];
-                    }
-                    warp_append(claim, xs[i], dg.x, lvl_out.ctr, P.ebits, lvl_out.v, lvl_out.pre, lvl_out.tiles,
-                                lvl_out.p0, lvl_out.e0);
-                    warp_add((unsigned long long)dg.y, &P.ctr->indeg_vis);  // visited in-edge mass
-                }
+                olds[i] = 1.0;
+                if (dxs[i] == -1 || dxs[i] == d) olds[i] = atomicAdd(&P.sigma[xs[i]], ws.val[js[i]]);
             }
+            __syncwarp();  // own[] / first[] / beg[] become the claim buffers below
+            int cnt = 0;
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) {
+                const bool claim = olds[i] == 0.0;
+                const unsigned cm = __ballot_sync(FULL, claim);
+                if (claim) {
+                    const int32_t x = xs[i];
+                    P.depth[x] = d;
+                    P.du[x] = 0.0;
+                    bit_set(P.fbm[d & 1], x);
+                    const int64_t b = adj_ptr[x];
+                    const int64_t dg = adj_ptr[x + 1] - b;
+                    const int pos = cnt + __popc(cm & ((1u << lane) - 1u));
+                    ws.own[pos] = x;
+                    ws.first[pos] = (int32_t)dg;
+                    ws.beg[pos] = b;
+                }
+                cnt += __popc(cm);
+            }
+            __syncwarp();
+            warp_flush(cnt, ws.own, ws.first, ws.beg, out, P.ebits);
         } else {
             double vals[kLaneItems];
+            if (MODE == MODE_PULL) {
+                // f_t(w) = sum over in-neighbours x on level d-1 of sigma(x)   (Alg.3 l.9-11)
+                const uint32_t *front = P.fbm[(d - 1) & 1];
+                bool hit[kLaneItems];
 #pragma unroll
-            for (int i = 0; i < kLaneItems; ++i) {
-                vals[i] = 0.0;
-                if (js[i] >= 0) {
-                    if (MODE == MODE_PULL) {
-                        // f_t(w) = sum over in-neighbours x on level d-1 of sigma(x)  (Alg.3 l.9-11)
-                        if (P.depth[xs[i]] == d - 1) vals[i] = P.sigma[xs[i]];
-                    } else {
-                        // (A delta_u)(v): out-neighbour x on level d+1; the level parity is the sign
-                        // of the stored delta_u, so concurrent same-level writes are rejected.
-                        const double u = P.du[xs[i]];
-                        const double want = ((d + 1) & 1) ? -u : u;
-                        vals[i] = want > 0.0 ? want : 0.0;
-                    }
+                for (int i = 0; i < kLaneItems; ++i) hit[i] = js[i] >= 0 && bit_test(front, xs[i]);
+#pragma unroll
+                for (int i = 0; i < kLaneItems; ++i) vals[i] = hit[i] ? P.sigma[xs[i]] : 0.0;
+            } else {
+                // (A delta_u)(v): out-neighbour x on level d+1.  The level parity is the sign of
+                // the stored delta_u, so neighbours on other levels contribute exactly 0.
+                const uint32_t *below = P.bbm[(d + 1) & 1];
+                bool hit[kLaneItems];
+#pragma unroll
+                for (int i = 0; i < kLaneItems; ++i) hit[i] = js[i] >= 0 && bit_test(below, xs[i]);
+#pragma unroll
+                for (int i = 0; i < kLaneItems; ++i) {
+                    const double u = hit[i] ? P.du[xs[i]] : 0.0;
+                    const double want = ((d + 1) & 1) ? -u : u;
+                    vals[i] = want > 0.0 ? want : 0.0;
                 }
             }
+            // transpose the values to lane-contiguous slots through shared memory (beg[] is dead)
+            double *vb = reinterpret_cast<double *>(ws.beg);
+            __syncwarp();
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) vb[i * 32 + lane] = vals[i];
+            __syncwarp();
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) vals[i] = vb[lane * kLaneItems + i];
+            // per-lane runs: interior runs are complete owners of this lane; the head run may
+            // continue an owner from the previous lane, the tail run may continue into the next
+            int head_o = o[0], tail_o = o[0];
+            double head_sum = 0.0, run = 0.0;
+            bool single = true;
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
-                // segmented (by owner) warp reduction; owners are non-decreasing across lanes
-                double val = vals[i];
-                const int ow = js[i];
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const double v2 = __shfl_down_sync(FULL, val, o);
-                    const int o2 = __shfl_down_sync(FULL, ow, o);
-                    if (lane + o < 32 && o2 == ow) val += v2;
+                if (o[i] < 0) continue;
+                if (o[i] != tail_o) {
+                    if (single) head_sum = run;
+                    else ws.val[tail_o] = run;
+                    single = false;
+                    run = 0.0;
+                    tail_o = o[i];
                 }
-                const int up = __shfl_up_sync(FULL, ow, 1);
-                if ((lane == 0 || up != ow) && ow >= 0 && val != 0.0) ws.val[ow] += val;
-                __syncwarp();
+                run += vals[i];
             }
-
-            // ---- owner finalisation (warp-uniform loop: appends are warp collectives)
-            for (int base = 0; base < nwin; base += 32) {
-                const int j = base + lane;
-                bool fin = false;
-                double total = 0.0;
-                int32_t v = 0;
-                if (j < nwin) {
-                    v = ov[ps + j];
-                    const bool end_in = ps + j < pe;
-                    const bool start_in = j > 0 || ws.start0;
-                    if (end_in && start_in) {
-                        fin = true;
-                        total = ws.val[j];
-                    } else {
-                        // owner split across tiles: partial sums meet in gacc[v]; the tile that
-                        // completes the item count (deg + 1) finalises and resets the slots
-                        const int c = (ws.first[j + 1] - ws.first[j]) + (end_in ? 1 : 0);
-                        if (c > 0) {
-                            if (ws.val[j] != 0.0) atomicAdd(&P.gacc[v], ws.val[j]);
-                            fence_acq_rel();
-                            const int old = atomicAdd(&P.gcnt[v], c);
-                            if (old + c == ws.deg[j] + 1) {
-                                fence_acq_rel();
-                                total = atomic_exch_d(&P.gacc[v], 0.0);
-                                P.gcnt[v] = 0;
-                                fin = true;
-                            }
-                        }
-                    }
+            // segmented inclusive scan of the tail runs across lanes (segment = same owner
+            // carried through lanes that hold a single run)
+            const int prev_tail = __shfl_up_sync(FULL, tail_o, 1);
+            bool flag = !(single && lane > 0 && prev_tail == tail_o && tail_o >= 0);
+            double S = run;
+#pragma unroll
+            for (int k = 1; k < 32; k <<= 1) {
+                const double s_up = __shfl_up_sync(FULL, S, k);
+                const bool f_up = __shfl_up_sync(FULL, flag, k);
+                if (lane >= k && !flag) {
+                    S += s_up;
+                    flag = f_up;
                 }
-                if (MODE == MODE_PULL) {
-                    // mask of Alg.1 l.20-25 / Alg.3 l.12-13: discovered iff the sum is non-zero
-                    const bool disc = fin && total > 0.0;
-                    const bool keep = fin && !(total > 0.0);
-                    int2 dg = make_int2(0, 0);
-                    if (disc) {
-                        P.depth[v] = d;
-                        P.sigma[v] = total;
-                        P.du[v] = 0.0;
-                        dg = P.deg2[v];
-                    }
-                    warp_append(disc, v, dg.x, lvl_out.ctr, P.ebits, lvl_out.v, lvl_out.pre, lvl_out.tiles,
-                                lvl_out.p0, lvl_out.e0);
-                    warp_add((unsigned long long)dg.y, &P.ctr->indeg_vis);
-                    warp_append(keep, v, keep ? (int64_t)ws.deg[j] : 0, cand_out.ctr, P.ebits, cand_out.v,
-                                cand_out.pre, cand_out.tiles, cand_out.p0, cand_out.e0);
-                } else if (fin) {
-                    // Alg.1 l.38-39 (delta = sigma * A delta_u), l.45 + P:180, then l.35 for level d
-                    const double sg = P.sigma[v];
-                    const double delta = sg * total;
-                    P.bc[v] += delta * P.bc_scale;
-                    const double dun = (1.0 + delta) / sg;
-                    P.du[v] = (d & 1) ? -dun : dun;
-                    P.sigma[v] = 0.0;
-                    P.depth[v] = -1;
-                }
+            }
+            const double S_prev = __shfl_up_sync(FULL, S, 1);
+            if (!single && head_o >= 0)
+                ws.val[head_o] = head_sum + ((lane > 0 && prev_tail == head_o) ? S_prev : 0.0);
+            const int next_head = __shfl_down_sync(FULL, head_o, 1);
+            if (tail_o >= 0 && (lane == 31 || next_head != tail_o)) ws.val[tail_o] = S;
+            __syncwarp();
+            // ---- hand each owner's sum to the owner pass
+            for (int j = lane; j < nwin; j += 32) {
+                const double t = ws.val[j];
+                if (t == 0.0) continue;
+                const bool whole = (j > 0 || start0) && (ps + j < pe);
+                if (whole) P.gacc[ws.v[j]] = t;
+                else atomicAdd(&P.gacc[ws.v[j]], t);
             }
         }
         __syncwarp();
     }
 }
 
+// ------------------------------------------------------------------ edge-stream pass
+//
+// The scCOOC form (Alg. 2; "less affected by load unbalance"): every stored
+// entry k of a format is visited, as the pair (owner own_arr[k], other end idx[k]), with two
+// 16-byte loads per lane for kLaneItems consecutive entries -- the whole edge array streams at
+// HBM rate with no owner window, and level filters decide which entries contribute:
+//   PUSH (CSR, owner u): u on level d-1 and x on level {-1, d}  -> sigma(x) += sigma(u), claims
+//   PULL (CSC, owner w): w undiscovered and x on level d-1 (fbm) -> acc(w) += sigma(x)
+//   BWD  (CSR, owner u): u on level L and x on level L+1 (bbm)   -> acc(u) += delta_u(x)
+// With owners sorted (CSC/CSR order) a lane's entries form owner runs, reduced in registers and
+// joined across lanes by one segmented scan; only the warp chunk's first and last owners can
+// continue into a neighbouring chunk and use an atomic.  Unsorted owners (the BWD / PUSH of a
+// directed COO^T graph, whose only format is column-major) use one atomic per contribution.
+template <int MODE>
+__device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const int32_t *__restrict__ own_arr,
+                                            const int32_t *__restrict__ idx, bool sorted, int d, int64_t gwarp,
+                                            int64_t nwarps, const ListOut &out) {
+    const int lane = threadIdx.x & 31;
+    const int64_t m = P.m;
+    const uint64_t pol = policy_evict_first();
+    const int owner_level = (MODE == MODE_PUSH) ? d - 1 : (MODE == MODE_PULL ? -1 : d);
+    for (int64_t base = gwarp * kWT; base < m; base += nwarps * kWT) {
+        const int64_t k0 = base + lane * kLaneItems;
+        int o[kLaneItems], x[kLaneItems];
+        if (k0 + kLaneItems <= m) {
+            const int4 a0 = ld_stream4(own_arr + k0, pol), a1 = ld_stream4(own_arr + k0 + 4, pol);
+            const int4 b0 = ld_stream4(idx + k0, pol), b1 = ld_stream4(idx + k0 + 4, pol);
+            o[0] = a0.x; o[1] = a0.y; o[2] = a0.z; o[3] = a0.w; o[4] = a1.x; o[5] = a1.y; o[6] = a1.z; o[7] = a1.w;
+            x[0] = b0.x; x[1] = b0.y; x[2] = b0.z; x[3] = b0.w; x[4] = b1.x; x[5] = b1.y; x[6] = b1.z; x[7] = b1.w;
+        } else {
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) {
+                const bool ok = k0 + i < m;
+                o[i] = ok ? own_arr[k0 + i] : -1;
+                x[i] = ok ? idx[k0 + i] : 0;
+            }
+        }
+        // owner filter, evaluated once per owner run
+        bool act[kLaneItems];
+        double osig[kLaneItems];
+        {
+            int last = -2;
+            bool last_ok = false;
+            double last_sig = 0.0;
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) {
+                if (o[i] != last) {
+                    last = o[i];
+                    last_ok = o[i] >= 0 && P.depth[o[i]] == owner_level;
+                    if (MODE == MODE_PUSH && last_ok) last_sig = P.sigma[o[i]];
+                }
+                act[i] = last_ok;
+                osig[i] = last_sig;
+            }
+        }
+        if (MODE == MODE_PUSH) {
+            int dxs[kLaneItems];
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) dxs[i] = act[i] ? P.depth[x[i]] : -2;
+            double olds[kLaneItems];
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) {
+                olds[i] = 1.0;
+                if (dxs[i] == -1 || dxs[i] == d) olds[i] = atomicAdd(&P.sigma[x[i]], osig[i]);
+            }
+            int cnt = 0;
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) {
+                const bool claim = olds[i] == 0.0;
+                const unsigned cm = __ballot_sync(FULL, claim);
+                if (claim) {
+                    const int32_t xv = x[i];
+                    P.depth[xv] = d;
+                    P.du[xv] = 0.0;
+                    bit_set(P.fbm[d & 1], xv);
+                    const int pos = cnt + __popc(cm & ((1u << lane) - 1u));
+                    ws.own[pos] = xv;
+                    ws.first[pos] = P.out_ptr ? (int32_t)(P.out_ptr[xv + 1] - P.out_ptr[xv]) : 0;
+                    ws.beg[pos] = P.out_ptr ? P.out_ptr[xv] : 0;
+                }
+                cnt += __popc(cm);
+            }
+            __syncwarp();
+            warp_flush(cnt, ws.own, ws.first, ws.beg, out, P.ebits);
+            __syncwarp();
+        } else {
+            double vals[kLaneItems];
+            const uint32_t *bm = (MODE == MODE_PULL) ? P.fbm[(d - 1) & 1] : P.bbm[(d + 1) & 1];
+            bool hit[kLaneItems];
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) hit[i] = act[i] && bit_test(bm, x[i]);
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) {
+                if (MODE == MODE_PULL) {
+                    vals[i] = hit[i] ? P.sigma[x[i]] : 0.0;
+                } else {
+                    const double u = hit[i] ? P.du[x[i]] : 0.0;
+                    const double want = ((d + 1) & 1) ? -u : u;
+                    vals[i] = want > 0.0 ? want : 0.0;
+                }
+            }
+            if (!sorted) {
+#pragma unroll
+                for (int i = 0; i < kLaneItems; ++i)
+                    if (vals[i] != 0.0) atomicAdd(&P.gacc[o[i]], vals[i]);
+                continue;
+            }
+            // owner runs of this lane (inactive owners contribute zeros)
+            int head_o = o[0], tail_o = o[0];
+            double head_sum = 0.0, run = 0.0;
+            bool single = true;
+            const int first_o = __shfl_sync(FULL, o[0], 0);
+            int last_valid = -1;
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) {
+                if (o[i] < 0) continue;
+                last_valid = o[i];
+                if (o[i] != tail_o) {
+                    if (single) head_sum = run;
+                    else if (run != 0.0) P.gacc[tail_o] = run;  // interior run: a whole owner
+                    single = false;
+                    run = 0.0;
+                    tail_o = o[i];
+                }
+                run += vals[i];
+            }
+            // the chunk's last owner: the last valid entry of the highest lane that has one
+            const unsigned vm = __ballot_sync(FULL, last_valid >= 0);
+            const int last_o = vm ? __shfl_sync(FULL, last_valid, 31 - __clz(vm)) : -1;
+            const int prev_tail = __shfl_up_sync(FULL, tail_o, 1);
+            bool flag = !(single && lane > 0 && prev_tail == tail_o && tail_o >= 0);
+            double S = run;
+#pragma unroll
+            for (int k = 1; k < 32; k <<= 1) {
+                const double s_up = __shfl_up_sync(FULL, S, k);
+                const bool f_up = __shfl_up_sync(FULL, flag, k);
+                if (lane >= k && !flag) {
+                    S += s_up;
+                    flag = f_up;
+                }
+            }
+            const double S_prev = __shfl_up_sync(FULL, S, 1);
+            const int next_head = __shfl_down_sync(FULL, head_o, 1);
+            if (!single && head_o >= 0) {
+                const double t = head_sum + ((lane > 0 && prev_tail == head_o) ? S_prev : 0.0);
+                if (t != 0.0) {
+                    if (head_o == first_o) atomicAdd(&P.gacc[head_o], t);
+                    else P.gacc[head_o] = t;
+                }
+            }
+            if (tail_o >= 0 && (lane == 31 || next_head != tail_o) && S != 0.0) {
+                if (tail_o == first_o || tail_o == last_o) atomicAdd(&P.gacc[tail_o], S);
+                else P.gacc[tail_o] = S;
+            }
+        }
+    }
+}
+
+// ------------------------------------------------------------------ owner passes
+
+// PULL owner pass over the candidate list: the mask of Alg.1 l.20-25 / Alg.3 l.12-13.
+// Discovered (sum > 0) -> depth = d, sigma = sum, appended to the level list; otherwise the
+// candidate survives into the next candidate list.  Chunks of kWT owners per warp.
+__device__ __forceinline__ void pull_owner_pass(const Params &P, WarpSmem &ws, const int32_t *cv, int64_t N, int d,
+                                                int64_t gwarp, int64_t nwarps, const ListOut &lvl_out,
+                                                const ListOut &cand_out) {
+    const int lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    for (int64_t base = gwarp * kWT; base < N; base += nwarps * kWT) {
+        int32_t vv[kLaneItems];
+        double tot[kLaneItems];
+#pragma unroll
+        for (int i = 0; i < kLaneItems; ++i) {
+            const int64_t p = base + i * 32 + lane;
+            vv[i] = p < N ? (cv ? cv[p] : (int32_t)p) : -1;
+            // static first pull (cv == nullptr): every undiscovered vertex with in-edges
+            if (!cv && vv[i] >= 0 && (P.depth[vv[i]] != -1 || P.deg2[vv[i]].y == 0)) vv[i] = -1;
+        }
+#pragma unroll
+        for (int i = 0; i < kLaneItems; ++i) tot[i] = vv[i] >= 0 ? P.gacc[vv[i]] : 0.0;
+        int nd = 0;
+#pragma unroll
+        for (int i = 0; i < kLaneItems; ++i) {
+            const bool disc = vv[i] >= 0 && tot[i] > 0.0;
+            const unsigned dm = __ballot_sync(FULL, disc);
+            if (disc) {
+                const int32_t v = vv[i];
+                P.gacc[v] = 0.0;
+                P.depth[v] = d;
+                P.sigma[v] = tot[i];
+                P.du[v] = 0.0;
+                bit_set(P.fbm[d & 1], v);
+                const int64_t b = P.out_ptr ? P.out_ptr[v] : 0;
+                const int pos = nd + __popc(dm & lt);
+                ws.own[pos] = v;
+                ws.first[pos] = P.out_ptr ? (int32_t)(P.out_ptr[v + 1] - b) : 0;
+                ws.beg[pos] = b;
+            }
+            nd += __popc(dm);
+        }
+        __syncwarp();
+        warp_flush(nd, ws.own, ws.first, ws.beg, lvl_out, P.ebits);
+        __syncwarp();
+        int nk = 0;
+#pragma unroll
+        for (int i = 0; i < kLaneItems; ++i) {
+            const bool keep = vv[i] >= 0 && !(tot[i] > 0.0);
+            const unsigned km = __ballot_sync(FULL, keep);
+            if (keep) {  // survivors: next candidate list, keyed by in-degree
+                const int32_t v = vv[i];
+                const int64_t b = P.in_ptr[v];
+                const int pos = nk + __popc(km & lt);
+                ws.own[pos] = v;
+                ws.first[pos] = (int32_t)(P.in_ptr[v + 1] - b);
+                ws.beg[pos] = b;
+            }
+            nk += __popc(km);
+        }
+        __syncwarp();
+        warp_flush(nk, ws.own, ws.first, ws.beg, cand_out, P.ebits);
+        __syncwarp();
+    }
+}
+
+// BWD owner pass over level L: Alg.1 l.38-39 (delta = sigma * A delta_u), l.45 with the 1/2
+// of P:180, then l.35 (delta_u for the level above), and the reset of the vertex.
+__device__ __forceinline__ void bwd_owner_pass(const Params &P, const int32_t *lv, int64_t N, int L, int64_t gtid,
+                                               int64_t nthreads) {
+    constexpr int U = 4;
+    for (int64_t base = gtid; base < N; base += U * nthreads) {
+        int32_t v[U];
+        double acc[U], sg[U], b[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t p = base + u * nthreads;
+            v[u] = p < N ? lv[p] : -1;
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            if (v[u] >= 0) {
+                acc[u] = P.gacc[v[u]];
+                sg[u] = P.sigma[v[u]];
+                b[u] = P.bc ? P.bc[v[u]] : 0.0;
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            if (v[u] < 0) continue;
+            const double delta = sg[u] * acc[u];
+            if (acc[u] != 0.0) {
+                P.gacc[v[u]] = 0.0;
+                P.bc[v[u]] = b[u] + delta * P.bc_scale;
+            }
+            const double dun = (1.0 + delta) / sg[u];
+            P.du[v[u]] = (L & 1) ? -dun : dun;
+            bit_set(P.bbm[L & 1], v[u]);
+            P.sigma[v[u]] = 0.0;
+            P.depth[v[u]] = -1;
+        }
+    }
+}
+
+// ------------------------------------------------------------------ trace
+
+// per-level timeline of one traced source (TBC_OPT_TRACE): {t_ns, kind, level, N, E, a, b, 0}
+enum { TR_INIT = 0, TR_SCAN = 1, TR_PUSH = 2, TR_PULL = 3, TR_BWD = 4, TR_OWNER = 5 };
+
+__device__ __forceinline__ void trace(const Params &P, bool on, int kind, int64_t level, int64_t N, int64_t E,
+                                      int64_t a, int64_t b) {
+    if (!on || blockIdx.x != 0 || threadIdx.x != 0) return;
+    const unsigned long long i = P.ctr->trace_n;
+    if ((int64_t)i >= P.trace_cap) return;
+    int64_t *t = P.trace + 8 * i;
+    t[0] = (int64_t)globaltimer_ns(); t[1] = kind; t[2] = level; t[3] = N; t[4] = E; t[5] = a; t[6] = b; t[7] = 0;
+    P.ctr->trace_n = i + 1;
+}
+
 // ------------------------------------------------------------------ the persistent kernel
 
-__global__ void __launch_bounds__(kBlock, 3) k_bc(Params P) {
+__global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
     extern __shared__ __align__(16) unsigned char dyn_smem[];
-    WarpSmem *smem = reinterpret_cast<WarpSmem *>(dyn_smem);
-    WarpSmem &ws = smem[threadIdx.x >> 5];
+    WarpSmem &ws = reinterpret_cast<WarpSmem *>(dyn_smem)[threadIdx.x >> 5];
     const int64_t nwarps = (int64_t)gridDim.x * kWarpsPerBlock;
     const int64_t gwarp = (int64_t)blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
     const int tid = threadIdx.x;
@@ -404,8 +697,15 @@ __global__ void __launch_bounds__(kBlock, 3) k_bc(Params P) {
             if (cta0 && tid == 0) atomicAdd(&C->bad_sources, 1ull);
             continue;
         }
+        const bool tr = (si == P.trace_src);
         // ---------------- init (Alg.1 l.7-10, l.15-18): depth(s)=0, sigma(s)=1, frontier={s}
         const int64_t dego = P.deg2[s].x;
+        for (int64_t w = gtid; w < P.nwords; w += nthreads) {
+            P.fbm[0][w] = 0u;
+            P.fbm[1][w] = 0u;
+            P.bbm[0][w] = 0u;
+            P.bbm[1][w] = 0u;
+        }
         if (cta0) {
             if (tid == 0) {
                 if (prev_s >= 0) {
@@ -417,15 +717,17 @@ __global__ void __launch_bounds__(kBlock, 3) k_bc(Params P) {
                 P.du[s] = 0.0;
                 P.list_v[0] = s;
                 P.list_pre[0] = 0;
+                P.list_beg[0] = P.out_ptr ? P.out_ptr[s] : 0;
                 C->list = (1ull << P.ebits) | (unsigned long long)dego;
-                C->indeg_vis = (unsigned long long)P.deg2[s].y;
                 C->cand[0] = 0;
                 C->cand[1] = 0;
+                if (tr) C->trace_n = 0;
             }
             for (int64_t i = tid; i <= dego / kWT; i += kBlock) P.tiles[i] = 0;
         }
         prev_s = s;
         grid_sync(C, gen);
+        trace(P, tr, TR_INIT, 0, 1, dego, s, 0);
 
         Level cur{0, 1, 0, dego, 0};  // level d-1 (frontier)
         int d = 1;
@@ -433,51 +735,58 @@ __global__ void __launch_bounds__(kBlock, 3) k_bc(Params P) {
         int cb = 0;
         int64_t candN = 0, candE = 0;
         int64_t fwd_edges = 0, pulls = 0, scans = 0;
+        // stream-pass arrays: (owner, other end) of every stored entry in the format each mode
+        // walks; a directed COO^T graph has only the column-major pairs (unsorted rows)
+        const bool coot_dir = P.coot && P.directed;
+        const int32_t *push_own = coot_dir ? P.in_idx : P.out_row;
+        const int32_t *push_idx = coot_dir ? P.in_col : P.out_idx;
         for (;;) {
             const int64_t ntiles_f = ceil_div(cur.N + cur.E, kWT);
             Level nxt{cur.p0 + cur.N, 0, cur.e0 + cur.E, 0, cur.tbase + ntiles_f};
-            // ---- direction (push cost = frontier out-edges, pull cost = in-edges
-            //      of the undiscovered candidates (+ a scan of n vertices to list them))
-            bool pull = false;
-            if (P.dir_mode == 2) {
-                pull = d >= 2;
-            } else if (P.dir_mode == 0 && d >= 2) {
-                const double pull_cost = cand_valid
-                    ? (double)candE
-                    : (double)(P.m - (int64_t)ld_volatile_u64(&C->indeg_vis)) + 0.25 * (double)P.n;
-                pull = P.alpha * pull_cost < (double)cur.E;
-            }
-            if (pull && !cand_valid) {
-                // candidate scan: undiscovered vertices with in-edges, in-degree prefix + tiles
-                AppendTarget ct{&C->cand[cb], P.cand_v[cb], P.cand_pre[cb], P.cand_tiles[cb], 0, 0};
-                for (int64_t base = gtid - (tid & 31); base < P.n; base += nthreads) {
-                    const int64_t v = base + (tid & 31);
-                    bool pr = false;
-                    int64_t ind = 0;
-                    if (v < P.n && P.depth[v] == -1) {
-                        ind = P.deg2[v].y;
-                        pr = ind > 0;
-                    }
-                    warp_append(pr, (int32_t)v, pr ? ind : 0, ct.ctr, P.ebits, ct.v, ct.pre, ct.tiles, 0, 0);
+            // ---- per-level choice: modelled cost of
+            //      push over the frontier list, push over all entries, pull over the survivors
+            //      of the previous pull, pull over all entries.  Pull needs d >= 2.
+            const double mE = (double)P.m;
+            double cost[4] = {(double)cur.E * (P.c_list + P.c_atom), mE * P.c_stream + (double)cur.E * P.c_atom,
+                              cand_valid ? (double)candE * P.c_list + (double)candN * P.c_vert : 1e300,
+                              mE * P.c_stream + (double)P.n * P.c_vert};
+            if (d < 2 || P.dir_mode == 1) cost[2] = cost[3] = 1e300;   // push only
+            if (d >= 2 && P.dir_mode == 2) cost[0] = cost[1] = 1e300;  // pull whenever possible
+            if (P.fmt_mode == 1 && !P.coot) cost[1] = cost[3] = 1e300; // list passes only
+            if (P.fmt_mode == 2 || P.coot) cost[0] = cost[2] = 1e300;  // edge streams only
+            int choice = 0;
+            for (int c = 1; c < 4; ++c)
+                if (cost[c] < cost[choice]) choice = c;
+            const bool pull = choice >= 2;
+            const ListOut lo{&C->list, P.list_v, P.list_pre, P.list_beg, P.tiles + nxt.tbase, nxt.p0, nxt.e0};
+            if (pull) {
+                const bool stream = choice == 3;
+                const ListOut co{&C->cand[cb ^ 1], P.cand_v[cb ^ 1], P.cand_pre[cb ^ 1], P.cand_beg[cb ^ 1],
+                                 P.cand_tiles[cb ^ 1], 0, 0};
+                if (stream) {
+                    stream_pass<MODE_PULL>(P, ws, P.in_col, P.in_idx, true, d, gwarp, nwarps, lo);
+                    candN = P.n;
+                    candE = P.m;
+                    ++scans;
+                } else {
+                    edge_pass<MODE_PULL>(P, ws, P.cand_v[cb], P.cand_pre[cb], P.cand_beg[cb], P.cand_tiles[cb], candN,
+                                         candE, 0, P.in_ptr, P.in_idx, d, gwarp, nwarps, lo);
                 }
                 grid_sync(C, gen);
-                const unsigned long long cv = ld_volatile_u64(&C->cand[cb]);
-                candN = (int64_t)(cv >> P.ebits);
-                candE = (int64_t)(cv & emask);
-                cand_valid = true;
-                ++scans;
-            }
-            AppendTarget lo{&C->list, P.list_v, P.list_pre, P.tiles + nxt.tbase, nxt.p0, nxt.e0};
-            if (pull) {
-                AppendTarget co{&C->cand[cb ^ 1], P.cand_v[cb ^ 1], P.cand_pre[cb ^ 1], P.cand_tiles[cb ^ 1], 0, 0};
-                level_pass<MODE_PULL>(P, ws, P.cand_v[cb], P.cand_pre[cb], P.cand_tiles[cb], candN, candE, 0,
-                                      P.in_ptr, P.in_idx, d, gwarp, nwarps, lo, co);
+                trace(P, tr, TR_PULL, d, candN, candE, stream, 0);
+                // owner pass: the survivors of a stream pull are all undiscovered vertices
+                pull_owner_pass(P, ws, stream ? nullptr : P.cand_v[cb], candN, d, gwarp, nwarps, lo, co);
                 fwd_edges += candE;
                 ++pulls;
+                cand_valid = !P.coot;
             } else {
-                level_pass<MODE_PUSH>(P, ws, P.list_v + cur.p0, P.list_pre + cur.p0, P.tiles + cur.tbase, cur.N,
-                                      cur.E, cur.e0, P.out_ptr, P.out_idx, d, gwarp, nwarps, lo, lo);
-                fwd_edges += cur.E;
+                if (choice == 1)
+                    stream_pass<MODE_PUSH>(P, ws, push_own, push_idx, !coot_dir, d, gwarp, nwarps, lo);
+                else
+                    edge_pass<MODE_PUSH>(P, ws, P.list_v + cur.p0, P.list_pre + cur.p0, P.list_beg + cur.p0,
+                                         P.tiles + cur.tbase, cur.N, cur.E, cur.e0, P.out_ptr, P.out_idx, d, gwarp,
+                                         nwarps, lo);
+                fwd_edges += choice == 1 ? P.m : cur.E;
                 if (cta0 && tid == 0) {
                     C->cand[0] = 0;  // candidate lists are stale after a push level
                     C->cand[1] = 0;
@@ -490,6 +799,7 @@ __global__ void __launch_bounds__(kBlock, 3) k_bc(Params P) {
                 nxt.N = (int64_t)(lv >> P.ebits) - nxt.p0;
                 nxt.E = (int64_t)(lv & emask) - nxt.e0;
             }
+            trace(P, tr, pull ? TR_OWNER : TR_PUSH, d, nxt.N, nxt.E, choice, pull ? candE : cur.E);
             if (pull) {
                 const unsigned long long cv = ld_volatile_u64(&C->cand[cb ^ 1]);
                 candN = (int64_t)(cv >> P.ebits);
@@ -508,8 +818,6 @@ __global__ void __launch_bounds__(kBlock, 3) k_bc(Params P) {
         }
         const int D = d - 1;  // height of the BFS tree (levels 0..D non-empty)
         if (cta0 && tid == 0) {
-            int64_t *l0 = P.lvl;
-            l0[0] = 0; l0[1] = 1; l0[2] = 0; l0[3] = dego; l0[4] = 0;
             C->st_sources += 1;
             C->st_reached += cur.p0 + cur.N;
             C->st_reached_edges += cur.e0 + cur.E;
@@ -521,7 +829,7 @@ __global__ void __launch_bounds__(kBlock, 3) k_bc(Params P) {
         }
         if (P.bfs_only) break;
 
-        // ---------------- backward (Alg.1 l.29-47): L = D (owner-only) down to 1
+        // ---------------- backward (Alg.1 l.29-47): L = D (owner pass only: delta = 0) .. 1
         int64_t bwd_edges = 0;
         for (int L = D; L >= 1; --L) {
             Level lv;
@@ -530,23 +838,22 @@ __global__ void __launch_bounds__(kBlock, 3) k_bc(Params P) {
             } else {
                 const int64_t *l = P.lvl + 5 * (int64_t)L;
                 lv = Level{l[0], l[1], l[2], l[3], l[4]};
+                const ListOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0};
+                const bool stream = P.coot || P.fmt_mode == 2 ||
+                                    (P.fmt_mode == 0 && (double)P.m * P.c_stream < (double)lv.E * P.c_list);
+                if (stream)
+                    stream_pass<MODE_BWD>(P, ws, push_own, push_idx, !coot_dir, L, gwarp, nwarps, none);
+                else
+                    edge_pass<MODE_BWD>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.list_beg + lv.p0,
+                                        P.tiles + lv.tbase, lv.N, lv.E, lv.e0, P.out_ptr, P.out_idx, L, gwarp, nwarps,
+                                        none);
+                bwd_edges += stream ? P.m : lv.E;
+                grid_sync(C, gen);
+                trace(P, tr, TR_BWD, L, lv.N, lv.E, 0, 0);
             }
-            if (L == D) {
-                // deepest level: delta = 0, so delta_u = 1/sigma (Alg.1 l.35) and bc += 0
-                for (int64_t i = gtid; i < lv.N; i += nthreads) {
-                    const int32_t v = P.list_v[lv.p0 + i];
-                    const double dun = 1.0 / P.sigma[v];
-                    P.du[v] = (L & 1) ? -dun : dun;
-                    P.sigma[v] = 0.0;
-                    P.depth[v] = -1;
-                }
-            } else {
-                AppendTarget none{nullptr, nullptr, nullptr, nullptr, 0, 0};
-                level_pass<MODE_BWD>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.tiles + lv.tbase, lv.N, lv.E,
-                                     lv.e0, P.out_ptr, P.out_idx, L, gwarp, nwarps, none, none);
-                bwd_edges += lv.E;
-            }
+            bwd_owner_pass(P, P.list_v + lv.p0, lv.N, L, gtid, nthreads);
             grid_sync(C, gen);
+            trace(P, tr, TR_OWNER, L, lv.N, lv.E, 1, 0);
         }
         if (cta0 && tid == 0) C->st_bwd_edges += bwd_edges;
     }
@@ -580,13 +887,19 @@ tbc_status engine_setup(tbc_graph *g) {
     const int64_t list_tiles = (n + m) / kWT + n + 2;
     const int64_t cand_tiles = (n + m) / kWT + 2;
     if ((e = alloc(&g->depth, n)) || (e = alloc(&g->sigma, n)) || (e = alloc(&g->du, n)) ||
-        (e = alloc(&g->gacc, n)) || (e = alloc(&g->gcnt, n)) || (e = alloc(&g->list_v, n + 1)) ||
-        (e = alloc(&g->list_pre, n + 1)) || (e = alloc(&g->tiles, list_tiles)) ||
-        (e = alloc(&g->lvl, 5 * (n + 2))) || (e = alloc(&g->ctr, 1)))
+        (e = alloc(&g->gacc, n)) || (e = alloc(&g->list_v, n + 1)) || (e = alloc(&g->list_pre, n + 1)) ||
+        (e = alloc(&g->list_beg, n + 1)) ||
+        (e = alloc(&g->tiles, list_tiles)) || (e = alloc(&g->lvl, 5 * (n + 2))) || (e = alloc(&g->ctr, 1)) ||
+        (e = alloc(&g->trace, 8 * kTraceCap)))
         return cuda_error(e, "workspace cudaMalloc");
-    if (g->engine == TBC_ENGINE_CSC) {
+    const int64_t nwords = (n + 31) / 32;
+    for (int b = 0; b < 2; ++b)
+        if ((e = alloc(&g->fbm[b], nwords)) || (e = alloc(&g->bbm[b], nwords)))
+            return cuda_error(e, "workspace cudaMalloc");
+    {
         for (int b = 0; b < 2; ++b)
             if ((e = alloc(&g->cand_v[b], n + 1)) || (e = alloc(&g->cand_pre[b], n + 1)) ||
+                (e = alloc(&g->cand_beg[b], n + 1)) ||
                 (e = alloc(&g->cand_tiles[b], cand_tiles)))
                 return cuda_error(e, "workspace cudaMalloc");
     }
@@ -594,7 +907,6 @@ tbc_status engine_setup(tbc_graph *g) {
         (e = cudaMemsetAsync(g->sigma, 0, sizeof(double) * n, s)) ||
         (e = cudaMemsetAsync(g->du, 0, sizeof(double) * n, s)) ||
         (e = cudaMemsetAsync(g->gacc, 0, sizeof(double) * n, s)) ||
-        (e = cudaMemsetAsync(g->gcnt, 0, sizeof(int32_t) * n, s)) ||
         (e = cudaMemsetAsync(g->ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s)))
         return cuda_error(e, "workspace init");
     int per_sm = 0, sms = 0;
@@ -609,8 +921,6 @@ tbc_status engine_setup(tbc_graph *g) {
 
 tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
                       int bfs_only) {
-    if (g->engine != TBC_ENGINE_CSC)
-        return set_error(TBC_ERR_UNSUPPORTED, "engine %d not available in this build", g->engine);
     Params P{};
     P.n = g->n;
     P.m = g->m;
@@ -623,13 +933,28 @@ tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
     P.sigma = g->sigma;
     P.du = g->du;
     P.gacc = g->gacc;
-    P.gcnt = g->gcnt;
     P.list_v = g->list_v;
     P.list_pre = g->list_pre;
+    P.list_beg = g->list_beg;
+    P.nwords = (g->n + 31) / 32;
+    for (int b = 0; b < 2; ++b) {
+        P.fbm[b] = g->fbm[b];
+        P.bbm[b] = g->bbm[b];
+    }
+    P.directed = g->directed;
+    P.coot = g->engine == TBC_ENGINE_COOT;
+    P.in_col = g->in_col;
+    P.out_row = g->out_row;
+    P.fmt_mode = g->fmt_mode;
+    P.c_list = g->c_list;
+    P.c_stream = g->c_stream;
+    P.c_atom = g->c_atom;
+    P.c_vert = g->c_vert;
     P.tiles = g->tiles;
     for (int b = 0; b < 2; ++b) {
         P.cand_v[b] = g->cand_v[b];
         P.cand_pre[b] = g->cand_pre[b];
+        P.cand_beg[b] = g->cand_beg[b];
         P.cand_tiles[b] = g->cand_tiles[b];
     }
     P.lvl = g->lvl;
@@ -641,9 +966,12 @@ tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
     P.ebits = g->ebits;
     P.bfs_only = bfs_only;
     P.dir_mode = g->dir_mode;
-    P.alpha = g->alpha;
+    P.trace = g->trace;
+    P.trace_cap = g->trace ? kTraceCap : 0;
+    P.trace_src = g->trace_src;
     void *args[] = {&P};
-    cudaError_t e = cudaLaunchCooperativeKernel((const void *)k_bc, dim3(g->grid), dim3(kBlock), args, kSmemBytes, stream);
+    cudaError_t e = cudaLaunchCooperativeKernel((const void *)k_bc, dim3(g->grid), dim3(kBlock), args, kSmemBytes,
+                                                stream);
     if (e != cudaSuccess) return cuda_error(e, "cudaLaunchCooperativeKernel(k_bc)");
     return TBC_OK;
 }

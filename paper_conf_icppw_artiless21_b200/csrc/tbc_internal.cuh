@@ -8,16 +8,17 @@
 
 namespace tbc {
 
-constexpr int kBlock = 256;  // threads per CTA of the persistent kernel
+constexpr int kBlock = 512;        // threads per CTA of the persistent kernel (one CTA per SM)
+constexpr int64_t kTraceCap = 65536; // trace entries (one per barrier of the traced source)
 
 // Device-side counters of one graph; all fields are touched by the persistent kernel only.
 struct Ctrs {
     unsigned long long list;      // packed (count << ebits) | edge_sum of the BFS-order list
-    unsigned long long indeg_vis; // sum of in-degrees of visited vertices (pull heuristic)
     unsigned long long cand[2];   // packed counters of the two pull-candidate buffers
     unsigned int bar_count;       // grid barrier arrival counter
     unsigned int bar_gen;         // grid barrier generation
     unsigned long long bad_sources;
+    unsigned long long trace_n;   // entries written to the trace buffer
     // accumulated statistics (tbc_stats)
     long long st_sources, st_reached, st_reached_edges, st_fwd_edges, st_bwd_edges, st_levels, st_pull_levels,
         st_scans, st_max_depth;
@@ -33,13 +34,17 @@ struct Params {
     int32_t *depth;                       // -1 unvisited
     double *sigma;                        // path counts, 0 when not on the current BFS
     double *du;                           // signed delta_u, sign = parity of the level
-    double *gacc;                         // split-owner partial sums (self-resetting)
-    int32_t *gcnt;                        // split-owner item counters (self-resetting)
+    double *gacc;                         // per-owner sums handed from edge to owner pass (0 between)
     int32_t *list_v;                      // BFS-order vertex list (levels concatenated)
     int64_t *list_pre;                    // exclusive out-degree prefix along list_v
+    int64_t *list_beg;                    // out_ptr[v] of each list entry (written at append)
+    uint32_t *fbm[2];                     // forward level bitmaps (level parity)
+    uint32_t *bbm[2];                     // backward level bitmaps (level parity)
+    int64_t nwords;                       // 32-bit words per bitmap
     int32_t *tiles;                       // per level: owner index starting each tile
     int32_t *cand_v[2];                   // pull candidate buffers
     int64_t *cand_pre[2];
+    int64_t *cand_beg[2];
     int32_t *cand_tiles[2];
     int64_t *lvl;                         // per level: p0, N, e0, E, tile_base
     Ctrs *ctr;
@@ -49,11 +54,16 @@ struct Params {
     double bc_scale;                      // 0.5 undirected, 1 directed
     int ebits;                            // low bits of packed counters hold edge sums
     int bfs_only;                         // forward stage only (tbc_bfs)
-    int dir_mode;                         // 0 auto, 1 push, 2 pull
-    double alpha;                         // pull when alpha*pull_cost < push_cost
-    // COO^T engine
-    const int32_t *coo_row;               // column-major (row, col) pairs = A's COOC arrays
-    const int32_t *coo_col;
+    int directed;
+    int coot;                             // TBC_ENGINE_COOT: edge-stream passes only
+    int dir_mode;                         // 0 auto, 1 push only, 2 pull whenever possible
+    int64_t *trace;                       // per-level timeline of one source (8 int64 per entry)
+    int64_t trace_cap, trace_src;
+    // edge-stream passes (the scCOOC form of Alg. 2): owner of every stored entry
+    const int32_t *__restrict__ in_col;   // column of each CSC entry (sorted)
+    const int32_t *__restrict__ out_row;  // row of each CSR entry (sorted); nullptr for COO^T directed
+    int fmt_mode;                         // 0 auto, 1 list passes only, 2 stream passes only
+    double c_list, c_stream, c_atom, c_vert;  // per-item cost model (ps) for the per-level choice
 };
 
 }  // namespace tbc
@@ -70,16 +80,20 @@ struct tbc_graph {
     int64_t *out_ptr = nullptr;  // aliases in_ptr when undirected
     int32_t *out_idx = nullptr;
     int2 *deg2 = nullptr;
-    int32_t *coo_col = nullptr;  // COO^T engine: column of each stored entry (rows = in_idx)
+    int32_t *in_col = nullptr;   // column (owner) of every CSC entry: with in_idx, the COOC arrays
+    int32_t *out_row = nullptr;  // row (owner) of every CSR entry (== in_col when undirected)
     // workspace (device)
     int32_t *depth = nullptr;
     double *sigma = nullptr, *du = nullptr, *gacc = nullptr;
-    int32_t *gcnt = nullptr;
     int32_t *list_v = nullptr;
     int64_t *list_pre = nullptr;
+    int64_t *list_beg = nullptr;
+    uint32_t *fbm[2] = {nullptr, nullptr};
+    uint32_t *bbm[2] = {nullptr, nullptr};
     int32_t *tiles = nullptr;
     int32_t *cand_v[2] = {nullptr, nullptr};
     int64_t *cand_pre[2] = {nullptr, nullptr};
+    int64_t *cand_beg[2] = {nullptr, nullptr};
     int32_t *cand_tiles[2] = {nullptr, nullptr};
     int64_t *lvl = nullptr;
     tbc::Ctrs *ctr = nullptr;
@@ -90,7 +104,10 @@ struct tbc_graph {
     int grid = 0;
     int ebits = 38;
     int dir_mode = 0;
-    double alpha = 1.0;
+    int fmt_mode = 0;
+    double c_list = 10.0, c_stream = 2.0, c_atom = 20.0, c_vert = 1.0;
+    int64_t *trace = nullptr;     // device, 8 * kTraceCap int64
+    int64_t trace_src = -1;       // index in the next call's source list to trace (-1: off)
     cudaStream_t stream = nullptr;  // internal stream for the synchronous host API
     size_t device_bytes = 0;
 };

@@ -13,7 +13,14 @@ import paper_conf_icppw_artiless21_b200 as tbc
 
 pytestmark = pytest.mark.gpu
 
-MODES = [tbc.DIR_AUTO, tbc.DIR_PUSH, tbc.DIR_PULL]
+# (direction, format) pairs: every forward/backward pass kind gets exercised
+MODES = [(tbc.DIR_AUTO, tbc.FMT_AUTO), (tbc.DIR_PUSH, tbc.FMT_LIST), (tbc.DIR_PUSH, tbc.FMT_STREAM),
+         (tbc.DIR_PULL, tbc.FMT_AUTO), (tbc.DIR_PULL, tbc.FMT_STREAM)]
+
+
+def set_mode(G, mode):
+    G.set_direction(mode[0])
+    G.set_format(mode[1])
 
 
 def assert_bc(got, want, rel=1e-9):
@@ -39,6 +46,9 @@ def gpu_graph(g, **kw):
     return tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, **kw)
 
 
+ENGINES = [tbc.ENGINE_CSC, tbc.ENGINE_COOT]
+
+
 # ------------------------------------------------------------------ closed forms / small graphs
 
 SMALL = [gg.star(7), gg.star(7, directed_both=True), gg.path(7), gg.path(7, directed=True), gg.cycle(8),
@@ -46,11 +56,12 @@ SMALL = [gg.star(7), gg.star(7, directed_both=True), gg.path(7), gg.path(7, dire
          gg.mycielski(6), gg.from_edges("one", 1, [], False), gg.from_edges("iso", 4, [(1, 2), (2, 3)], False)]
 
 
-@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("engine", ENGINES)
+@pytest.mark.parametrize("mode", MODES, ids=lambda m: f"dir{m[0]}fmt{m[1]}")
 @pytest.mark.parametrize("g", SMALL, ids=lambda g: g.name)
-def test_small_graphs_all_sources(g, mode):
-    with gpu_graph(g) as G:
-        G.set_direction(mode)
+def test_small_graphs_all_sources(g, mode, engine):
+    with gpu_graph(g, engine=engine) as G:
+        set_mode(G, mode)
         src = np.arange(g.n, dtype=np.int32)
         assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, g.directed, src))
         for s in range(min(g.n, 5)):
@@ -70,17 +81,20 @@ def test_random_small_graphs_many(directed):
         u, v = np.nonzero(A)
         g = gg.from_edges("r", n, np.stack([u, v], 1), directed)
         src = rng.integers(0, n, size=int(rng.integers(0, 2 * n))).astype(np.int32)
+        want = oracle.bc(g.col_ptr, g.row_idx, directed, src)
         with gpu_graph(g) as G:
             for mode in MODES:
-                G.set_direction(mode)
-                assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, directed, src))
+                set_mode(G, mode)
+                assert_bc(G.bc(src), want)
+        with gpu_graph(g, engine=tbc.ENGINE_COOT) as G:
+            assert_bc(G.bc(src), want)
 
 
 def test_grid_sigma_crosses_2_53():
     g = gg.grid(40, 40)
     with gpu_graph(g) as G:
         for mode in MODES:
-            G.set_direction(mode)
+            set_mode(G, mode)
             assert_bfs(g, G, 0)
             assert_bfs(g, G, 820)
 
@@ -93,7 +107,7 @@ def test_hub_spans_many_tiles(leaves):
     g = gg.star(leaves + 1)
     with gpu_graph(g) as G:
         for mode in MODES:
-            G.set_direction(mode)
+            set_mode(G, mode)
             src = np.array([0, 1, 2, leaves], dtype=np.int32)
             assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, False, src))
 
@@ -106,7 +120,7 @@ def test_double_star_and_directed_hubs():
     for gr in (g, h):
         with gpu_graph(gr) as G:
             for mode in MODES:
-                G.set_direction(mode)
+                set_mode(G, mode)
                 src = np.array([0, 1, 2, 3001, 6999], dtype=np.int32)
                 assert_bc(G.bc(src), oracle.bc(gr.col_ptr, gr.row_idx, gr.directed, src))
                 assert_bfs(gr, G, 2)
@@ -169,7 +183,7 @@ def test_cfg1_exact_bc_all_sources():
     want = oracle.bc(g.col_ptr, g.row_idx, False, src)
     with gpu_graph(g) as G:
         for mode in MODES:
-            G.set_direction(mode)
+            set_mode(G, mode)
             assert_bc(G.bc(src), want)
         for s in (0, 17, 1023):
             assert_bfs(g, G, s)
@@ -180,9 +194,12 @@ def test_kronecker_reduced_scale_full_oracle(scale, directed):
     g = gg.kronecker(scale, 16, seed=2, directed=directed, device="cuda")
     src = gg.sources(g, 256, seed=12)
     want = oracle.bc(g.col_ptr, g.row_idx, directed, src)
+    with gpu_graph(g, engine=tbc.ENGINE_COOT) as G:
+        assert_bc(G.bc(src), want)
+        assert_bfs(g, G, src[0])
     with gpu_graph(g) as G:
         for mode in MODES:
-            G.set_direction(mode)
+            set_mode(G, mode)
             assert_bc(G.bc(src), want)
         for s in src[:3]:
             assert_bfs(g, G, s)
@@ -199,11 +216,14 @@ def test_cfg2_rmat18_sample():
 
 
 def test_cfg3_kron22_directed_sample_in_bench_launch_config():
-    """Config 3 at full size (the bench workload), sampled sources, auto direction."""
+    """Config 3 at full size (the bench workload), sampled sources, auto choice; and COO^T."""
     g, src = gg.make_config(3, device="cuda")
     sample = src[:8]
+    want = oracle.bc(g.col_ptr, g.row_idx, True, sample)
+    with gpu_graph(g, engine=tbc.ENGINE_COOT) as G:
+        assert_bc(G.bc(sample[:3]), oracle.bc(g.col_ptr, g.row_idx, True, sample[:3]))
     with gpu_graph(g) as G:
-        assert_bc(G.bc(sample), oracle.bc(g.col_ptr, g.row_idx, True, sample))
+        assert_bc(G.bc(sample), want)
         for s in sample[:2]:
             assert_bfs(g, G, s)
         # per-source invariant at any size: sum_v bc_s(v) = sum_t (depth_s(t) - 1)

@@ -72,10 +72,10 @@ enum {
                                 recorded (-1 = off, default) */
     TBC_OPT_FORMAT = 4,      /* 0 auto (default), 1 list passes only, 2 edge streams only
                                 (TBC_ENGINE_COOT always streams) */
-    TBC_OPT_COST_LIST = 5,   /* cost model, picoseconds per item: list-pass item (default 10) */
-    TBC_OPT_COST_STREAM = 6, /*   stream-pass stored entry (default 2) */
-    TBC_OPT_COST_ATOMIC = 7, /*   push contribution (fp64 atomic) (default 20) */
-    TBC_OPT_COST_VERTEX = 8  /*   vertex of a whole-graph owner pass (default 1) */
+    TBC_OPT_COST_LIST = 5,   /* cost model, picoseconds per item: list-pass item (default 12) */
+    TBC_OPT_COST_STREAM = 6, /*   stream-pass stored entry (default 4) */
+    TBC_OPT_COST_ATOMIC = 7, /*   push contribution (fp64 atomic) (default 18) */
+    TBC_OPT_COST_VERTEX = 8  /*   vertex of a whole-graph owner pass (default 10) */
 };
 
 /* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since

@@ -121,6 +121,8 @@ __global__ void k_count_rows(int64_t m, const int32_t *__restrict__ rows, int2 *
         atomicAdd(&deg2[rows[i]].x, 1);
 }
 
+constexpr int64_t kPad = 16;  // entries of slack after every edge array (TMA bulk copies round up)
+
 inline int grid_for(int64_t work) {
     int64_t b = (work + 255) / 256;
     if (b < 1) b = 1;
@@ -206,8 +208,8 @@ tbc_status build_from_keys(tbc_graph *g, unsigned long long *d_keys, int64_t nnz
     g->m = m;
     // CSC of A (in-neighbours)
     TBC_CUDA(dmalloc(g, &g->in_ptr, g->n + 1));
-    TBC_CUDA(dmalloc(g, &g->in_idx, m));
-    TBC_CUDA(dmalloc(g, &g->in_col, m));  // column (owner) of every CSC entry: the COOC col_A
+    TBC_CUDA(dmalloc(g, &g->in_idx, m + kPad));  // +pad: 16-byte bulk copies of the last chunk
+    TBC_CUDA(dmalloc(g, &g->in_col, m + kPad));  // column (owner) of every CSC entry: the COOC col_A
     k_keys_to_ptr<<<grid_for(m > g->n ? m : g->n + 1), 256, 0, s>>>(g->n, m, d_keys, g->in_ptr,
                                                                    g->in_idx, g->in_col);
     TBC_CUDA(cudaGetLastError());
@@ -247,8 +249,8 @@ tbc_status build_from_keys(tbc_graph *g, unsigned long long *d_keys, int64_t nnz
             g->out_row = g->in_col;
         } else {
             TBC_CUDA(dmalloc(g, &g->out_ptr, g->n + 1));
-            TBC_CUDA(dmalloc(g, &g->out_idx, m));
-            TBC_CUDA(dmalloc(g, &g->out_row, m));
+            TBC_CUDA(dmalloc(g, &g->out_idx, m + kPad));
+            TBC_CUDA(dmalloc(g, &g->out_row, m + kPad));
             k_keys_to_ptr<<<grid_for(m > g->n ? m : g->n + 1), 256, 0, s>>>(g->n, m, tkeys, g->out_ptr,
                                                                            g->out_idx, g->out_row);
             TBC_CUDA(cudaGetLastError());

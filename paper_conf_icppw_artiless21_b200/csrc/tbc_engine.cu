@@ -28,6 +28,20 @@ namespace tbc {
 namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
+
+#ifdef TBC_DEBUG
+#define TBC_CHECK(cond, ...)                                                           \
+    do {                                                                               \
+        if (!(cond)) {                                                                 \
+            printf("TBC_CHECK failed %s:%d (%s) ", __FILE__, __LINE__, #cond);          \
+            printf(__VA_ARGS__);                                                       \
+            printf("\n");                                                              \
+            __trap();                                                                  \
+        }                                                                              \
+    } while (0)
+#else
+#define TBC_CHECK(cond, ...) ((void)0)
+#endif
 enum { MODE_PUSH = 0, MODE_PULL = 1, MODE_BWD = 2 };
 
 constexpr int kLaneItems = 8;          // items per lane per warp tile
@@ -67,13 +81,43 @@ __device__ __forceinline__ int ld_stream(const int32_t *ptr, uint64_t pol) {
     return v;
 }
 
-// 16-byte streaming read of graph arrays (read-only for the whole kernel), L2 evict-first
-__device__ __forceinline__ int4 ld_stream4(const int32_t *ptr, uint64_t pol) {
-    int4 v;
-    asm volatile("ld.global.nc.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
-                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(ptr), "l"(pol));
-    return v;
+// ---- TMA bulk copies (cp.async.bulk) completing on an mbarrier: the edge-stream pipeline
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
 }
+
+__device__ __forceinline__ void mbar_inval(uint64_t *bar) {
+    asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ bool mbar_try_wait(uint64_t *bar, unsigned parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+
+// global -> shared bulk copy (TMA), bytes a multiple of 16, both addresses 16-byte aligned
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, uint64_t *bar, uint64_t pol) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+        : "memory");
+}
+
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
 
 __device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned long long *p) {
     return *(volatile const unsigned long long *)p;
@@ -163,6 +207,7 @@ __device__ __forceinline__ void warp_flush(int c, const int32_t *bv, const int32
     int64_t e = (int64_t)(old & ((1ull << ebits) - 1ull)) + inc - sum;
     for (int i = lo; i < hi; ++i, ++p) {
         const int64_t dg = bd[i];
+        TBC_CHECK(bv[i] >= 0 && dg >= 0, "flush v %d dg %lld", bv[i], (long long)dg);
         o.v[p] = bv[i];
         o.pre[p] = e;
         o.beg[p] = bb[i];
@@ -170,6 +215,53 @@ __device__ __forceinline__ void warp_flush(int c, const int32_t *bv, const int32
         const int64_t k1 = k0 + dg;
         for (int64_t t = (k0 + kWT - 1) / kWT; t <= k1 / kWT; ++t) o.tiles[t] = (int32_t)(p - o.p0);
         e += dg;
+    }
+}
+
+// Register variant of warp_flush for up to kLaneItems appends per lane (no shared memory): a
+// warp scan of the lanes' counts and degree sums gives every lane its consecutive slots.
+__device__ __forceinline__ void warp_flush_regs(const bool (&take)[kLaneItems], const int32_t (&v)[kLaneItems],
+                                                const int32_t (&dg)[kLaneItems], const int64_t (&bg)[kLaneItems],
+                                                const ListOut &o, int ebits) {
+    const int lane = threadIdx.x & 31;
+    int c = 0;
+    int64_t sum = 0;
+#pragma unroll
+    for (int i = 0; i < kLaneItems; ++i)
+        if (take[i]) {
+            ++c;
+            sum += dg[i];
+        }
+    if (!__any_sync(FULL, c > 0)) return;
+    int cinc = c;
+    int64_t inc = sum;
+#pragma unroll
+    for (int k = 1; k < 32; k <<= 1) {
+        const int tc = __shfl_up_sync(FULL, cinc, k);
+        const int64_t t = __shfl_up_sync(FULL, inc, k);
+        if (lane >= k) {
+            cinc += tc;
+            inc += t;
+        }
+    }
+    const int ctot = __shfl_sync(FULL, cinc, 31);
+    const int64_t tot = __shfl_sync(FULL, inc, 31);
+    unsigned long long old = 0;
+    if (lane == 0) old = atomicAdd(o.ctr, ((unsigned long long)ctot << ebits) + (unsigned long long)tot);
+    old = __shfl_sync(FULL, old, 0);
+    int64_t p = (int64_t)(old >> ebits) + cinc - c;
+    int64_t e = (int64_t)(old & ((1ull << ebits) - 1ull)) + inc - sum;
+#pragma unroll
+    for (int i = 0; i < kLaneItems; ++i) {
+        if (!take[i]) continue;
+        o.v[p] = v[i];
+        o.pre[p] = e;
+        o.beg[p] = bg[i];
+        const int64_t k0 = (e - o.e0) + (p - o.p0);
+        const int64_t k1 = k0 + dg[i];
+        for (int64_t t = (k0 + kWT - 1) / kWT; t <= k1 / kWT; ++t) o.tiles[t] = (int32_t)(p - o.p0);
+        e += dg[i];
+        ++p;
     }
 }
 
@@ -215,6 +307,9 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
         const int64_t es = ks - ps, ee = ke - pe;
         const int nwin = (int)(min(pe, N - 1) - ps + 1);
         const int ne = (int)(ee - es);
+        TBC_CHECK(nwin >= 1 && nwin <= kWT + 1 && ne >= 0 && ne <= kWT && ps >= 0 && pe <= N && ps <= pe,
+                  "mode %d tile %lld/%lld N %lld E %lld ps %lld pe %lld nwin %d ne %d", MODE, (long long)tile,
+                  (long long)ntiles, (long long)N, (long long)E, (long long)ps, (long long)pe, nwin, ne);
 
         // ---- owner window (three coalesced list reads): first in-tile slot, its adjacency position
         bool start0 = true;
@@ -222,6 +317,8 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
             const int64_t pre = opre[ps + j] - e0;
             const int64_t f = max(pre, es);
             const int32_t v = ov[ps + j];
+            TBC_CHECK(v >= 0 && v < P.n && f - es >= 0 && f - es <= kWT, "mode %d v %d f-es %lld", MODE, v,
+                      (long long)(f - es));
             ws.first[j] = (int32_t)(f - es);
             ws.beg[j] = obeg[ps + j] + (f - pre);
             ws.v[j] = v;
@@ -275,8 +372,11 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
             xs[i] = 0;
             if (sl < ne) {
                 const int j = ws.own[sl];
+                TBC_CHECK(j >= 0 && j < nwin, "mode %d own %d nwin %d sl %d", MODE, j, nwin, sl);
                 js[i] = j;
                 xs[i] = ld_stream(adj_idx + ws.beg[j] + (sl - ws.first[j]), pol_stream);
+                TBC_CHECK(xs[i] >= 0 && xs[i] < P.n, "mode %d x %d pos %lld", MODE, xs[i],
+                          (long long)(ws.beg[j] + (sl - ws.first[j])));
             }
         }
         if (MODE == MODE_PUSH) {
@@ -409,6 +509,14 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
 // joined across lanes by one segmented scan; only the warp chunk's first and last owners can
 // continue into a neighbouring chunk and use an atomic.  Unsorted owners (the BWD / PUSH of a
 // directed COO^T graph, whose only format is column-major) use one atomic per contribution.
+constexpr int kStages = 3;  // TMA stages per warp (2 chunks in flight while one is processed)
+
+struct StreamStage {
+    int32_t own[kWT];
+    int32_t idx[kWT];
+};
+static_assert(sizeof(StreamStage) * kStages + 8 * kStages <= sizeof(WarpSmem), "stream stages fit the warp slice");
+
 template <int MODE>
 __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const int32_t *__restrict__ own_arr,
                                             const int32_t *__restrict__ idx, bool sorted, int d, int64_t gwarp,
@@ -417,37 +525,94 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
     const int64_t m = P.m;
     const uint64_t pol = policy_evict_first();
     const int owner_level = (MODE == MODE_PUSH) ? d - 1 : (MODE == MODE_PULL ? -1 : d);
-    for (int64_t base = gwarp * kWT; base < m; base += nwarps * kWT) {
+    // this warp's chunks: gwarp, gwarp + nwarps, ...; the warp slice of smem becomes kStages
+    // stages of (owners, other ends), filled by lane 0 with two bulk copies per chunk
+    StreamStage *stage = reinterpret_cast<StreamStage *>(&ws);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(reinterpret_cast<unsigned char *>(&ws) + sizeof(StreamStage) * kStages);
+    const int64_t nchunks = ceil_div(m, kWT);
+    const int64_t mine = gwarp < nchunks ? (nchunks - 1 - gwarp) / nwarps + 1 : 0;
+    if (mine == 0) return;
+    __syncwarp();  // every lane is done with the previous contents of the warp slice
+    auto issue = [&](int64_t j) {  // lane 0 only
+        const int st = (int)(j % kStages);
+        const int64_t base = (gwarp + j * nwarps) * kWT;
+        const unsigned bytes = (unsigned)((min((int64_t)kWT, m - base) * 4 + 15) & ~15);
+        mbar_arrive_expect_tx(&bar[st], 2 * bytes);
+        bulk_g2s(stage[st].own, own_arr + base, bytes, &bar[st], pol);
+        bulk_g2s(stage[st].idx, idx + base, bytes, &bar[st], pol);
+    };
+    auto wait_stage = [&](int64_t j) {
+        const unsigned long long t0 = globaltimer_ns();
+        while (!mbar_try_wait(&bar[j % kStages], (unsigned)((j / kStages) & 1)))
+            if (globaltimer_ns() - t0 > kWatchdogNs) __trap();
+    };
+    // owner filter data of a chunk, loaded one chunk ahead: the depth of every owner run's owner
+    // (one load per run; entries repeating the previous owner get kSame)
+    constexpr int kSame = -7;
+    const uint32_t *tbm = (MODE == MODE_PULL) ? P.fbm[(d - 1) & 1] : (MODE == MODE_BWD ? P.bbm[(d + 1) & 1] : nullptr);
+    int od[kLaneItems];
+    auto prefetch = [&](int64_t j, int (&odv)[kLaneItems]) {
+        const int st = (int)(j % kStages);
+        const int64_t kb = (gwarp + j * nwarps) * kWT + lane * kLaneItems;
+        const int4 *so = reinterpret_cast<const int4 *>(stage[st].own + lane * kLaneItems);
+        const int4 a0 = so[0], a1 = so[1];
+        const int oo[kLaneItems] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+#pragma unroll
+        for (int i = 0; i < kLaneItems; ++i) {
+            const bool ok = kb + i < m;
+            odv[i] = !ok ? -3 : ((i > 0 && oo[i] == oo[i - 1]) ? kSame : P.depth[oo[i]]);
+        }
+    };
+    if (lane == 0) {
+        for (int st = 0; st < kStages; ++st) mbar_init(&bar[st], 1);
+        fence_mbar_init();
+        fence_proxy_async();
+        for (int64_t j = 0; j < min((int64_t)kStages, mine); ++j) issue(j);
+    }
+    __syncwarp();
+    wait_stage(0);
+    prefetch(0, od);
+    for (int64_t j = 0; j < mine; ++j) {
+        const int st = (int)(j % kStages);
+        const int64_t base = (gwarp + j * nwarps) * kWT;
         const int64_t k0 = base + lane * kLaneItems;
         int o[kLaneItems], x[kLaneItems];
-        if (k0 + kLaneItems <= m) {
-            const int4 a0 = ld_stream4(own_arr + k0, pol), a1 = ld_stream4(own_arr + k0 + 4, pol);
-            const int4 b0 = ld_stream4(idx + k0, pol), b1 = ld_stream4(idx + k0 + 4, pol);
+        {
+            const int4 *so = reinterpret_cast<const int4 *>(stage[st].own + lane * kLaneItems);
+            const int4 *sx = reinterpret_cast<const int4 *>(stage[st].idx + lane * kLaneItems);
+            const int4 a0 = so[0], a1 = so[1], b0 = sx[0], b1 = sx[1];
             o[0] = a0.x; o[1] = a0.y; o[2] = a0.z; o[3] = a0.w; o[4] = a1.x; o[5] = a1.y; o[6] = a1.z; o[7] = a1.w;
             x[0] = b0.x; x[1] = b0.y; x[2] = b0.z; x[3] = b0.w; x[4] = b1.x; x[5] = b1.y; x[6] = b1.z; x[7] = b1.w;
-        } else {
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
-                const bool ok = k0 + i < m;
-                o[i] = ok ? own_arr[k0 + i] : -1;
-                x[i] = ok ? idx[k0 + i] : 0;
+                if (k0 + i >= m) o[i] = -1;
+                TBC_CHECK(o[i] < 0 || (o[i] < P.n && x[i] >= 0 && x[i] < P.n), "stream mode %d k %lld o %d x %d",
+                          MODE, (long long)(k0 + i), o[i], x[i]);
             }
         }
-        // owner filter, evaluated once per owner run
+        int od_n[kLaneItems];
+        if (j + 1 < mine) {
+            wait_stage(j + 1);
+            prefetch(j + 1, od_n);
+        }
+        __syncwarp();  // stage st fully read: refill it with chunk j + kStages
+        if (lane == 0 && j + kStages < mine) {
+            fence_proxy_async();  // order our generic reads of the stage before the async refill
+            issue(j + kStages);
+        }
+        // owner filter (from the prefetched owner depths)
         bool act[kLaneItems];
         double osig[kLaneItems];
         {
-            int last = -2;
-            bool last_ok = false;
+            int dep = -3;
             double last_sig = 0.0;
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
-                if (o[i] != last) {
-                    last = o[i];
-                    last_ok = o[i] >= 0 && P.depth[o[i]] == owner_level;
-                    if (MODE == MODE_PUSH && last_ok) last_sig = P.sigma[o[i]];
+                if (od[i] != kSame) {
+                    dep = od[i];
+                    if (MODE == MODE_PUSH && dep == owner_level) last_sig = P.sigma[o[i]];
                 }
-                act[i] = last_ok;
+                act[i] = o[i] >= 0 && dep == owner_level;
                 osig[i] = last_sig;
             }
         }
@@ -461,32 +626,31 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
                 olds[i] = 1.0;
                 if (dxs[i] == -1 || dxs[i] == d) olds[i] = atomicAdd(&P.sigma[x[i]], osig[i]);
             }
-            int cnt = 0;
+            bool claim[kLaneItems];
+            int32_t cdg[kLaneItems];
+            int64_t cbg[kLaneItems];
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
-                const bool claim = olds[i] == 0.0;
-                const unsigned cm = __ballot_sync(FULL, claim);
-                if (claim) {
+                claim[i] = olds[i] == 0.0;
+                cdg[i] = 0;
+                cbg[i] = 0;
+                if (claim[i]) {
                     const int32_t xv = x[i];
                     P.depth[xv] = d;
                     P.du[xv] = 0.0;
                     bit_set(P.fbm[d & 1], xv);
-                    const int pos = cnt + __popc(cm & ((1u << lane) - 1u));
-                    ws.own[pos] = xv;
-                    ws.first[pos] = P.out_ptr ? (int32_t)(P.out_ptr[xv + 1] - P.out_ptr[xv]) : 0;
-                    ws.beg[pos] = P.out_ptr ? P.out_ptr[xv] : 0;
+                    if (P.out_ptr) {
+                        cbg[i] = P.out_ptr[xv];
+                        cdg[i] = (int32_t)(P.out_ptr[xv + 1] - cbg[i]);
+                    }
                 }
-                cnt += __popc(cm);
             }
-            __syncwarp();
-            warp_flush(cnt, ws.own, ws.first, ws.beg, out, P.ebits);
-            __syncwarp();
+            warp_flush_regs(claim, x, cdg, cbg, out, P.ebits);
         } else {
             double vals[kLaneItems];
-            const uint32_t *bm = (MODE == MODE_PULL) ? P.fbm[(d - 1) & 1] : P.bbm[(d + 1) & 1];
             bool hit[kLaneItems];
 #pragma unroll
-            for (int i = 0; i < kLaneItems; ++i) hit[i] = act[i] && bit_test(bm, x[i]);
+            for (int i = 0; i < kLaneItems; ++i) hit[i] = act[i] && bit_test(tbm, x[i]);
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
                 if (MODE == MODE_PULL) {
@@ -501,8 +665,7 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
 #pragma unroll
                 for (int i = 0; i < kLaneItems; ++i)
                     if (vals[i] != 0.0) atomicAdd(&P.gacc[o[i]], vals[i]);
-                continue;
-            }
+            } else {
             // owner runs of this lane (inactive owners contribute zeros)
             int head_o = o[0], tail_o = o[0];
             double head_sum = 0.0, run = 0.0;
@@ -550,8 +713,15 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
                 if (tail_o == first_o || tail_o == last_o) atomicAdd(&P.gacc[tail_o], S);
                 else P.gacc[tail_o] = S;
             }
+            }
         }
+#pragma unroll
+        for (int i = 0; i < kLaneItems; ++i) od[i] = od_n[i];
     }
+    __syncwarp();
+    if (lane == 0)
+        for (int st = 0; st < kStages; ++st) mbar_inval(&bar[st]);
+    __syncwarp();
 }
 
 // ------------------------------------------------------------------ owner passes
@@ -575,7 +745,10 @@ __device__ __forceinline__ void pull_owner_pass(const Params &P, WarpSmem &ws, c
             if (!cv && vv[i] >= 0 && (P.depth[vv[i]] != -1 || P.deg2[vv[i]].y == 0)) vv[i] = -1;
         }
 #pragma unroll
-        for (int i = 0; i < kLaneItems; ++i) tot[i] = vv[i] >= 0 ? P.gacc[vv[i]] : 0.0;
+        for (int i = 0; i < kLaneItems; ++i) {
+            TBC_CHECK(vv[i] < P.n, "pull owner v %d", vv[i]);
+            tot[i] = vv[i] >= 0 ? P.gacc[vv[i]] : 0.0;
+        }
         int nd = 0;
 #pragma unroll
         for (int i = 0; i < kLaneItems; ++i) {
@@ -632,6 +805,8 @@ __device__ __forceinline__ void bwd_owner_pass(const Params &P, const int32_t *l
         for (int u = 0; u < U; ++u) {
             const int64_t p = base + u * nthreads;
             v[u] = p < N ? lv[p] : -1;
+            TBC_CHECK(v[u] < P.n && (p >= N || v[u] >= 0), "bwd owner v %d p %lld N %lld", v[u], (long long)p,
+                      (long long)N);
         }
 #pragma unroll
         for (int u = 0; u < U; ++u) {

@@ -105,7 +105,7 @@ struct tbc_graph {
     int ebits = 38;
     int dir_mode = 0;
     int fmt_mode = 0;
-    double c_list = 10.0, c_stream = 2.0, c_atom = 20.0, c_vert = 1.0;
+    double c_list = 12.0, c_stream = 4.0, c_atom = 18.0, c_vert = 10.0;
     int64_t *trace = nullptr;     // device, 8 * kTraceCap int64
     int64_t trace_src = -1;       // index in the next call's source list to trace (-1: off)
     cudaStream_t stream = nullptr;  // internal stream for the synchronous host API

@@ -57,7 +57,8 @@ def lib():
     """Load libturbobc.so (building it in-tree first if the sources are newer)."""
     global _LIB
     if _LIB is None:
-        path = _build.build(debug=os.environ.get("TBC_DEBUG_LIB") == "1")
+        path = _build.build(debug=os.environ.get("TBC_DEBUG_LIB") == "1",
+                            variant=os.environ.get("TBC_VARIANT", ""))
         L = ctypes.CDLL(path)
         i64, i32, P = ctypes.c_int64, ctypes.c_int32, ctypes.POINTER
         vp = ctypes.c_void_p

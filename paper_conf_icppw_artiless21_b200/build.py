@@ -31,13 +31,19 @@ def _stale(lib=LIB) -> bool:
     return any(os.path.getmtime(p) > t for p in deps)
 
 
-def build(force: bool = False, verbose: bool = False, debug: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, debug: bool = False, variant: str = "") -> str:
+    """variant: extra -D flags for tuning experiments (e.g. "-DTBC_BLOCK=1024 -DTBC_LANE_ITEMS=4"),
+    built as libturbobc_<hash>.so next to the default library."""
     lib = LIB_DEBUG if debug else LIB
+    vflags = variant.split()
+    if vflags:
+        import hashlib
+        lib = os.path.join(PKG, "libturbobc_" + hashlib.sha1(variant.encode()).hexdigest()[:8] + ".so")
     if not force and not _stale(lib):
         return lib
     tmp = lib + f".tmp{os.getpid()}"
     cmd = [nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
-           *(["-DTBC_DEBUG"] if debug else []),
+           *(["-DTBC_DEBUG"] if debug else []), *vflags,
            "-Xptxas", "-v" if verbose else "-O3", f"-I{os.path.join(ROOT, 'include')}",
            "-o", tmp] + [os.path.join(CSRC, f) for f in SOURCES]
     res = subprocess.run(cmd, capture_output=True, text=True)

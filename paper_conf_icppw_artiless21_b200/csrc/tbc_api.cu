@@ -159,8 +159,6 @@ void free_graph(tbc_graph *g) {
     cudaFree(g->list_beg);
     cudaFree(g->tiles);
     for (int b = 0; b < 2; ++b) {
-        cudaFree(g->fbm[b]);
-        cudaFree(g->bbm[b]);
         cudaFree(g->cand_v[b]);
         cudaFree(g->cand_pre[b]);
         cudaFree(g->cand_beg[b]);

@@ -44,7 +44,7 @@ constexpr unsigned FULL = 0xffffffffu;
 #endif
 enum { MODE_PUSH = 0, MODE_PULL = 1, MODE_BWD = 2 };
 
-constexpr int kLaneItems = 8;          // items per lane per warp tile
+constexpr int kLaneItems = TBC_LANE_ITEMS;  // items per lane per warp tile
 constexpr int kWT = 32 * kLaneItems;   // diagonal items per warp tile
 constexpr int kWarpsPerBlock = kBlock / 32;
 
@@ -156,17 +156,6 @@ __device__ __forceinline__ void grid_sync(Ctrs *c, unsigned &gen) {
     gen += 1;
     __syncthreads();
 }
-
-// ------------------------------------------------------------------ level bitmaps
-// fbm[d&1]: vertices discovered on level d (forward); bbm[L&1]: vertices of level L whose
-// delta_u is final (backward).  Cleared per source.  Within a source they are exact filters:
-// the in-neighbours of a still-undiscovered vertex lie on level d-1 or are undiscovered, and
-// the out-neighbours of a level-L vertex lie on levels <= L+1, so the same-parity levels that
-// share a bitmap never meet the test.  A 0.5 MB bitmap (scale 22) stays in L2, so the 8 B
-// gathers of sigma / delta_u from the 33 MB arrays happen only for real contributions.
-
-__device__ __forceinline__ bool bit_test(const uint32_t *bm, int32_t x) { return (bm[x >> 5] >> (x & 31)) & 1u; }
-__device__ __forceinline__ void bit_set(uint32_t *bm, int32_t x) { atomicOr(&bm[x >> 5], 1u << (x & 31)); }
 
 // ------------------------------------------------------------------ warp-aggregated append
 
@@ -402,7 +391,6 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
                     const int32_t x = xs[i];
                     P.depth[x] = d;
                     P.du[x] = 0.0;
-                    bit_set(P.fbm[d & 1], x);
                     const int64_t b = adj_ptr[x];
                     const int64_t dg = adj_ptr[x + 1] - b;
                     const int pos = cnt + __popc(cm & ((1u << lane) - 1u));
@@ -417,23 +405,17 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
         } else {
             double vals[kLaneItems];
             if (MODE == MODE_PULL) {
-                // f_t(w) = sum over in-neighbours x on level d-1 of sigma(x)   (Alg.3 l.9-11)
-                const uint32_t *front = P.fbm[(d - 1) & 1];
-                bool hit[kLaneItems];
+                // f_t(w) = sum over in-neighbours x of sigma(x) (Alg.3 l.9-11).  No level test: an
+                // in-neighbour of a still-undiscovered w is on level d-1 or undiscovered (sigma = 0),
+                // so sigma itself is the masked frontier vector f.
 #pragma unroll
-                for (int i = 0; i < kLaneItems; ++i) hit[i] = js[i] >= 0 && bit_test(front, xs[i]);
-#pragma unroll
-                for (int i = 0; i < kLaneItems; ++i) vals[i] = hit[i] ? P.sigma[xs[i]] : 0.0;
+                for (int i = 0; i < kLaneItems; ++i) vals[i] = js[i] >= 0 ? P.sigma[xs[i]] : 0.0;
             } else {
                 // (A delta_u)(v): out-neighbour x on level d+1.  The level parity is the sign of
                 // the stored delta_u, so neighbours on other levels contribute exactly 0.
-                const uint32_t *below = P.bbm[(d + 1) & 1];
-                bool hit[kLaneItems];
-#pragma unroll
-                for (int i = 0; i < kLaneItems; ++i) hit[i] = js[i] >= 0 && bit_test(below, xs[i]);
 #pragma unroll
                 for (int i = 0; i < kLaneItems; ++i) {
-                    const double u = hit[i] ? P.du[xs[i]] : 0.0;
+                    const double u = js[i] >= 0 ? P.du[xs[i]] : 0.0;
                     const double want = ((d + 1) & 1) ? -u : u;
                     vals[i] = want > 0.0 ? want : 0.0;
                 }
@@ -503,13 +485,28 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
 // 16-byte loads per lane for kLaneItems consecutive entries -- the whole edge array streams at
 // HBM rate with no owner window, and level filters decide which entries contribute:
 //   PUSH (CSR, owner u): u on level d-1 and x on level {-1, d}  -> sigma(x) += sigma(u), claims
-//   PULL (CSC, owner w): w undiscovered and x on level d-1 (fbm) -> acc(w) += sigma(x)
-//   BWD  (CSR, owner u): u on level L and x on level L+1 (bbm)   -> acc(u) += delta_u(x)
+//   PULL (CSC, owner w): w undiscovered                    -> acc(w) += sigma(x)
+//   BWD  (CSR, owner u): u on level L                       -> acc(u) += delta_u(x) of parity L+1
+// (an undiscovered vertex's in-neighbours are on level d-1 or undiscovered with sigma = 0; a
+// level-L vertex's out-neighbours are on levels <= L+1, and only level L+1 holds delta_u of
+// parity L+1 -- so no per-entry level test is needed on the target side)
 // With owners sorted (CSC/CSR order) a lane's entries form owner runs, reduced in registers and
 // joined across lanes by one segmented scan; only the warp chunk's first and last owners can
 // continue into a neighbouring chunk and use an atomic.  Unsorted owners (the BWD / PUSH of a
 // directed COO^T graph, whose only format is column-major) use one atomic per contribution.
 constexpr int kStages = 3;  // TMA stages per warp (2 chunks in flight while one is processed)
+
+// a lane's kLaneItems consecutive int32 of a stage, as 16-byte shared-memory loads
+__device__ __forceinline__ void load_lane_items(const int4 *src, int (&dst)[kLaneItems]) {
+#pragma unroll
+    for (int q = 0; q < kLaneItems / 4; ++q) {
+        const int4 a = src[q];
+        dst[4 * q] = a.x;
+        dst[4 * q + 1] = a.y;
+        dst[4 * q + 2] = a.z;
+        dst[4 * q + 3] = a.w;
+    }
+}
 
 struct StreamStage {
     int32_t own[kWT];
@@ -549,14 +546,13 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
     // owner filter data of a chunk, loaded one chunk ahead: the depth of every owner run's owner
     // (one load per run; entries repeating the previous owner get kSame)
     constexpr int kSame = -7;
-    const uint32_t *tbm = (MODE == MODE_PULL) ? P.fbm[(d - 1) & 1] : (MODE == MODE_BWD ? P.bbm[(d + 1) & 1] : nullptr);
     int od[kLaneItems];
     auto prefetch = [&](int64_t j, int (&odv)[kLaneItems]) {
         const int st = (int)(j % kStages);
         const int64_t kb = (gwarp + j * nwarps) * kWT + lane * kLaneItems;
         const int4 *so = reinterpret_cast<const int4 *>(stage[st].own + lane * kLaneItems);
-        const int4 a0 = so[0], a1 = so[1];
-        const int oo[kLaneItems] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+        int oo[kLaneItems];
+        load_lane_items(so, oo);
 #pragma unroll
         for (int i = 0; i < kLaneItems; ++i) {
             const bool ok = kb + i < m;
@@ -580,9 +576,8 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
         {
             const int4 *so = reinterpret_cast<const int4 *>(stage[st].own + lane * kLaneItems);
             const int4 *sx = reinterpret_cast<const int4 *>(stage[st].idx + lane * kLaneItems);
-            const int4 a0 = so[0], a1 = so[1], b0 = sx[0], b1 = sx[1];
-            o[0] = a0.x; o[1] = a0.y; o[2] = a0.z; o[3] = a0.w; o[4] = a1.x; o[5] = a1.y; o[6] = a1.z; o[7] = a1.w;
-            x[0] = b0.x; x[1] = b0.y; x[2] = b0.z; x[3] = b0.w; x[4] = b1.x; x[5] = b1.y; x[6] = b1.z; x[7] = b1.w;
+            load_lane_items(so, o);
+            load_lane_items(sx, x);
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
                 if (k0 + i >= m) o[i] = -1;
@@ -638,7 +633,6 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
                     const int32_t xv = x[i];
                     P.depth[xv] = d;
                     P.du[xv] = 0.0;
-                    bit_set(P.fbm[d & 1], xv);
                     if (P.out_ptr) {
                         cbg[i] = P.out_ptr[xv];
                         cdg[i] = (int32_t)(P.out_ptr[xv + 1] - cbg[i]);
@@ -648,15 +642,12 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
             warp_flush_regs(claim, x, cdg, cbg, out, P.ebits);
         } else {
             double vals[kLaneItems];
-            bool hit[kLaneItems];
-#pragma unroll
-            for (int i = 0; i < kLaneItems; ++i) hit[i] = act[i] && bit_test(tbm, x[i]);
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
                 if (MODE == MODE_PULL) {
-                    vals[i] = hit[i] ? P.sigma[x[i]] : 0.0;
+                    vals[i] = act[i] ? P.sigma[x[i]] : 0.0;  // sigma is the masked frontier (see edge_pass)
                 } else {
-                    const double u = hit[i] ? P.du[x[i]] : 0.0;
+                    const double u = act[i] ? P.du[x[i]] : 0.0;  // parity-signed delta_u selects level L+1
                     const double want = ((d + 1) & 1) ? -u : u;
                     vals[i] = want > 0.0 ? want : 0.0;
                 }
@@ -760,7 +751,6 @@ __device__ __forceinline__ void pull_owner_pass(const Params &P, WarpSmem &ws, c
                 P.depth[v] = d;
                 P.sigma[v] = tot[i];
                 P.du[v] = 0.0;
-                bit_set(P.fbm[d & 1], v);
                 const int64_t b = P.out_ptr ? P.out_ptr[v] : 0;
                 const int pos = nd + __popc(dm & lt);
                 ws.own[pos] = v;
@@ -826,7 +816,6 @@ __device__ __forceinline__ void bwd_owner_pass(const Params &P, const int32_t *l
             }
             const double dun = (1.0 + delta) / sg[u];
             P.du[v[u]] = (L & 1) ? -dun : dun;
-            bit_set(P.bbm[L & 1], v[u]);
             P.sigma[v[u]] = 0.0;
             P.depth[v[u]] = -1;
         }
@@ -875,12 +864,6 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
         const bool tr = (si == P.trace_src);
         // ---------------- init (Alg.1 l.7-10, l.15-18): depth(s)=0, sigma(s)=1, frontier={s}
         const int64_t dego = P.deg2[s].x;
-        for (int64_t w = gtid; w < P.nwords; w += nthreads) {
-            P.fbm[0][w] = 0u;
-            P.fbm[1][w] = 0u;
-            P.bbm[0][w] = 0u;
-            P.bbm[1][w] = 0u;
-        }
         if (cta0) {
             if (tid == 0) {
                 if (prev_s >= 0) {
@@ -1067,10 +1050,6 @@ tbc_status engine_setup(tbc_graph *g) {
         (e = alloc(&g->tiles, list_tiles)) || (e = alloc(&g->lvl, 5 * (n + 2))) || (e = alloc(&g->ctr, 1)) ||
         (e = alloc(&g->trace, 8 * kTraceCap)))
         return cuda_error(e, "workspace cudaMalloc");
-    const int64_t nwords = (n + 31) / 32;
-    for (int b = 0; b < 2; ++b)
-        if ((e = alloc(&g->fbm[b], nwords)) || (e = alloc(&g->bbm[b], nwords)))
-            return cuda_error(e, "workspace cudaMalloc");
     {
         for (int b = 0; b < 2; ++b)
             if ((e = alloc(&g->cand_v[b], n + 1)) || (e = alloc(&g->cand_pre[b], n + 1)) ||
@@ -1111,11 +1090,6 @@ tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
     P.list_v = g->list_v;
     P.list_pre = g->list_pre;
     P.list_beg = g->list_beg;
-    P.nwords = (g->n + 31) / 32;
-    for (int b = 0; b < 2; ++b) {
-        P.fbm[b] = g->fbm[b];
-        P.bbm[b] = g->bbm[b];
-    }
     P.directed = g->directed;
     P.coot = g->engine == TBC_ENGINE_COOT;
     P.in_col = g->in_col;

@@ -8,7 +8,13 @@
 
 namespace tbc {
 
-constexpr int kBlock = 512;        // threads per CTA of the persistent kernel (one CTA per SM)
+#ifndef TBC_BLOCK
+#define TBC_BLOCK 512
+#endif
+#ifndef TBC_LANE_ITEMS
+#define TBC_LANE_ITEMS 8
+#endif
+constexpr int kBlock = TBC_BLOCK;  // threads per CTA of the persistent kernel (one CTA per SM)
 constexpr int64_t kTraceCap = 65536; // trace entries (one per barrier of the traced source)
 
 // Device-side counters of one graph; all fields are touched by the persistent kernel only.
@@ -38,9 +44,6 @@ struct Params {
     int32_t *list_v;                      // BFS-order vertex list (levels concatenated)
     int64_t *list_pre;                    // exclusive out-degree prefix along list_v
     int64_t *list_beg;                    // out_ptr[v] of each list entry (written at append)
-    uint32_t *fbm[2];                     // forward level bitmaps (level parity)
-    uint32_t *bbm[2];                     // backward level bitmaps (level parity)
-    int64_t nwords;                       // 32-bit words per bitmap
     int32_t *tiles;                       // per level: owner index starting each tile
     int32_t *cand_v[2];                   // pull candidate buffers
     int64_t *cand_pre[2];
@@ -88,8 +91,6 @@ struct tbc_graph {
     int32_t *list_v = nullptr;
     int64_t *list_pre = nullptr;
     int64_t *list_beg = nullptr;
-    uint32_t *fbm[2] = {nullptr, nullptr};
-    uint32_t *bbm[2] = {nullptr, nullptr};
     int32_t *tiles = nullptr;
     int32_t *cand_v[2] = {nullptr, nullptr};
     int64_t *cand_pre[2] = {nullptr, nullptr};

@@ -58,7 +58,10 @@ enum {
 /* create flags */
 enum {
     TBC_FLAG_ONE_FORMAT = 1u << 0,  /* reserved (strict single-format directed mode, not yet built) */
-    TBC_FLAG_NO_VALIDATE = 1u << 1  /* skip host-side input validation (caller guarantees it) */
+    TBC_FLAG_NO_VALIDATE = 1u << 1, /* skip host-side input validation (caller guarantees it) */
+    TBC_FLAG_NO_REORDER = 1u << 2   /* keep the caller's vertex labels internally (default: relabel by
+                                       decreasing degree for cache locality; all inputs and outputs
+                                       stay in the caller's labels either way) */
 };
 
 /* options for tbc_graph_set_option.  Every forward level is run as one of four passes, chosen

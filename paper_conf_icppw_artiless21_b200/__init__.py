@@ -23,7 +23,7 @@ __all__ = ["Graph", "TBCError", "lib", "ENGINE_CSC", "ENGINE_COOT", "DIR_AUTO", 
            "FMT_AUTO", "FMT_LIST", "FMT_STREAM"]
 
 ENGINE_CSC, ENGINE_COOT = 0, 1
-FLAG_ONE_FORMAT, FLAG_NO_VALIDATE = 1, 2
+FLAG_ONE_FORMAT, FLAG_NO_VALIDATE, FLAG_NO_REORDER = 1, 2, 4
 OPT_DIRECTION, OPT_TRACE, OPT_FORMAT = 1, 3, 4
 OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8}
 FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
@@ -105,12 +105,12 @@ class Graph:
 
     @classmethod
     def from_csc(cls, col_ptr, row_idx, directed: bool, engine: int = ENGINE_CSC, device: int = 0,
-                 validate: bool = True):
+                 validate: bool = True, reorder: bool = True):
         cp = np.ascontiguousarray(col_ptr, dtype=np.int64)
         ri = np.ascontiguousarray(row_idx, dtype=np.int32)
         n = cp.size - 1
         h = ctypes.c_void_p()
-        flags = 0 if validate else FLAG_NO_VALIDATE
+        flags = (0 if validate else FLAG_NO_VALIDATE) | (0 if reorder else FLAG_NO_REORDER)
         _check(lib().tbc_graph_create_csc(n, int(cp[-1]) if n >= 0 else 0, _p(cp, ctypes.c_int64),
                                           _p(ri, ctypes.c_int32) if ri.size else None, int(directed),
                                           engine, flags, device, ctypes.byref(h)))
@@ -118,11 +118,11 @@ class Graph:
 
     @classmethod
     def from_coo(cls, n, src, dst, directed: bool, engine: int = ENGINE_CSC, device: int = 0,
-                 validate: bool = True):
+                 validate: bool = True, reorder: bool = True):
         s = np.ascontiguousarray(src, dtype=np.int32)
         d = np.ascontiguousarray(dst, dtype=np.int32)
         h = ctypes.c_void_p()
-        flags = 0 if validate else FLAG_NO_VALIDATE
+        flags = (0 if validate else FLAG_NO_VALIDATE) | (0 if reorder else FLAG_NO_REORDER)
         _check(lib().tbc_graph_create_coo(int(n), s.size, _p(s, ctypes.c_int32) if s.size else None,
                                           _p(d, ctypes.c_int32) if d.size else None, int(directed), engine,
                                           flags, device, ctypes.byref(h)))

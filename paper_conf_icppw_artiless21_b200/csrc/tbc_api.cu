@@ -102,6 +102,41 @@ __global__ void k_count_mismatch(int64_t m, const unsigned long long *__restrict
     if (local) atomicAdd(bad, local);
 }
 
+// degree-descending relabelling: endpoint counts of the raw entries
+__global__ void k_endpoint_count(int64_t nnz, const unsigned long long *__restrict__ keys, int32_t *deg) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x) {
+        const unsigned long long k = keys[i];
+        atomicAdd(&deg[(int64_t)(k >> 32)], 1);
+        atomicAdd(&deg[(int64_t)(k & 0xffffffffull)], 1);
+    }
+}
+
+__global__ void k_iota(int64_t n, int32_t *a) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        a[i] = (int32_t)i;
+}
+
+__global__ void k_invert(int64_t n, const int32_t *__restrict__ inv, int32_t *perm) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        perm[inv[i]] = (int32_t)i;
+}
+
+__global__ void k_relabel(int64_t nnz, unsigned long long *keys, const int32_t *__restrict__ perm) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x) {
+        const unsigned long long k = keys[i];
+        keys[i] = ((unsigned long long)(unsigned)perm[(int64_t)(k >> 32)] << 32) |
+                  (unsigned)perm[(int64_t)(k & 0xffffffffull)];
+    }
+}
+
+__global__ void k_unpermute_bfs(int64_t n, const int32_t *__restrict__ perm, const int32_t *__restrict__ depth,
+                                const double *__restrict__ sigma, int32_t *depth_out, double *sigma_out) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        depth_out[v] = depth[perm[v]];
+        sigma_out[v] = sigma[perm[v]];
+    }
+}
+
 __global__ void k_deg2(int64_t n, const int64_t *__restrict__ out_ptr,
                        const int64_t *__restrict__ in_ptr, int2 *deg2) {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
@@ -148,6 +183,8 @@ void free_graph(tbc_graph *g) {
     cudaFree(g->in_ptr);
     cudaFree(g->in_idx);
     cudaFree(g->deg2);
+    cudaFree(g->perm);
+    cudaFree(g->inv);
     cudaFree(g->in_col);
     if (g->out_row != g->in_col) cudaFree(g->out_row);
     cudaFree(g->depth);
@@ -191,6 +228,39 @@ tbc_status build_from_keys(tbc_graph *g, unsigned long long *d_keys, int64_t nnz
 
     TBC_CUDA(cudaMalloc(&alt, sizeof(unsigned long long) * (nnz > 0 ? nnz : 1)));
     TBC_CUDA(cudaMalloc(&d_num, sizeof(int64_t)));
+    if (!(g->flags & TBC_FLAG_NO_REORDER) && nnz > 0) {
+        // vertex ids by decreasing degree: hubs get small ids, so the gathers of sigma / delta_u
+        // that dominate the traversal hit a compact, cache-resident head of the arrays
+        int32_t *deg = nullptr, *deg_s = nullptr, *ids = nullptr;
+        void *rtemp = nullptr;
+        size_t rbytes = 0;
+        cudaError_t e1 = cudaMalloc(&deg, sizeof(int32_t) * g->n);
+        if (!e1) e1 = cudaMalloc(&deg_s, sizeof(int32_t) * g->n);
+        if (!e1) e1 = cudaMalloc(&ids, sizeof(int32_t) * g->n);
+        if (!e1) e1 = dmalloc(g, &g->inv, g->n);
+        if (!e1) e1 = dmalloc(g, &g->perm, g->n);
+        if (!e1) e1 = cudaMemsetAsync(deg, 0, sizeof(int32_t) * g->n, s);
+        if (!e1) {
+            k_endpoint_count<<<grid_for(nnz), 256, 0, s>>>(nnz, d_keys, deg);
+            k_iota<<<grid_for(g->n), 256, 0, s>>>(g->n, ids);
+            e1 = cub::DeviceRadixSort::SortPairsDescending(nullptr, rbytes, deg, deg_s, ids, g->inv, g->n, 0, 32, s);
+        }
+        if (!e1) e1 = cudaMalloc(&rtemp, rbytes);
+        if (!e1) e1 = cub::DeviceRadixSort::SortPairsDescending(rtemp, rbytes, deg, deg_s, ids, g->inv, g->n, 0, 32, s);
+        if (!e1) {
+            k_invert<<<grid_for(g->n), 256, 0, s>>>(g->n, g->inv, g->perm);
+            k_relabel<<<grid_for(nnz), 256, 0, s>>>(nnz, d_keys, g->perm);
+            e1 = cudaStreamSynchronize(s);
+        }
+        cudaFree(deg);
+        cudaFree(deg_s);
+        cudaFree(ids);
+        cudaFree(rtemp);
+        if (e1) {
+            st = cuda_error(e1, "relabel");
+            goto fail;
+        }
+    }
     TBC_CUDA(cudaMalloc(&d_bad, sizeof(unsigned long long)));
     if (nnz > 0) {
         TBC_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, need, d_keys, alt, nnz, 0, end_bit, s));
@@ -522,10 +592,22 @@ tbc_status tbc_bfs(tbc_graph *g, int32_t source, int32_t *depth_out, double *sig
     TBC_CUDA(cudaMemcpyAsync(g->src_tmp, &source, sizeof(int32_t), cudaMemcpyHostToDevice, g->stream));
     st = engine_run(g, g->src_tmp, 1, nullptr, g->stream, 1);
     if (st != TBC_OK) return st;
-    if (depth_out)
-        TBC_CUDA(cudaMemcpyAsync(depth_out, g->depth, sizeof(int32_t) * g->n, cudaMemcpyDeviceToHost, g->stream));
-    if (sigma_out)
-        TBC_CUDA(cudaMemcpyAsync(sigma_out, g->sigma, sizeof(double) * g->n, cudaMemcpyDeviceToHost, g->stream));
+    {
+        const int32_t *dsrc = g->depth;
+        const double *ssrc = g->sigma;
+        if (g->perm) {  // back to the caller's labels (list_v / bc_tmp are free scratch here)
+            if (!g->bc_tmp) TBC_CUDA(dmalloc(g, &g->bc_tmp, g->n));
+            k_unpermute_bfs<<<grid_for(g->n), 256, 0, g->stream>>>(g->n, g->perm, g->depth, g->sigma, g->list_v,
+                                                                   g->bc_tmp);
+            TBC_CUDA(cudaGetLastError());
+            dsrc = g->list_v;
+            ssrc = g->bc_tmp;
+        }
+        if (depth_out)
+            TBC_CUDA(cudaMemcpyAsync(depth_out, dsrc, sizeof(int32_t) * g->n, cudaMemcpyDeviceToHost, g->stream));
+        if (sigma_out)
+            TBC_CUDA(cudaMemcpyAsync(sigma_out, ssrc, sizeof(double) * g->n, cudaMemcpyDeviceToHost, g->stream));
+    }
     // forward-only runs leave depth/sigma set: restore the all-unvisited workspace invariant
     TBC_CUDA(cudaMemsetAsync(g->depth, 0xff, sizeof(int32_t) * g->n, g->stream));
     TBC_CUDA(cudaMemsetAsync(g->sigma, 0, sizeof(double) * g->n, g->stream));

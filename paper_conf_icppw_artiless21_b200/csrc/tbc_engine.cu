@@ -789,7 +789,7 @@ __device__ __forceinline__ void bwd_owner_pass(const Params &P, const int32_t *l
                                                int64_t nthreads) {
     constexpr int U = 4;
     for (int64_t base = gtid; base < N; base += U * nthreads) {
-        int32_t v[U];
+        int32_t v[U], vb[U];
         double acc[U], sg[U], b[U];
 #pragma unroll
         for (int u = 0; u < U; ++u) {
@@ -803,7 +803,8 @@ __device__ __forceinline__ void bwd_owner_pass(const Params &P, const int32_t *l
             if (v[u] >= 0) {
                 acc[u] = P.gacc[v[u]];
                 sg[u] = P.sigma[v[u]];
-                b[u] = P.bc ? P.bc[v[u]] : 0.0;
+                vb[u] = P.inv ? P.inv[v[u]] : v[u];
+                b[u] = P.bc[vb[u]];
             }
         }
 #pragma unroll
@@ -812,7 +813,7 @@ __device__ __forceinline__ void bwd_owner_pass(const Params &P, const int32_t *l
             const double delta = sg[u] * acc[u];
             if (acc[u] != 0.0) {
                 P.gacc[v[u]] = 0.0;
-                P.bc[v[u]] = b[u] + delta * P.bc_scale;
+                P.bc[vb[u]] = b[u] + delta * P.bc_scale;
             }
             const double dun = (1.0 + delta) / sg[u];
             P.du[v[u]] = (L & 1) ? -dun : dun;
@@ -856,11 +857,12 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
     int32_t prev_s = -1;
 
     for (int64_t si = 0; si < P.k; ++si) {
-        const int32_t s = P.sources[si];
-        if (s < 0 || s >= P.n) {
+        const int32_t s_caller = P.sources[si];
+        if (s_caller < 0 || s_caller >= P.n) {
             if (cta0 && tid == 0) atomicAdd(&C->bad_sources, 1ull);
             continue;
         }
+        const int32_t s = P.perm ? P.perm[s_caller] : s_caller;
         const bool tr = (si == P.trace_src);
         // ---------------- init (Alg.1 l.7-10, l.15-18): depth(s)=0, sigma(s)=1, frontier={s}
         const int64_t dego = P.deg2[s].x;
@@ -1109,6 +1111,8 @@ tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
     P.lvl = g->lvl;
     P.ctr = g->ctr;
     P.bc = d_bc;
+    P.perm = g->perm;
+    P.inv = g->inv;
     P.sources = d_sources;
     P.k = k;
     P.bc_scale = g->directed ? 1.0 : 0.5;

@@ -51,8 +51,10 @@ struct Params {
     int32_t *cand_tiles[2];
     int64_t *lvl;                         // per level: p0, N, e0, E, tile_base
     Ctrs *ctr;
-    double *bc;
-    const int32_t *sources;
+    double *bc;                           // indexed by caller labels
+    const int32_t *sources;               // caller labels
+    const int32_t *__restrict__ perm;     // caller -> internal label (nullptr: identity)
+    const int32_t *__restrict__ inv;      // internal -> caller label
     int64_t k;
     double bc_scale;                      // 0.5 undirected, 1 directed
     int ebits;                            // low bits of packed counters hold edge sums
@@ -83,6 +85,8 @@ struct tbc_graph {
     int64_t *out_ptr = nullptr;  // aliases in_ptr when undirected
     int32_t *out_idx = nullptr;
     int2 *deg2 = nullptr;
+    int32_t *perm = nullptr;     // caller label -> internal label (degree-descending); nullptr = identity
+    int32_t *inv = nullptr;      // internal label -> caller label
     int32_t *in_col = nullptr;   // column (owner) of every CSC entry: with in_idx, the COOC arrays
     int32_t *out_row = nullptr;  // row (owner) of every CSR entry (== in_col when undirected)
     // workspace (device)

@@ -239,3 +239,33 @@ def test_road_lattice(side):
     with gpu_graph(g) as G:
         assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, False, src))
         assert_bfs(g, G, src[0])
+
+
+@pytest.mark.slow
+def test_cfg4_road_lattice_full_size():
+    """Config 4 at full size (4096^2 road-like lattice, D in the thousands): sampled sources vs
+    the oracle, and the per-source delta-sum invariant.  sigma exceeds 2^53 here (relative check)."""
+    g, src = gg.make_config(4)
+    sample = src[:2]
+    with gpu_graph(g) as G:
+        assert_bc(G.bc(sample), oracle.bc(g.col_ptr, g.row_idx, False, sample))
+        assert_bfs(g, G, sample[0])
+        depth, _ = G.bfs(int(src[5]))
+        got = G.bc([int(src[5])]).sum()
+        want = 0.5 * float(np.sum(depth[depth > 0] - 1))
+        assert abs(got - want) <= 1e-9 * want
+
+
+@pytest.mark.slow
+def test_cfg5_kron25_full_size():
+    """Config 5 at full size (scale 25, ~1.05e9 stored entries): one source's depth and sigma
+    against the oracle BFS, and the delta-sum invariant for two more sources."""
+    g, src = gg.make_config(5, device="cuda")
+    with gpu_graph(g) as G:
+        assert G.nnz == g.nnz
+        assert_bfs(g, G, src[0])
+        for s in src[1:3]:
+            depth, _ = G.bfs(int(s))
+            got = G.bc([int(s)]).sum()
+            want = 0.5 * float(np.sum(depth[depth > 0] - 1))
+            assert abs(got - want) <= 1e-9 * want

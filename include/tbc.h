@@ -64,13 +64,17 @@ enum {
                                        stay in the caller's labels either way) */
 };
 
-/* options for tbc_graph_set_option.  Every forward level is run as one of four passes, chosen
+/* options for tbc_graph_set_option.  Every forward level is run as one of five passes, chosen
  * by a per-item cost model: push over the frontier list,
  * push over all stored entries (edge stream, the scCOOC form of Alg. 2), pull over the
- * survivors of the previous pull, pull over all stored entries; every backward level as a
- * list pass or an edge stream.  The options restrict or re-weight that choice. */
+ * survivors of the previous pull, pull over all stored entries, or a candidate scan followed
+ * by a pull over the candidates; every backward level L as a pull over the out-edges of level
+ * L (list pass or edge stream) or a push from level L+1 over its in-edges (list pass, fp64
+ * atomics).  The options restrict or re-weight that choice. */
 enum {
-    TBC_OPT_DIRECTION = 1,   /* 0 auto (default), 1 push only, 2 pull whenever possible (level >= 2) */
+    TBC_OPT_DIRECTION = 1,   /* forward: 0 auto (default), 1 push only, 2 pull whenever possible (level >= 2) */
+    TBC_OPT_BWD_DIRECTION = 2, /* backward: 0 auto (default), 1 pull over the out-edges of level L only,
+                                  2 push from level L+1 over its in-edges whenever possible (list passes) */
     TBC_OPT_TRACE = 3,       /* index in the next calls' source lists whose per-level timeline is
                                 recorded (-1 = off, default) */
     TBC_OPT_FORMAT = 4,      /* 0 auto (default), 1 list passes only, 2 edge streams only
@@ -78,7 +82,9 @@ enum {
     TBC_OPT_COST_LIST = 5,   /* cost model, picoseconds per item: list-pass item (default 12) */
     TBC_OPT_COST_STREAM = 6, /*   stream-pass stored entry (default 4) */
     TBC_OPT_COST_ATOMIC = 7, /*   push contribution (fp64 atomic) (default 18) */
-    TBC_OPT_COST_VERTEX = 8  /*   vertex of a whole-graph owner pass (default 10) */
+    TBC_OPT_COST_VERTEX = 8, /*   vertex of a whole-graph owner pass (default 10) */
+    TBC_OPT_COST_SCAN = 9,   /*   vertex of a candidate scan before a pull that follows a push (default 3) */
+    TBC_OPT_COST_BPUSH = 10  /*   extra per in-edge of a backward push level over a list item (default 6) */
 };
 
 /* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since

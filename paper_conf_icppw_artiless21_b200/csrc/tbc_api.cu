@@ -195,6 +195,10 @@ void free_graph(tbc_graph *g) {
     cudaFree(g->list_pre);
     cudaFree(g->list_beg);
     cudaFree(g->tiles);
+    cudaFree(g->ilist_v);
+    cudaFree(g->ilist_pre);
+    cudaFree(g->ilist_beg);
+    cudaFree(g->itiles);
     for (int b = 0; b < 2; ++b) {
         cudaFree(g->cand_v[b]);
         cudaFree(g->cand_pre[b]);
@@ -528,9 +532,15 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->fmt_mode = v;
         return TBC_OK;
     }
-    if (key >= TBC_OPT_COST_LIST && key <= TBC_OPT_COST_VERTEX) {
+    if (key == TBC_OPT_BWD_DIRECTION) {
+        int v = (int)value;
+        if (v < 0 || v > 2 || (double)v != value) return set_error(TBC_ERR_INVALID, "bwd direction %g", value);
+        g->bwd_mode = v;
+        return TBC_OK;
+    }
+    if (key >= TBC_OPT_COST_LIST && key <= TBC_OPT_COST_BPUSH) {
         if (!(value >= 0)) return set_error(TBC_ERR_INVALID, "cost %g", value);
-        double *c[] = {&g->c_list, &g->c_stream, &g->c_atom, &g->c_vert};
+        double *c[] = {&g->c_list, &g->c_stream, &g->c_atom, &g->c_vert, &g->c_scan, &g->c_bpush};
         *c[key - TBC_OPT_COST_LIST] = value;
         return TBC_OK;
     }

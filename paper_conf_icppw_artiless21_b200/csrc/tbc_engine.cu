@@ -16,7 +16,7 @@
 // Edge passes are merge-path passes over (owner list, adjacency): the diagonal of (owner end
 // items + edges) is cut into warp tiles of kWT items, so a 600k-edge hub and a million
 // degree-1 vertices cost the same per tile.  The producer of a list writes the start owner of
-// every tile while appending (warp_flush), so no search is needed, and tiles are dealt to
+// every tile while appending (warp_append), so no search is needed, and tiles are dealt to
 // warps round-robin (equal items per tile => balanced).  Phases are separated by a grid
 // barrier inside the kernel: no host round trip per level (cf. the paper's per-level kernels
 // and host loop).
@@ -42,7 +42,9 @@ constexpr unsigned FULL = 0xffffffffu;
 #else
 #define TBC_CHECK(cond, ...) ((void)0)
 #endif
-enum { MODE_PUSH = 0, MODE_PULL = 1, MODE_BWD = 2 };
+// PUSH/PULL: forward level; BWD: backward level pulled over the owners' out-edges;
+// BPUSH: backward level pushed from level L+1 over its in-edges (fp64 atomics into level L)
+enum { MODE_PUSH = 0, MODE_PULL = 1, MODE_BWD = 2, MODE_BPUSH = 3 };
 
 constexpr int kLaneItems = TBC_LANE_ITEMS;  // items per lane per warp tile
 constexpr int kWT = 32 * kLaneItems;   // diagonal items per warp tile
@@ -159,12 +161,8 @@ __device__ __forceinline__ void grid_sync(Ctrs *c, unsigned &gen) {
 
 // ------------------------------------------------------------------ warp-aggregated append
 
-// Append c buffered entries (vertex bv[i], degree bd[i], adjacency begin bb[i]) with ONE packed
-// 64-bit atomic for the whole warp: (count << ebits) | degree_sum.  Count and prefix are
-// reserved together, so list order and prefix order agree and each owner knows its merge-path
-// span [k0, k0+deg] inside its level: it writes the start owner of every tile whose first
-// diagonal lies in that span.  Lane l takes entries [l*q, l*q+q); a warp scan of the lanes'
-// degree sums gives the prefixes.  c must be warp-uniform; all 32 lanes call this.
+// A list being appended to: packed counter (count << ebits) | degree_sum, the arrays, the
+// level's tile table, and the level's start (list position, degree prefix).
 struct ListOut {
     unsigned long long *ctr;
     int32_t *v;
@@ -174,91 +172,73 @@ struct ListOut {
     int64_t p0, e0;  // level start within the list (list position, edge prefix)
 };
 
-__device__ __forceinline__ void warp_flush(int c, const int32_t *bv, const int32_t *bd, const int64_t *bb,
-                                           const ListOut &o, int ebits) {
-    if (c == 0) return;
+// Append the entries a warp holds in registers (lane l, item i: vertex v[i], degree dg[i],
+// adjacency begin bg[i], if take[i]) with ONE packed 64-bit atomic for the whole warp:
+// (count << ebits) | degree_sum, so list order and degree-prefix order agree and every
+// appended owner knows its merge-path span [k0, k0 + deg] inside its level: it writes the start
+// owner of every tile whose first diagonal item lies in that span.  Entries are ordered
+// item-major, lane-minor, so each item's stores are coalesced across the warp; the prefix is
+// one warp scan per item.  Degrees of distinct vertices sum to <= m < 2^32 (engine_setup).
+// All 32 lanes call this (warp-uniform control flow).
+__device__ __forceinline__ void warp_append(const bool (&take)[kLaneItems], const int32_t (&v)[kLaneItems],
+                                            const uint32_t (&dg)[kLaneItems], const int64_t (&bg)[kLaneItems],
+                                            const ListOut &o, int ebits) {
     const int lane = threadIdx.x & 31;
-    const int q = (c + 31) >> 5;
-    const int lo = min(lane * q, c), hi = min(lo + q, c);
-    int64_t sum = 0;
-    for (int i = lo; i < hi; ++i) sum += bd[i];
-    int64_t inc = sum;
+    const unsigned lt = (1u << lane) - 1u;
+    unsigned cnt = 0;
+    unsigned long long esum = 0;
 #pragma unroll
-    for (int k = 1; k < 32; k <<= 1) {
-        const int64_t t = __shfl_up_sync(FULL, inc, k);
-        if (lane >= k) inc += t;
+    for (int i = 0; i < kLaneItems; ++i) {
+        cnt += __popc(__ballot_sync(FULL, take[i]));
+        esum += __reduce_add_sync(FULL, take[i] ? dg[i] : 0u);
     }
-    const int64_t tot = __shfl_sync(FULL, inc, 31);
+    if (cnt == 0) return;
     unsigned long long old = 0;
-    if (lane == 0) old = atomicAdd(o.ctr, ((unsigned long long)c << ebits) + (unsigned long long)tot);
+    if (lane == 0) old = atomicAdd(o.ctr, ((unsigned long long)cnt << ebits) + esum);
     old = __shfl_sync(FULL, old, 0);
-    int64_t p = (int64_t)(old >> ebits) + lo;
-    int64_t e = (int64_t)(old & ((1ull << ebits) - 1ull)) + inc - sum;
-    for (int i = lo; i < hi; ++i, ++p) {
-        const int64_t dg = bd[i];
-        TBC_CHECK(bv[i] >= 0 && dg >= 0, "flush v %d dg %lld", bv[i], (long long)dg);
-        o.v[p] = bv[i];
-        o.pre[p] = e;
-        o.beg[p] = bb[i];
-        const int64_t k0 = (e - o.e0) + (p - o.p0);
-        const int64_t k1 = k0 + dg;
-        for (int64_t t = (k0 + kWT - 1) / kWT; t <= k1 / kWT; ++t) o.tiles[t] = (int32_t)(p - o.p0);
-        e += dg;
+    int64_t p = (int64_t)(old >> ebits);
+    int64_t e = (int64_t)(old & ((1ull << ebits) - 1ull));
+#pragma unroll
+    for (int i = 0; i < kLaneItems; ++i) {
+        const unsigned msk = __ballot_sync(FULL, take[i]);
+        if (msk == 0) continue;
+        const uint32_t x = take[i] ? dg[i] : 0u;
+        uint32_t inc = x;
+#pragma unroll
+        for (int k = 1; k < 32; k <<= 1) {
+            const uint32_t t = __shfl_up_sync(FULL, inc, k);
+            if (lane >= k) inc += t;
+        }
+        if (take[i]) {
+            const int64_t pp = p + __popc(msk & lt);
+            const int64_t ee = e + (int64_t)(inc - x);
+            TBC_CHECK(v[i] >= 0, "append v %d", v[i]);
+            o.v[pp] = v[i];
+            o.pre[pp] = ee;
+            o.beg[pp] = bg[i];
+            const int64_t k0 = (ee - o.e0) + (pp - o.p0);
+            const int64_t k1 = k0 + x;
+            for (int64_t t = (k0 + kWT - 1) / kWT; t <= k1 / kWT; ++t) o.tiles[t] = (int32_t)(pp - o.p0);
+        }
+        p += __popc(msk);
+        e += __shfl_sync(FULL, inc, 31);
     }
 }
 
-// Register variant of warp_flush for up to kLaneItems appends per lane (no shared memory): a
-// warp scan of the lanes' counts and degree sums gives every lane its consecutive slots.
-__device__ __forceinline__ void warp_flush_regs(const bool (&take)[kLaneItems], const int32_t (&v)[kLaneItems],
-                                                const int32_t (&dg)[kLaneItems], const int64_t (&bg)[kLaneItems],
-                                                const ListOut &o, int ebits) {
-    const int lane = threadIdx.x & 31;
-    int c = 0;
-    int64_t sum = 0;
-#pragma unroll
-    for (int i = 0; i < kLaneItems; ++i)
-        if (take[i]) {
-            ++c;
-            sum += dg[i];
-        }
-    if (!__any_sync(FULL, c > 0)) return;
-    int cinc = c;
-    int64_t inc = sum;
-#pragma unroll
-    for (int k = 1; k < 32; k <<= 1) {
-        const int tc = __shfl_up_sync(FULL, cinc, k);
-        const int64_t t = __shfl_up_sync(FULL, inc, k);
-        if (lane >= k) {
-            cinc += tc;
-            inc += t;
-        }
-    }
-    const int ctot = __shfl_sync(FULL, cinc, 31);
-    const int64_t tot = __shfl_sync(FULL, inc, 31);
-    unsigned long long old = 0;
-    if (lane == 0) old = atomicAdd(o.ctr, ((unsigned long long)ctot << ebits) + (unsigned long long)tot);
-    old = __shfl_sync(FULL, old, 0);
-    int64_t p = (int64_t)(old >> ebits) + cinc - c;
-    int64_t e = (int64_t)(old & ((1ull << ebits) - 1ull)) + inc - sum;
-#pragma unroll
-    for (int i = 0; i < kLaneItems; ++i) {
-        if (!take[i]) continue;
-        o.v[p] = v[i];
-        o.pre[p] = e;
-        o.beg[p] = bg[i];
-        const int64_t k0 = (e - o.e0) + (p - o.p0);
-        const int64_t k1 = k0 + dg[i];
-        for (int64_t t = (k0 + kWT - 1) / kWT; t <= k1 / kWT; ++t) o.tiles[t] = (int32_t)(p - o.p0);
-        e += dg[i];
-        ++p;
-    }
+// degree and adjacency begin of v in a pointer array (CSC in_ptr or CSR out_ptr)
+__device__ __forceinline__ void adj_span(const int64_t *ptr, int32_t v, uint32_t &dg, int64_t &bg) {
+    bg = ptr[v];
+    dg = (uint32_t)(ptr[v + 1] - bg);
 }
 
 // ------------------------------------------------------------------ level descriptors
 
+// a BFS level: list positions [p0, p0+N) (both lists), out-edge prefix base e0 and sum E with
+// its tile base, in-edge prefix base ie0 and sum IE of the in-degree list with its tile base
 struct Level {
-    int64_t p0, N, e0, E, tbase;
+    int64_t p0, N, e0, E, tbase, ie0, IE, itbase;
 };
+constexpr int kLvlWords = 8;
 
 __device__ __forceinline__ int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
@@ -283,7 +263,7 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
                                           const int64_t *obeg, const int32_t *otiles, int64_t N, int64_t E,
                                           int64_t e0, const int64_t *__restrict__ adj_ptr,
                                           const int32_t *__restrict__ adj_idx, int d, int64_t gwarp, int64_t nwarps,
-                                          ListOut out) {
+                                          ListOut out, ListOut out_in) {
     const int lane = threadIdx.x & 31;
     const int64_t K = N + E;
     const int64_t ntiles = ceil_div(K, kWT);
@@ -312,8 +292,14 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
             ws.beg[j] = obeg[ps + j] + (f - pre);
             ws.v[j] = v;
             ws.own[j] = -1;
-            if (MODE == MODE_PUSH) ws.val[j] = P.sigma[v];
-            else ws.val[j] = 0.0;
+            if (MODE == MODE_PUSH) {
+                ws.val[j] = P.sigma[v];
+            } else if (MODE == MODE_BPUSH) {  // owner on level d+1: its delta_u, sign by parity
+                const double u = P.du[v];
+                ws.val[j] = ((d + 1) & 1) ? -u : u;
+            } else {
+                ws.val[j] = 0.0;
+            }
             if (j == 0) start0 = pre >= es;  // owner 0 begins inside this tile
 
         }
@@ -381,27 +367,36 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
                 olds[i] = 1.0;
                 if (dxs[i] == -1 || dxs[i] == d) olds[i] = atomicAdd(&P.sigma[xs[i]], ws.val[js[i]]);
             }
-            __syncwarp();  // own[] / first[] / beg[] become the claim buffers below
-            int cnt = 0;
+            bool claim[kLaneItems];
+            uint32_t cdg[kLaneItems];
+            int64_t cbg[kLaneItems];
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
-                const bool claim = olds[i] == 0.0;
-                const unsigned cm = __ballot_sync(FULL, claim);
-                if (claim) {
-                    const int32_t x = xs[i];
-                    P.depth[x] = d;
-                    P.du[x] = 0.0;
-                    const int64_t b = adj_ptr[x];
-                    const int64_t dg = adj_ptr[x + 1] - b;
-                    const int pos = cnt + __popc(cm & ((1u << lane) - 1u));
-                    ws.own[pos] = x;
-                    ws.first[pos] = (int32_t)dg;
-                    ws.beg[pos] = b;
+                claim[i] = olds[i] == 0.0;
+                cdg[i] = 0;
+                cbg[i] = 0;
+                if (claim[i]) {
+                    P.depth[xs[i]] = d;
+                    P.du[xs[i]] = 0.0;
+                    adj_span(adj_ptr, xs[i], cdg[i], cbg[i]);
                 }
-                cnt += __popc(cm);
             }
-            __syncwarp();
-            warp_flush(cnt, ws.own, ws.first, ws.beg, out, P.ebits);
+            warp_append(claim, xs, cdg, cbg, out, P.ebits);
+            if (out_in.ctr) {
+#pragma unroll
+                for (int i = 0; i < kLaneItems; ++i)
+                    if (claim[i]) adj_span(P.in_ptr, xs[i], cdg[i], cbg[i]);
+                warp_append(claim, xs, cdg, cbg, out_in, P.ebits);
+            }
+        } else if (MODE == MODE_BPUSH) {
+            // transposed SpMV of Alg.1 l.37 (reading R1: A delta_u) as a push: every in-edge
+            // v -> w of an owner w on level d+1 adds delta_u(w) to acc(v) when v is on level d
+            int dxs[kLaneItems];
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i) dxs[i] = js[i] >= 0 ? P.depth[xs[i]] : -2;
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i)
+                if (dxs[i] == d) atomicAdd(&P.gacc[xs[i]], ws.val[js[i]]);
         } else {
             double vals[kLaneItems];
             if (MODE == MODE_PULL) {
@@ -517,7 +512,7 @@ static_assert(sizeof(StreamStage) * kStages + 8 * kStages <= sizeof(WarpSmem), "
 template <int MODE>
 __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const int32_t *__restrict__ own_arr,
                                             const int32_t *__restrict__ idx, bool sorted, int d, int64_t gwarp,
-                                            int64_t nwarps, const ListOut &out) {
+                                            int64_t nwarps, const ListOut &out, const ListOut &out_in) {
     const int lane = threadIdx.x & 31;
     const int64_t m = P.m;
     const uint64_t pol = policy_evict_first();
@@ -622,7 +617,7 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
                 if (dxs[i] == -1 || dxs[i] == d) olds[i] = atomicAdd(&P.sigma[x[i]], osig[i]);
             }
             bool claim[kLaneItems];
-            int32_t cdg[kLaneItems];
+            uint32_t cdg[kLaneItems];
             int64_t cbg[kLaneItems];
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
@@ -630,16 +625,18 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
                 cdg[i] = 0;
                 cbg[i] = 0;
                 if (claim[i]) {
-                    const int32_t xv = x[i];
-                    P.depth[xv] = d;
-                    P.du[xv] = 0.0;
-                    if (P.out_ptr) {
-                        cbg[i] = P.out_ptr[xv];
-                        cdg[i] = (int32_t)(P.out_ptr[xv + 1] - cbg[i]);
-                    }
+                    P.depth[x[i]] = d;
+                    P.du[x[i]] = 0.0;
+                    if (P.out_ptr) adj_span(P.out_ptr, x[i], cdg[i], cbg[i]);
                 }
             }
-            warp_flush_regs(claim, x, cdg, cbg, out, P.ebits);
+            warp_append(claim, x, cdg, cbg, out, P.ebits);
+            if (out_in.ctr) {
+#pragma unroll
+                for (int i = 0; i < kLaneItems; ++i)
+                    if (claim[i]) adj_span(P.in_ptr, x[i], cdg[i], cbg[i]);
+                warp_append(claim, x, cdg, cbg, out_in, P.ebits);
+            }
         } else {
             double vals[kLaneItems];
 #pragma unroll
@@ -720,11 +717,10 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
 // PULL owner pass over the candidate list: the mask of Alg.1 l.20-25 / Alg.3 l.12-13.
 // Discovered (sum > 0) -> depth = d, sigma = sum, appended to the level list; otherwise the
 // candidate survives into the next candidate list.  Chunks of kWT owners per warp.
-__device__ __forceinline__ void pull_owner_pass(const Params &P, WarpSmem &ws, const int32_t *cv, int64_t N, int d,
+__device__ __forceinline__ void pull_owner_pass(const Params &P, const int32_t *cv, int64_t N, int d,
                                                 int64_t gwarp, int64_t nwarps, const ListOut &lvl_out,
-                                                const ListOut &cand_out) {
+                                                const ListOut &ilvl_out, const ListOut &cand_out) {
     const int lane = threadIdx.x & 31;
-    const unsigned lt = (1u << lane) - 1u;
     for (int64_t base = gwarp * kWT; base < N; base += nwarps * kWT) {
         int32_t vv[kLaneItems];
         double tot[kLaneItems];
@@ -740,46 +736,70 @@ __device__ __forceinline__ void pull_owner_pass(const Params &P, WarpSmem &ws, c
             TBC_CHECK(vv[i] < P.n, "pull owner v %d", vv[i]);
             tot[i] = vv[i] >= 0 ? P.gacc[vv[i]] : 0.0;
         }
-        int nd = 0;
+        bool take[kLaneItems];
+        uint32_t dg[kLaneItems];
+        int64_t bg[kLaneItems];
 #pragma unroll
         for (int i = 0; i < kLaneItems; ++i) {
-            const bool disc = vv[i] >= 0 && tot[i] > 0.0;
-            const unsigned dm = __ballot_sync(FULL, disc);
-            if (disc) {
+            take[i] = vv[i] >= 0 && tot[i] > 0.0;
+            dg[i] = 0;
+            bg[i] = 0;
+            if (take[i]) {
                 const int32_t v = vv[i];
                 P.gacc[v] = 0.0;
                 P.depth[v] = d;
                 P.sigma[v] = tot[i];
                 P.du[v] = 0.0;
-                const int64_t b = P.out_ptr ? P.out_ptr[v] : 0;
-                const int pos = nd + __popc(dm & lt);
-                ws.own[pos] = v;
-                ws.first[pos] = P.out_ptr ? (int32_t)(P.out_ptr[v + 1] - b) : 0;
-                ws.beg[pos] = b;
+                if (P.out_ptr) adj_span(P.out_ptr, v, dg[i], bg[i]);
             }
-            nd += __popc(dm);
         }
-        __syncwarp();
-        warp_flush(nd, ws.own, ws.first, ws.beg, lvl_out, P.ebits);
-        __syncwarp();
-        int nk = 0;
+        warp_append(take, vv, dg, bg, lvl_out, P.ebits);
+        if (ilvl_out.ctr) {
+#pragma unroll
+            for (int i = 0; i < kLaneItems; ++i)
+                if (take[i]) adj_span(P.in_ptr, vv[i], dg[i], bg[i]);
+            warp_append(take, vv, dg, bg, ilvl_out, P.ebits);
+        }
+        // survivors: next candidate list, keyed by in-degree
 #pragma unroll
         for (int i = 0; i < kLaneItems; ++i) {
-            const bool keep = vv[i] >= 0 && !(tot[i] > 0.0);
-            const unsigned km = __ballot_sync(FULL, keep);
-            if (keep) {  // survivors: next candidate list, keyed by in-degree
-                const int32_t v = vv[i];
-                const int64_t b = P.in_ptr[v];
-                const int pos = nk + __popc(km & lt);
-                ws.own[pos] = v;
-                ws.first[pos] = (int32_t)(P.in_ptr[v + 1] - b);
-                ws.beg[pos] = b;
-            }
-            nk += __popc(km);
+            take[i] = vv[i] >= 0 && !(tot[i] > 0.0);
+            if (take[i]) adj_span(P.in_ptr, vv[i], dg[i], bg[i]);
         }
-        __syncwarp();
-        warp_flush(nk, ws.own, ws.first, ws.beg, cand_out, P.ebits);
-        __syncwarp();
+        warp_append(take, vv, dg, bg, cand_out, P.ebits);
+    }
+}
+
+// Candidate scan before a pull that follows push levels: every undiscovered vertex with
+// in-edges (labels [0, n_scan) -- degree-sorted labels put the isolated vertices last) is
+// appended to the candidate list, keyed by in-degree, so the pull pass costs the candidates'
+// in-edges instead of all m (Alg.3 examines every column; the mask of l.20 makes
+// the discovered columns' work void).
+__device__ __forceinline__ void cand_scan_pass(const Params &P, int64_t gwarp, int64_t nwarps,
+                                               const ListOut &cand_out) {
+    const int lane = threadIdx.x & 31;
+    const int64_t N = P.n_scan;
+    for (int64_t base = gwarp * kWT; base < N; base += nwarps * kWT) {
+        bool take[kLaneItems];
+        int32_t vv[kLaneItems];
+        uint32_t dg[kLaneItems];
+        int64_t bg[kLaneItems];
+#pragma unroll
+        for (int i = 0; i < kLaneItems; ++i) {
+            const int64_t v = base + i * 32 + lane;
+            vv[i] = (int32_t)v;
+            take[i] = v < N && P.depth[v] == -1;
+        }
+#pragma unroll
+        for (int i = 0; i < kLaneItems; ++i) {
+            dg[i] = 0;
+            bg[i] = 0;
+            if (take[i]) {
+                adj_span(P.in_ptr, vv[i], dg[i], bg[i]);
+                take[i] = dg[i] > 0;
+            }
+        }
+        warp_append(take, vv, dg, bg, cand_out, P.ebits);
     }
 }
 
@@ -855,6 +875,8 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
     unsigned gen = (tid == 0) ? ld_acquire(&C->bar_gen) : 0u;
     const unsigned long long emask = (1ull << P.ebits) - 1ull;
     int32_t prev_s = -1;
+    // the in-degree list: a separate list for directed graphs, the out-list itself otherwise
+    unsigned long long *ictr = P.in_list ? &C->ilist : &C->list;
 
     for (int64_t si = 0; si < P.k; ++si) {
         const int32_t s_caller = P.sources[si];
@@ -866,6 +888,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
         const bool tr = (si == P.trace_src);
         // ---------------- init (Alg.1 l.7-10, l.15-18): depth(s)=0, sigma(s)=1, frontier={s}
         const int64_t dego = P.deg2[s].x;
+        const int64_t degi = P.deg2[s].y;
         if (cta0) {
             if (tid == 0) {
                 if (prev_s >= 0) {
@@ -879,17 +902,26 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
                 P.list_pre[0] = 0;
                 P.list_beg[0] = P.out_ptr ? P.out_ptr[s] : 0;
                 C->list = (1ull << P.ebits) | (unsigned long long)dego;
+                if (P.in_list) {
+                    P.ilist_v[0] = s;
+                    P.ilist_pre[0] = 0;
+                    P.ilist_beg[0] = P.in_ptr[s];
+                    C->ilist = (1ull << P.ebits) | (unsigned long long)degi;
+                }
                 C->cand[0] = 0;
                 C->cand[1] = 0;
                 if (tr) C->trace_n = 0;
             }
             for (int64_t i = tid; i <= dego / kWT; i += kBlock) P.tiles[i] = 0;
+            if (P.in_list)
+                for (int64_t i = tid; i <= degi / kWT; i += kBlock) P.itiles[i] = 0;
         }
         prev_s = s;
         grid_sync(C, gen);
         trace(P, tr, TR_INIT, 0, 1, dego, s, 0);
 
-        Level cur{0, 1, 0, dego, 0};  // level d-1 (frontier)
+        // level d-1 (frontier)
+        Level cur{0, 1, 0, dego, 0, 0, P.in_list ? degi : dego, 0};
         int d = 1;
         bool cand_valid = false;
         int cb = 0;
@@ -902,50 +934,72 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
         const int32_t *push_idx = coot_dir ? P.in_col : P.out_idx;
         for (;;) {
             const int64_t ntiles_f = ceil_div(cur.N + cur.E, kWT);
-            Level nxt{cur.p0 + cur.N, 0, cur.e0 + cur.E, 0, cur.tbase + ntiles_f};
+            const int64_t ntiles_i = ceil_div(cur.N + cur.IE, kWT);
+            Level nxt{cur.p0 + cur.N, 0, cur.e0 + cur.E, 0, cur.tbase + ntiles_f,
+                      cur.ie0 + cur.IE, 0, cur.itbase + ntiles_i};
             // ---- per-level choice: modelled cost of
-            //      push over the frontier list, push over all entries, pull over the survivors
-            //      of the previous pull, pull over all entries.  Pull needs d >= 2.
+            //      0 push over the frontier list, 1 push over all entries, 2 pull over the
+            //      survivors of the previous pull, 3 pull over all entries, 4 candidate scan +
+            //      pull over the candidates' in-edges.  Pull needs d >= 2.
             const double mE = (double)P.m;
-            double cost[4] = {(double)cur.E * (P.c_list + P.c_atom), mE * P.c_stream + (double)cur.E * P.c_atom,
+            // candidates of a scan: undiscovered vertices with in-edges and their in-edges
+            const double scanE = (double)max((int64_t)0, P.m - nxt.ie0);
+            const double scanN = (double)max((int64_t)0, P.n_in - nxt.p0);
+            double cost[5] = {(double)cur.E * (P.c_list + P.c_atom), mE * P.c_stream + (double)cur.E * P.c_atom,
                               cand_valid ? (double)candE * P.c_list + (double)candN * P.c_vert : 1e300,
-                              mE * P.c_stream + (double)P.n * P.c_vert};
-            if (d < 2 || P.dir_mode == 1) cost[2] = cost[3] = 1e300;   // push only
-            if (d >= 2 && P.dir_mode == 2) cost[0] = cost[1] = 1e300;  // pull whenever possible
-            if (P.fmt_mode == 1 && !P.coot) cost[1] = cost[3] = 1e300; // list passes only
-            if (P.fmt_mode == 2 || P.coot) cost[0] = cost[2] = 1e300;  // edge streams only
+                              mE * P.c_stream + (double)P.n * P.c_vert,
+                              cand_valid ? 1e300
+                                         : (double)P.n_scan * P.c_scan + scanE * P.c_list + scanN * P.c_vert};
+            if (d < 2 || P.dir_mode == 1) cost[2] = cost[3] = cost[4] = 1e300;  // push only
+            if (d >= 2 && P.dir_mode == 2) cost[0] = cost[1] = 1e300;             // pull whenever possible
+            if (P.fmt_mode == 1 && !P.coot) cost[1] = cost[3] = 1e300;            // list passes only
+            if (P.fmt_mode == 2 || P.coot) cost[0] = cost[2] = cost[4] = 1e300;   // edge streams only
             int choice = 0;
-            for (int c = 1; c < 4; ++c)
+            for (int c = 1; c < 5; ++c)
                 if (cost[c] < cost[choice]) choice = c;
             const bool pull = choice >= 2;
             const ListOut lo{&C->list, P.list_v, P.list_pre, P.list_beg, P.tiles + nxt.tbase, nxt.p0, nxt.e0};
+            const ListOut li = P.in_list ? ListOut{&C->ilist, P.ilist_v, P.ilist_pre, P.ilist_beg,
+                                                   P.itiles + nxt.itbase, nxt.p0, nxt.ie0}
+                                         : ListOut{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0};
             if (pull) {
                 const bool stream = choice == 3;
+                if (choice == 4) {
+                    // candidate list cb is empty here (reset by the push level before its barrier)
+                    const ListOut sc{&C->cand[cb], P.cand_v[cb], P.cand_pre[cb], P.cand_beg[cb], P.cand_tiles[cb], 0, 0};
+                    cand_scan_pass(P, gwarp, nwarps, sc);
+                    grid_sync(C, gen);
+                    const unsigned long long cv = ld_volatile_u64(&C->cand[cb]);
+                    candN = (int64_t)(cv >> P.ebits);
+                    candE = (int64_t)(cv & emask);
+                    ++scans;
+                    trace(P, tr, TR_SCAN, d, candN, candE, 0, 0);
+                }
                 const ListOut co{&C->cand[cb ^ 1], P.cand_v[cb ^ 1], P.cand_pre[cb ^ 1], P.cand_beg[cb ^ 1],
                                  P.cand_tiles[cb ^ 1], 0, 0};
                 if (stream) {
-                    stream_pass<MODE_PULL>(P, ws, P.in_col, P.in_idx, true, d, gwarp, nwarps, lo);
+                    stream_pass<MODE_PULL>(P, ws, P.in_col, P.in_idx, true, d, gwarp, nwarps, lo, li);
                     candN = P.n;
                     candE = P.m;
                     ++scans;
                 } else {
                     edge_pass<MODE_PULL>(P, ws, P.cand_v[cb], P.cand_pre[cb], P.cand_beg[cb], P.cand_tiles[cb], candN,
-                                         candE, 0, P.in_ptr, P.in_idx, d, gwarp, nwarps, lo);
+                                         candE, 0, P.in_ptr, P.in_idx, d, gwarp, nwarps, lo, li);
                 }
                 grid_sync(C, gen);
                 trace(P, tr, TR_PULL, d, candN, candE, stream, 0);
                 // owner pass: the survivors of a stream pull are all undiscovered vertices
-                pull_owner_pass(P, ws, stream ? nullptr : P.cand_v[cb], candN, d, gwarp, nwarps, lo, co);
+                pull_owner_pass(P, stream ? nullptr : P.cand_v[cb], candN, d, gwarp, nwarps, lo, li, co);
                 fwd_edges += candE;
                 ++pulls;
                 cand_valid = !P.coot;
             } else {
                 if (choice == 1)
-                    stream_pass<MODE_PUSH>(P, ws, push_own, push_idx, !coot_dir, d, gwarp, nwarps, lo);
+                    stream_pass<MODE_PUSH>(P, ws, push_own, push_idx, !coot_dir, d, gwarp, nwarps, lo, li);
                 else
                     edge_pass<MODE_PUSH>(P, ws, P.list_v + cur.p0, P.list_pre + cur.p0, P.list_beg + cur.p0,
                                          P.tiles + cur.tbase, cur.N, cur.E, cur.e0, P.out_ptr, P.out_idx, d, gwarp,
-                                         nwarps, lo);
+                                         nwarps, lo, li);
                 fwd_edges += choice == 1 ? P.m : cur.E;
                 if (cta0 && tid == 0) {
                     C->cand[0] = 0;  // candidate lists are stale after a push level
@@ -958,6 +1012,8 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
                 const unsigned long long lv = ld_volatile_u64(&C->list);
                 nxt.N = (int64_t)(lv >> P.ebits) - nxt.p0;
                 nxt.E = (int64_t)(lv & emask) - nxt.e0;
+                const unsigned long long il = ld_volatile_u64(ictr);
+                nxt.IE = (int64_t)(il & emask) - nxt.ie0;
             }
             trace(P, tr, pull ? TR_OWNER : TR_PUSH, d, nxt.N, nxt.E, choice, pull ? candE : cur.E);
             if (pull) {
@@ -968,8 +1024,9 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
                 cb ^= 1;
             }
             if (cta0 && tid == 0) {
-                int64_t *l = P.lvl + 5 * (int64_t)d;
+                int64_t *l = P.lvl + kLvlWords * (int64_t)d;
                 l[0] = nxt.p0; l[1] = nxt.N; l[2] = nxt.e0; l[3] = nxt.E; l[4] = nxt.tbase;
+                l[5] = nxt.ie0; l[6] = nxt.IE; l[7] = nxt.itbase;
             }
             if (nxt.N == 0) break;
             if (d > P.n + 1) __trap();  // impossible for a correct BFS: fail loudly, never spin
@@ -990,30 +1047,51 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
         if (P.bfs_only) break;
 
         // ---------------- backward (Alg.1 l.29-47): L = D (owner pass only: delta = 0) .. 1
+        // Each level L < D is one of: pull over the out-edges of level L (list or stream), or
+        // push from level L+1 over its in-edges (the transposed product with atomics), by cost.
         int64_t bwd_edges = 0;
+        Level up = cur;  // level L+1 while processing level L
         for (int L = D; L >= 1; --L) {
             Level lv;
             if (L == D) {
                 lv = cur;
             } else {
-                const int64_t *l = P.lvl + 5 * (int64_t)L;
-                lv = Level{l[0], l[1], l[2], l[3], l[4]};
+                const int64_t *l = P.lvl + kLvlWords * (int64_t)L;
+                lv = Level{l[0], l[1], l[2], l[3], l[4], l[5], l[6], l[7]};
                 const ListOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0};
-                const bool stream = P.coot || P.fmt_mode == 2 ||
-                                    (P.fmt_mode == 0 && (double)P.m * P.c_stream < (double)lv.E * P.c_list);
-                if (stream)
-                    stream_pass<MODE_BWD>(P, ws, push_own, push_idx, !coot_dir, L, gwarp, nwarps, none);
-                else
+                double bcost[3] = {(double)lv.E * P.c_list, (double)P.m * P.c_stream,
+                                   (double)up.IE * (P.c_list + P.c_bpush)};
+                if (P.coot || P.fmt_mode == 2) bcost[0] = bcost[2] = 1e300;
+                if (P.fmt_mode == 1 && !P.coot) bcost[1] = 1e300;
+                if (P.bwd_mode == 1) bcost[2] = 1e300;
+                if (P.bwd_mode == 2 && bcost[2] < 1e300) bcost[0] = bcost[1] = 1e300;
+                int bsel = 0;
+                for (int c = 1; c < 3; ++c)
+                    if (bcost[c] < bcost[bsel]) bsel = c;
+                if (bsel == 1) {
+                    stream_pass<MODE_BWD>(P, ws, push_own, push_idx, !coot_dir, L, gwarp, nwarps, none, none);
+                    bwd_edges += P.m;
+                } else if (bsel == 0) {
                     edge_pass<MODE_BWD>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.list_beg + lv.p0,
                                         P.tiles + lv.tbase, lv.N, lv.E, lv.e0, P.out_ptr, P.out_idx, L, gwarp, nwarps,
-                                        none);
-                bwd_edges += stream ? P.m : lv.E;
+                                        none, none);
+                    bwd_edges += lv.E;
+                } else {
+                    const int32_t *iv = P.in_list ? P.ilist_v : P.list_v;
+                    const int64_t *ip = P.in_list ? P.ilist_pre : P.list_pre;
+                    const int64_t *ib = P.in_list ? P.ilist_beg : P.list_beg;
+                    const int32_t *it = P.in_list ? P.itiles + up.itbase : P.tiles + up.tbase;
+                    edge_pass<MODE_BPUSH>(P, ws, iv + up.p0, ip + up.p0, ib + up.p0, it, up.N, up.IE, up.ie0,
+                                          P.in_ptr, P.in_idx, L, gwarp, nwarps, none, none);
+                    bwd_edges += up.IE;
+                }
                 grid_sync(C, gen);
-                trace(P, tr, TR_BWD, L, lv.N, lv.E, 0, 0);
+                trace(P, tr, TR_BWD, L, lv.N, lv.E, bsel, 0);
             }
             bwd_owner_pass(P, P.list_v + lv.p0, lv.N, L, gtid, nthreads);
             grid_sync(C, gen);
             trace(P, tr, TR_OWNER, L, lv.N, lv.E, 1, 0);
+            up = lv;
         }
         if (cta0 && tid == 0) C->st_bwd_edges += bwd_edges;
     }
@@ -1027,6 +1105,15 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
 }  // namespace
 
 // ------------------------------------------------------------------ host side
+
+// n_scan = 1 + the largest vertex with in-degree > 0; n_in = how many vertices have one
+__global__ void k_in_range(int64_t n, const int2 *__restrict__ deg2, unsigned long long *out) {
+    const int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const bool has = v < n && deg2[v].y > 0;
+    const unsigned m = __ballot_sync(FULL, has);
+    if (has) atomicMax(&out[0], (unsigned long long)(v + 1));
+    if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&out[1], (unsigned long long)__popc(m));
+}
 
 tbc_status engine_setup(tbc_graph *g) {
     const int64_t n = g->n, m = g->m;
@@ -1049,9 +1136,14 @@ tbc_status engine_setup(tbc_graph *g) {
     if ((e = alloc(&g->depth, n)) || (e = alloc(&g->sigma, n)) || (e = alloc(&g->du, n)) ||
         (e = alloc(&g->gacc, n)) || (e = alloc(&g->list_v, n + 1)) || (e = alloc(&g->list_pre, n + 1)) ||
         (e = alloc(&g->list_beg, n + 1)) ||
-        (e = alloc(&g->tiles, list_tiles)) || (e = alloc(&g->lvl, 5 * (n + 2))) || (e = alloc(&g->ctr, 1)) ||
+        (e = alloc(&g->tiles, list_tiles)) || (e = alloc(&g->lvl, kLvlWords * (n + 2))) || (e = alloc(&g->ctr, 1)) ||
         (e = alloc(&g->trace, 8 * kTraceCap)))
         return cuda_error(e, "workspace cudaMalloc");
+    if (g->directed && g->engine == TBC_ENGINE_CSC) {
+        if ((e = alloc(&g->ilist_v, n + 1)) || (e = alloc(&g->ilist_pre, n + 1)) ||
+            (e = alloc(&g->ilist_beg, n + 1)) || (e = alloc(&g->itiles, list_tiles)))
+            return cuda_error(e, "workspace cudaMalloc");
+    }
     {
         for (int b = 0; b < 2; ++b)
             if ((e = alloc(&g->cand_v[b], n + 1)) || (e = alloc(&g->cand_pre[b], n + 1)) ||
@@ -1065,6 +1157,20 @@ tbc_status engine_setup(tbc_graph *g) {
         (e = cudaMemsetAsync(g->gacc, 0, sizeof(double) * n, s)) ||
         (e = cudaMemsetAsync(g->ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s)))
         return cuda_error(e, "workspace init");
+    {  // vertices that can have in-edges: [0, n_scan); count of in-degree > 0 (scan cost model)
+        unsigned long long *d_cnt = nullptr;
+        if ((e = cudaMalloc(&d_cnt, 2 * sizeof(unsigned long long))) ||
+            (e = cudaMemsetAsync(d_cnt, 0, 2 * sizeof(unsigned long long), s)))
+            return cuda_error(e, "scan range");
+        k_in_range<<<(int)((n + 255) / 256), 256, 0, s>>>(n, g->deg2, d_cnt);
+        unsigned long long h[2] = {0, 0};
+        e = cudaMemcpyAsync(h, d_cnt, sizeof h, cudaMemcpyDeviceToHost, s);
+        if (!e) e = cudaStreamSynchronize(s);
+        cudaFree(d_cnt);
+        if (e) return cuda_error(e, "scan range");
+        g->n_scan = (int64_t)h[0];
+        g->n_in = (int64_t)h[1];
+    }
     int per_sm = 0, sms = 0;
     if ((e = cudaFuncSetAttribute(k_bc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes)) ||
         (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_bc, kBlock, kSmemBytes)) ||
@@ -1102,6 +1208,16 @@ tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
     P.c_atom = g->c_atom;
     P.c_vert = g->c_vert;
     P.tiles = g->tiles;
+    P.in_list = g->ilist_v != nullptr;
+    P.ilist_v = P.in_list ? g->ilist_v : g->list_v;
+    P.ilist_pre = P.in_list ? g->ilist_pre : g->list_pre;
+    P.ilist_beg = P.in_list ? g->ilist_beg : g->list_beg;
+    P.itiles = P.in_list ? g->itiles : g->tiles;
+    P.n_scan = g->n_scan;
+    P.n_in = g->n_in;
+    P.c_scan = g->c_scan;
+    P.c_bpush = g->c_bpush;
+    P.bwd_mode = g->bwd_mode;
     for (int b = 0; b < 2; ++b) {
         P.cand_v[b] = g->cand_v[b];
         P.cand_pre[b] = g->cand_pre[b];

@@ -21,6 +21,7 @@ constexpr int64_t kTraceCap = 65536; // trace entries (one per barrier of the tr
 struct Ctrs {
     unsigned long long list;      // packed (count << ebits) | edge_sum of the BFS-order list
     unsigned long long cand[2];   // packed counters of the two pull-candidate buffers
+    unsigned long long ilist;     // packed (count << ebits) | in-edge sum of the in-degree list (directed)
     unsigned int bar_count;       // grid barrier arrival counter
     unsigned int bar_gen;         // grid barrier generation
     unsigned long long bad_sources;
@@ -45,11 +46,20 @@ struct Params {
     int64_t *list_pre;                    // exclusive out-degree prefix along list_v
     int64_t *list_beg;                    // out_ptr[v] of each list entry (written at append)
     int32_t *tiles;                       // per level: owner index starting each tile
+    // in-degree list (directed CSC engine): the same vertices per level as list_*, keyed by
+    // in-degree (prefix over in_ptr) -- the owners of the backward push pass; == list_* otherwise
+    int32_t *ilist_v;
+    int64_t *ilist_pre;
+    int64_t *ilist_beg;
+    int32_t *itiles;
+    int in_list;                          // 1: ilist_* is a separate list appended beside list_*
+    int64_t n_scan;                       // vertices [0, n_scan) can have in-edges (degree-sorted labels)
+    int64_t n_in;                         // vertices with in-degree > 0
     int32_t *cand_v[2];                   // pull candidate buffers
     int64_t *cand_pre[2];
     int64_t *cand_beg[2];
     int32_t *cand_tiles[2];
-    int64_t *lvl;                         // per level: p0, N, e0, E, tile_base
+    int64_t *lvl;                         // per level: p0, N, e0, E, tile_base, ie0, IE, itile_base
     Ctrs *ctr;
     double *bc;                           // indexed by caller labels
     const int32_t *sources;               // caller labels
@@ -62,6 +72,7 @@ struct Params {
     int directed;
     int coot;                             // TBC_ENGINE_COOT: edge-stream passes only
     int dir_mode;                         // 0 auto, 1 push only, 2 pull whenever possible
+    int bwd_mode;                         // 0 auto, 1 pull only, 2 push whenever possible
     int64_t *trace;                       // per-level timeline of one source (8 int64 per entry)
     int64_t trace_cap, trace_src;
     // edge-stream passes (the scCOOC form of Alg. 2): owner of every stored entry
@@ -69,6 +80,7 @@ struct Params {
     const int32_t *__restrict__ out_row;  // row of each CSR entry (sorted); nullptr for COO^T directed
     int fmt_mode;                         // 0 auto, 1 list passes only, 2 stream passes only
     double c_list, c_stream, c_atom, c_vert;  // per-item cost model (ps) for the per-level choice
+    double c_scan, c_bpush;
 };
 
 }  // namespace tbc
@@ -96,6 +108,11 @@ struct tbc_graph {
     int64_t *list_pre = nullptr;
     int64_t *list_beg = nullptr;
     int32_t *tiles = nullptr;
+    int32_t *ilist_v = nullptr;   // in-degree list (directed CSC engine only)
+    int64_t *ilist_pre = nullptr;
+    int64_t *ilist_beg = nullptr;
+    int32_t *itiles = nullptr;
+    int64_t n_scan = 0, n_in = 0;
     int32_t *cand_v[2] = {nullptr, nullptr};
     int64_t *cand_pre[2] = {nullptr, nullptr};
     int64_t *cand_beg[2] = {nullptr, nullptr};
@@ -109,8 +126,9 @@ struct tbc_graph {
     int grid = 0;
     int ebits = 38;
     int dir_mode = 0;
+    int bwd_mode = 0;
     int fmt_mode = 0;
-    double c_list = 12.0, c_stream = 4.0, c_atom = 18.0, c_vert = 10.0;
+    double c_list = 12.0, c_stream = 4.0, c_atom = 18.0, c_vert = 10.0, c_scan = 3.0, c_bpush = 6.0;
     int64_t *trace = nullptr;     // device, 8 * kTraceCap int64
     int64_t trace_src = -1;       // index in the next call's source list to trace (-1: off)
     cudaStream_t stream = nullptr;  // internal stream for the synchronous host API

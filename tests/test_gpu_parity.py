@@ -13,14 +13,18 @@ import paper_conf_icppw_artiless21_b200 as tbc
 
 pytestmark = pytest.mark.gpu
 
-# (direction, format) pairs: every forward/backward pass kind gets exercised
-MODES = [(tbc.DIR_AUTO, tbc.FMT_AUTO), (tbc.DIR_PUSH, tbc.FMT_LIST), (tbc.DIR_PUSH, tbc.FMT_STREAM),
-         (tbc.DIR_PULL, tbc.FMT_AUTO), (tbc.DIR_PULL, tbc.FMT_STREAM)]
+# (forward direction, format, backward direction) triples: every forward/backward pass kind
+# gets exercised -- (PULL, LIST) forces the candidate scan + list pull after the first push
+# level; backward 1 = pull over level L's out-edges only, 2 = push from level L+1 (in-edges)
+MODES = [(tbc.DIR_AUTO, tbc.FMT_AUTO, 0), (tbc.DIR_PUSH, tbc.FMT_LIST, 1), (tbc.DIR_PUSH, tbc.FMT_STREAM, 0),
+         (tbc.DIR_PULL, tbc.FMT_AUTO, 0), (tbc.DIR_PULL, tbc.FMT_STREAM, 0), (tbc.DIR_PULL, tbc.FMT_LIST, 2),
+         (tbc.DIR_AUTO, tbc.FMT_LIST, 2)]
 
 
 def set_mode(G, mode):
     G.set_direction(mode[0])
     G.set_format(mode[1])
+    G.set_bwd_direction(mode[2] if len(mode) > 2 else 0)
 
 
 def assert_bc(got, want, rel=1e-9):
@@ -57,7 +61,7 @@ SMALL = [gg.star(7), gg.star(7, directed_both=True), gg.path(7), gg.path(7, dire
 
 
 @pytest.mark.parametrize("engine", ENGINES)
-@pytest.mark.parametrize("mode", MODES, ids=lambda m: f"dir{m[0]}fmt{m[1]}")
+@pytest.mark.parametrize("mode", MODES, ids=lambda m: f"dir{m[0]}fmt{m[1]}bwd{m[2]}")
 @pytest.mark.parametrize("g", SMALL, ids=lambda g: g.name)
 def test_small_graphs_all_sources(g, mode, engine):
     with gpu_graph(g, engine=engine, reorder=(mode[1] != tbc.FMT_LIST)) as G:
@@ -226,6 +230,11 @@ def test_cfg3_kron22_directed_sample_in_bench_launch_config():
         assert_bc(G.bc(sample), want)
         for s in sample[:2]:
             assert_bfs(g, G, s)
+        for mode in [(tbc.DIR_AUTO, tbc.FMT_AUTO, 1), (tbc.DIR_AUTO, tbc.FMT_AUTO, 2),
+                     (tbc.DIR_PULL, tbc.FMT_LIST, 2), (tbc.DIR_PUSH, tbc.FMT_LIST, 0)]:
+            set_mode(G, mode)
+            assert_bc(G.bc(sample[:4]), oracle.bc(g.col_ptr, g.row_idx, True, sample[:4]))
+        set_mode(G, MODES[0])
         # per-source invariant at any size: sum_v bc_s(v) = sum_t (depth_s(t) - 1)
         s = int(src[100])
         depth, _ = G.bfs(s)

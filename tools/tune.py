@@ -1,0 +1,60 @@
+"""Tuning helper (GPU): time option settings of the engine on a config and dump per-level traces.
+
+    python tools/tune.py --config 3 --sources 256 --settings "fmt=0;fmt=1;fmt=2" --trace 0,1
+Each setting is a comma list of key=value: fmt, dir, list, stream, atomic, vertex (cost model, ps).
+Prints one JSON line per setting (ms/source, GTEPS) and TRACE lines for the traced sources.
+"""
+import argparse
+import json
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+import graphgen as gg  # noqa: E402
+import paper_conf_icppw_artiless21_b200 as tbc  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", type=int, default=3)
+ap.add_argument("--sources", type=int, default=256)
+ap.add_argument("--settings", default="fmt=0")
+ap.add_argument("--trace", default="")
+ap.add_argument("--reps", type=int, default=2)
+a = ap.parse_args()
+
+g, _ = gg.make_config(a.config, device="cuda")
+src = gg.sources(g, a.sources, seed=gg.CONFIGS[a.config]["src_seed"])
+G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed)
+s_d = torch.from_numpy(src).cuda()
+bc = torch.zeros(g.n, dtype=torch.float64, device="cuda")
+st = torch.cuda.current_stream()
+for setting in a.settings.split(";"):
+    kv = dict(x.split("=") for x in setting.split(",") if x)
+    G.set_format(int(kv.get("fmt", 0)))
+    G.set_direction(int(kv.get("dir", 0)))
+    G.set_cost(**{k: float(v) for k, v in kv.items() if k in ("list", "stream", "atomic", "vertex")})
+    G.bc_device(s_d, bc, st)  # warm-up
+    torch.cuda.synchronize()
+    G.reset_stats()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(st)
+    for _ in range(a.reps):
+        G.bc_device(s_d, bc, st)
+    e1.record(st)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / a.reps
+    s = G.stats()
+    print(json.dumps({"setting": setting, "ms_per_source": ms / a.sources,
+                      "gteps": a.sources * g.nnz / (ms / 1e3) / 1e9,
+                      "fwd_edges_per_src": s["fwd_edges"] / max(s["sources"], 1),
+                      "bwd_edges_per_src": s["bwd_edges"] / max(s["sources"], 1),
+                      "pull_levels": s["pull_levels"] / max(s["sources"], 1)}), flush=True)
+    for t in [int(x) for x in a.trace.split(",") if x]:
+        G.set_trace(t)
+        G.bc(src[: t + 1])
+        for r in G.trace():
+            print("TRACE " + json.dumps({"setting": setting, "src": t, **r}), flush=True)
+        G.set_trace(-1)
+    G.set_cost(list=12, stream=4, atomic=18, vertex=10)
+G.close()

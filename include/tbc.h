@@ -84,7 +84,13 @@ enum {
     TBC_OPT_COST_ATOMIC = 7, /*   push contribution (fp64 atomic) (default 18) */
     TBC_OPT_COST_VERTEX = 8, /*   vertex of a whole-graph owner pass (default 10) */
     TBC_OPT_COST_SCAN = 9,   /*   vertex of a candidate scan before a pull that follows a push (default 3) */
-    TBC_OPT_COST_BPUSH = 10  /*   extra per in-edge of a backward push level over a list item (default 6) */
+    TBC_OPT_COST_BPUSH = 10, /*   extra per in-edge of a backward push level over a list item (default 6) */
+    TBC_OPT_PARTITIONS = 11  /* SM partitions (1..8, default 8): the source list is dealt round-robin
+                                to this many disjoint groups of SMs, each running its sources with its
+                                own workspace and partition-local barriers; the partial bc vectors
+                                are summed in partition order at the end of the call (deterministic
+                                for a given value).  Costs one workspace (~50 B/vertex + 8 B/edge/64)
+                                per partition. */
 };
 
 /* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since

@@ -24,7 +24,7 @@ __all__ = ["Graph", "TBCError", "lib", "ENGINE_CSC", "ENGINE_COOT", "DIR_AUTO", 
 
 ENGINE_CSC, ENGINE_COOT = 0, 1
 FLAG_ONE_FORMAT, FLAG_NO_VALIDATE, FLAG_NO_REORDER = 1, 2, 4
-OPT_DIRECTION, OPT_BWD_DIRECTION, OPT_TRACE, OPT_FORMAT = 1, 2, 3, 4
+OPT_DIRECTION, OPT_BWD_DIRECTION, OPT_TRACE, OPT_FORMAT, OPT_PARTITIONS = 1, 2, 3, 4, 11
 OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8, "scan": 9, "bpush": 10}
 FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
 DIR_AUTO, DIR_PUSH, DIR_PULL = 0, 1, 2
@@ -161,6 +161,10 @@ class Graph:
     def set_bwd_direction(self, mode: int):
         """Backward levels: 0 auto, 1 pull over level L's out-edges only, 2 push from level L+1 when possible."""
         _check(lib().tbc_graph_set_option(self._h, OPT_BWD_DIRECTION, float(mode)))
+
+    def set_partitions(self, parts: int):
+        """Number of SM partitions running sources concurrently (1..8; TBC_OPT_PARTITIONS)."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_PARTITIONS, float(parts)))
 
     def set_format(self, mode: int):
         """0 auto, 1 list passes only, 2 edge-stream passes only."""

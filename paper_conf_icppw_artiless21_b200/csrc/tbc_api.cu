@@ -187,27 +187,7 @@ void free_graph(tbc_graph *g) {
     cudaFree(g->inv);
     cudaFree(g->in_col);
     if (g->out_row != g->in_col) cudaFree(g->out_row);
-    cudaFree(g->depth);
-    cudaFree(g->sigma);
-    cudaFree(g->du);
-    cudaFree(g->gacc);
-    cudaFree(g->list_v);
-    cudaFree(g->list_pre);
-    cudaFree(g->list_beg);
-    cudaFree(g->tiles);
-    cudaFree(g->ilist_v);
-    cudaFree(g->ilist_pre);
-    cudaFree(g->ilist_beg);
-    cudaFree(g->itiles);
-    for (int b = 0; b < 2; ++b) {
-        cudaFree(g->cand_v[b]);
-        cudaFree(g->cand_pre[b]);
-        cudaFree(g->cand_beg[b]);
-        cudaFree(g->cand_tiles[b]);
-    }
-    cudaFree(g->lvl);
-    cudaFree(g->ctr);
-    cudaFree(g->trace);
+    engine_free(g);
     cudaFree(g->bc_tmp);
     cudaFree(g->src_tmp);
     if (g->stream) cudaStreamDestroy(g->stream);
@@ -532,6 +512,13 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->fmt_mode = v;
         return TBC_OK;
     }
+    if (key == TBC_OPT_PARTITIONS) {
+        int v = (int)value;
+        if (v < 1 || v > kMaxPartitions || (double)v != value)
+            return set_error(TBC_ERR_INVALID, "partitions %g not in [1, %d]", value, kMaxPartitions);
+        g->nparts = v;
+        return TBC_OK;
+    }
     if (key == TBC_OPT_BWD_DIRECTION) {
         int v = (int)value;
         if (v < 0 || v > 2 || (double)v != value) return set_error(TBC_ERR_INVALID, "bwd direction %g", value);
@@ -603,14 +590,15 @@ tbc_status tbc_bfs(tbc_graph *g, int32_t source, int32_t *depth_out, double *sig
     st = engine_run(g, g->src_tmp, 1, nullptr, g->stream, 1);
     if (st != TBC_OK) return st;
     {
-        const int32_t *dsrc = g->depth;
-        const double *ssrc = g->sigma;
+        const Workspace &w = g->ws[0];  // a forward-only run uses partition 0
+        const int32_t *dsrc = w.depth;
+        const double *ssrc = w.sigma;
         if (g->perm) {  // back to the caller's labels (list_v / bc_tmp are free scratch here)
             if (!g->bc_tmp) TBC_CUDA(dmalloc(g, &g->bc_tmp, g->n));
-            k_unpermute_bfs<<<grid_for(g->n), 256, 0, g->stream>>>(g->n, g->perm, g->depth, g->sigma, g->list_v,
+            k_unpermute_bfs<<<grid_for(g->n), 256, 0, g->stream>>>(g->n, g->perm, w.depth, w.sigma, w.list_v,
                                                                    g->bc_tmp);
             TBC_CUDA(cudaGetLastError());
-            dsrc = g->list_v;
+            dsrc = w.list_v;
             ssrc = g->bc_tmp;
         }
         if (depth_out)
@@ -619,8 +607,8 @@ tbc_status tbc_bfs(tbc_graph *g, int32_t source, int32_t *depth_out, double *sig
             TBC_CUDA(cudaMemcpyAsync(sigma_out, ssrc, sizeof(double) * g->n, cudaMemcpyDeviceToHost, g->stream));
     }
     // forward-only runs leave depth/sigma set: restore the all-unvisited workspace invariant
-    TBC_CUDA(cudaMemsetAsync(g->depth, 0xff, sizeof(int32_t) * g->n, g->stream));
-    TBC_CUDA(cudaMemsetAsync(g->sigma, 0, sizeof(double) * g->n, g->stream));
+    TBC_CUDA(cudaMemsetAsync(g->ws[0].depth, 0xff, sizeof(int32_t) * g->n, g->stream));
+    TBC_CUDA(cudaMemsetAsync(g->ws[0].sigma, 0, sizeof(double) * g->n, g->stream));
     TBC_CUDA(cudaStreamSynchronize(g->stream));
     return TBC_OK;
 fail:
@@ -633,16 +621,19 @@ tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
     Ctrs c;
     TBC_CUDA(cudaSetDevice(g->device));
     TBC_CUDA(cudaDeviceSynchronize());
-    TBC_CUDA(cudaMemcpy(&c, g->ctr, sizeof c, cudaMemcpyDeviceToHost));
-    out->sources = c.st_sources;
-    out->reached = c.st_reached;
-    out->reached_edges = c.st_reached_edges;
-    out->fwd_edges = c.st_fwd_edges;
-    out->bwd_edges = c.st_bwd_edges;
-    out->levels = c.st_levels;
-    out->pull_levels = c.st_pull_levels;
-    out->scans = c.st_scans;
-    out->max_depth = c.st_max_depth;
+    *out = tbc_stats{};
+    for (int i = 0; i < g->ws_count; ++i) {  // summed over the SM partitions' counters
+        TBC_CUDA(cudaMemcpy(&c, g->ws[i].ctr, sizeof c, cudaMemcpyDeviceToHost));
+        out->sources += c.st_sources;
+        out->reached += c.st_reached;
+        out->reached_edges += c.st_reached_edges;
+        out->fwd_edges += c.st_fwd_edges;
+        out->bwd_edges += c.st_bwd_edges;
+        out->levels += c.st_levels;
+        out->pull_levels += c.st_pull_levels;
+        out->scans += c.st_scans;
+        if (c.st_max_depth > out->max_depth) out->max_depth = c.st_max_depth;
+    }
     return TBC_OK;
 fail:
     return st;
@@ -655,7 +646,7 @@ tbc_status tbc_trace_get(tbc_graph *g, int64_t *out, int64_t cap, int64_t *count
     int64_t nrec = 0;
     TBC_CUDA(cudaSetDevice(g->device));
     TBC_CUDA(cudaDeviceSynchronize());
-    TBC_CUDA(cudaMemcpy(&c, g->ctr, sizeof c, cudaMemcpyDeviceToHost));
+    TBC_CUDA(cudaMemcpy(&c, g->gctr, sizeof c, cudaMemcpyDeviceToHost));
     nrec = (int64_t)c.trace_n;
     if (nrec > kTraceCap) nrec = kTraceCap;
     *count = nrec;
@@ -671,7 +662,8 @@ tbc_status tbc_stats_reset(tbc_graph *g) {
     tbc_status st = TBC_OK;
     TBC_CUDA(cudaSetDevice(g->device));
     TBC_CUDA(cudaDeviceSynchronize());
-    TBC_CUDA(cudaMemset(&g->ctr->st_sources, 0, sizeof(long long) * 9));
+    for (int i = 0; i < g->ws_count; ++i)
+        TBC_CUDA(cudaMemset(&g->ws[i].ctr->st_sources, 0, sizeof(long long) * 9));
     return TBC_OK;
 fail:
     return st;

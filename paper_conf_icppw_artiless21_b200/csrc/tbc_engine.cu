@@ -136,13 +136,13 @@ constexpr unsigned long long kWatchdogNs = 20ull * 1000 * 1000 * 1000;  // 20 s 
 // Grid-wide barrier of the cooperative (co-resident) grid: release fence + arrival atomic,
 // the last arriver bumps the generation; waiters acquire it.  The acquire-side gpu fence also
 // invalidates this SM's L1, so plain loads after the barrier see other CTAs' writes.
-__device__ __forceinline__ void grid_sync(Ctrs *c, unsigned &gen) {
+__device__ __forceinline__ void grid_sync(Ctrs *c, unsigned &gen, unsigned nblocks) {
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned g0 = gen;
         fence_acq_rel();
         const unsigned arrived = atomicAdd(&c->bar_count, 1u);
-        if (arrived == gridDim.x - 1) {
+        if (arrived == nblocks - 1) {
             c->bar_count = 0;
             fence_acq_rel();
             atomicExch(&c->bar_gen, g0 + 1);
@@ -209,16 +209,24 @@ __device__ __forceinline__ void warp_append(const bool (&take)[kLaneItems], cons
             const uint32_t t = __shfl_up_sync(FULL, inc, k);
             if (lane >= k) inc += t;
         }
+        const int64_t pp = p + __popc(msk & lt);
+        const int64_t ee = e + (int64_t)(inc - x);
+        const int64_t k0 = (ee - o.e0) + (pp - o.p0);
+        const int64_t t0 = (k0 + kWT - 1) / kWT, t1 = (k0 + x) / kWT;
+        const bool wide = take[i] && t1 - t0 >= 8;  // a hub: the whole warp writes its tile starts
         if (take[i]) {
-            const int64_t pp = p + __popc(msk & lt);
-            const int64_t ee = e + (int64_t)(inc - x);
             TBC_CHECK(v[i] >= 0, "append v %d", v[i]);
             o.v[pp] = v[i];
             o.pre[pp] = ee;
             o.beg[pp] = bg[i];
-            const int64_t k0 = (ee - o.e0) + (pp - o.p0);
-            const int64_t k1 = k0 + x;
-            for (int64_t t = (k0 + kWT - 1) / kWT; t <= k1 / kWT; ++t) o.tiles[t] = (int32_t)(pp - o.p0);
+            if (!wide)
+                for (int64_t t = t0; t <= t1; ++t) o.tiles[t] = (int32_t)(pp - o.p0);
+        }
+        for (unsigned wm = __ballot_sync(FULL, wide); wm; wm &= wm - 1) {
+            const int src = __ffs(wm) - 1;
+            const int64_t a = __shfl_sync(FULL, t0, src), b = __shfl_sync(FULL, t1, src);
+            const int32_t val = (int32_t)(__shfl_sync(FULL, pp, src) - o.p0);
+            for (int64_t t = a + lane; t <= b; t += 32) o.tiles[t] = val;
         }
         p += __popc(msk);
         e += __shfl_sync(FULL, inc, 31);
@@ -850,26 +858,43 @@ enum { TR_INIT = 0, TR_SCAN = 1, TR_PUSH = 2, TR_PULL = 3, TR_BWD = 4, TR_OWNER 
 
 __device__ __forceinline__ void trace(const Params &P, bool on, int kind, int64_t level, int64_t N, int64_t E,
                                       int64_t a, int64_t b) {
-    if (!on || blockIdx.x != 0 || threadIdx.x != 0) return;
-    const unsigned long long i = P.ctr->trace_n;
+    if (!on || (int)blockIdx.x != P.cta_base || threadIdx.x != 0) return;
+    const unsigned long long i = P.gctr->trace_n;
     if ((int64_t)i >= P.trace_cap) return;
     int64_t *t = P.trace + 8 * i;
     t[0] = (int64_t)globaltimer_ns(); t[1] = kind; t[2] = level; t[3] = N; t[4] = E; t[5] = a; t[6] = b; t[7] = 0;
-    P.ctr->trace_n = i + 1;
+    P.gctr->trace_n = i + 1;
 }
 
 // ------------------------------------------------------------------ the persistent kernel
 
-__global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
+// the launch: one Params per SM partition (workspace pointers, CTA range), plus the shared
+// counters (full-grid barrier, trace) and the caller's bc for the final partition reduction
+constexpr int kMaxParts = 8;
+struct ParamSet {
+    Params p[kMaxParts];
+    int nparts, cta_per_part;
+    Ctrs *gctr;
+    double *bc_out;
+};
+
+__global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamSet S) {
     extern __shared__ __align__(16) unsigned char dyn_smem[];
     WarpSmem &ws = reinterpret_cast<WarpSmem *>(dyn_smem)[threadIdx.x >> 5];
-    const int64_t nwarps = (int64_t)gridDim.x * kWarpsPerBlock;
-    const int64_t gwarp = (int64_t)blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
+    // SM partition of this CTA: partition `part` runs sources part, part + nparts, ... on its
+    // own workspace with its own (partition-local) grid barrier
+    const int part = (int)blockIdx.x / S.cta_per_part;
+    const Params &P = S.p[part];
+    const int lcta = (int)blockIdx.x - P.cta_base;
+    const unsigned ncta = (unsigned)S.cta_per_part;
+    const int64_t nwarps = (int64_t)ncta * kWarpsPerBlock;
+    const int64_t gwarp = (int64_t)lcta * kWarpsPerBlock + (threadIdx.x >> 5);
     const int tid = threadIdx.x;
-    const bool cta0 = blockIdx.x == 0;
-    const int64_t nthreads = (int64_t)gridDim.x * kBlock;
-    const int64_t gtid = (int64_t)blockIdx.x * kBlock + tid;
+    const bool cta0 = lcta == 0;
+    const int64_t nthreads = (int64_t)ncta * kBlock;
+    const int64_t gtid = (int64_t)lcta * kBlock + tid;
     Ctrs *C = P.ctr;
+    unsigned gen_all = (tid == 0) ? ld_acquire(&S.gctr->bar_gen) : 0u;
     // barrier generation: only thread 0 uses it (the first barrier cannot complete before
     // every CTA has read the current value, so reading it here is race-free)
     unsigned gen = (tid == 0) ? ld_acquire(&C->bar_gen) : 0u;
@@ -878,7 +903,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
     // the in-degree list: a separate list for directed graphs, the out-list itself otherwise
     unsigned long long *ictr = P.in_list ? &C->ilist : &C->list;
 
-    for (int64_t si = 0; si < P.k; ++si) {
+    for (int64_t si = part; si < P.k; si += S.nparts) {
         const int32_t s_caller = P.sources[si];
         if (s_caller < 0 || s_caller >= P.n) {
             if (cta0 && tid == 0) atomicAdd(&C->bad_sources, 1ull);
@@ -910,14 +935,14 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
                 }
                 C->cand[0] = 0;
                 C->cand[1] = 0;
-                if (tr) C->trace_n = 0;
+                if (tr) P.gctr->trace_n = 0;
             }
             for (int64_t i = tid; i <= dego / kWT; i += kBlock) P.tiles[i] = 0;
             if (P.in_list)
                 for (int64_t i = tid; i <= degi / kWT; i += kBlock) P.itiles[i] = 0;
         }
         prev_s = s;
-        grid_sync(C, gen);
+        grid_sync(C, gen, ncta);
         trace(P, tr, TR_INIT, 0, 1, dego, s, 0);
 
         // level d-1 (frontier)
@@ -968,7 +993,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
                     // candidate list cb is empty here (reset by the push level before its barrier)
                     const ListOut sc{&C->cand[cb], P.cand_v[cb], P.cand_pre[cb], P.cand_beg[cb], P.cand_tiles[cb], 0, 0};
                     cand_scan_pass(P, gwarp, nwarps, sc);
-                    grid_sync(C, gen);
+                    grid_sync(C, gen, ncta);
                     const unsigned long long cv = ld_volatile_u64(&C->cand[cb]);
                     candN = (int64_t)(cv >> P.ebits);
                     candE = (int64_t)(cv & emask);
@@ -986,7 +1011,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
                     edge_pass<MODE_PULL>(P, ws, P.cand_v[cb], P.cand_pre[cb], P.cand_beg[cb], P.cand_tiles[cb], candN,
                                          candE, 0, P.in_ptr, P.in_idx, d, gwarp, nwarps, lo, li);
                 }
-                grid_sync(C, gen);
+                grid_sync(C, gen, ncta);
                 trace(P, tr, TR_PULL, d, candN, candE, stream, 0);
                 // owner pass: the survivors of a stream pull are all undiscovered vertices
                 pull_owner_pass(P, stream ? nullptr : P.cand_v[cb], candN, d, gwarp, nwarps, lo, li, co);
@@ -1007,7 +1032,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
                 }
                 cand_valid = false;
             }
-            grid_sync(C, gen);
+            grid_sync(C, gen, ncta);
             {
                 const unsigned long long lv = ld_volatile_u64(&C->list);
                 nxt.N = (int64_t)(lv >> P.ebits) - nxt.p0;
@@ -1085,11 +1110,11 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
                                           P.in_ptr, P.in_idx, L, gwarp, nwarps, none, none);
                     bwd_edges += up.IE;
                 }
-                grid_sync(C, gen);
+                grid_sync(C, gen, ncta);
                 trace(P, tr, TR_BWD, L, lv.N, lv.E, bsel, 0);
             }
             bwd_owner_pass(P, P.list_v + lv.p0, lv.N, L, gtid, nthreads);
-            grid_sync(C, gen);
+            grid_sync(C, gen, ncta);
             trace(P, tr, TR_OWNER, L, lv.N, lv.E, 1, 0);
             up = lv;
         }
@@ -1099,6 +1124,21 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(Params P) {
     if (!P.bfs_only && cta0 && tid == 0 && prev_s >= 0) {
         P.depth[prev_s] = -1;
         P.sigma[prev_s] = 0.0;
+    }
+    if (S.nparts > 1 && !P.bfs_only) {
+        // every partition done: bc_out += the partitions' partial bc in partition order
+        // (deterministic), and the partials return to zero for the next call
+        grid_sync(S.gctr, gen_all, gridDim.x);
+        const int64_t nt = (int64_t)gridDim.x * kBlock;
+        for (int64_t v = (int64_t)blockIdx.x * kBlock + tid; v < P.n; v += nt) {
+            double sum = 0.0;
+            for (int q = 0; q < S.nparts; ++q) {
+                double *bq = S.p[q].bc;
+                sum += bq[v];
+                bq[v] = 0.0;
+            }
+            if (sum != 0.0) S.bc_out[v] += sum;
+        }
     }
 }
 
@@ -1115,48 +1155,98 @@ __global__ void k_in_range(int64_t n, const int2 *__restrict__ deg2, unsigned lo
     if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&out[1], (unsigned long long)__popc(m));
 }
 
-tbc_status engine_setup(tbc_graph *g) {
+tbc_status engine_workspaces(tbc_graph *g, int count) {
     const int64_t n = g->n, m = g->m;
     cudaStream_t s = g->stream;
-    cudaError_t e;
-    auto alloc = [&](auto **p, size_t count) -> cudaError_t {
-        size_t bytes = sizeof(**p) * (count > 0 ? count : 1);
+    cudaError_t e = cudaSuccess;
+    auto alloc = [&](auto **p, size_t cnt) -> cudaError_t {
+        size_t bytes = sizeof(**p) * (cnt > 0 ? cnt : 1);
         cudaError_t r = cudaMalloc((void **)p, bytes);
         if (r == cudaSuccess) g->device_bytes += bytes;
         return r;
     };
+    const int64_t list_tiles = (n + m) / kWT + n + 2;
+    const int64_t cand_tiles = (n + m) / kWT + 2;
+    for (int i = g->ws_count; i < count; ++i) {
+        Workspace &w = g->ws[i];
+        g->ws_count = i + 1;  // engine_free releases whatever of it was allocated
+        if ((e = alloc(&w.depth, n)) || (e = alloc(&w.sigma, n)) || (e = alloc(&w.du, n)) ||
+            (e = alloc(&w.gacc, n)) || (e = alloc(&w.list_v, n + 1)) || (e = alloc(&w.list_pre, n + 1)) ||
+            (e = alloc(&w.list_beg, n + 1)) || (e = alloc(&w.tiles, list_tiles)) ||
+            (e = alloc(&w.lvl, kLvlWords * (n + 2))) || (e = alloc(&w.ctr, 1)))
+            return cuda_error(e, "workspace cudaMalloc");
+        if (g->directed && g->engine == TBC_ENGINE_CSC) {
+            if ((e = alloc(&w.ilist_v, n + 1)) || (e = alloc(&w.ilist_pre, n + 1)) ||
+                (e = alloc(&w.ilist_beg, n + 1)) || (e = alloc(&w.itiles, list_tiles)))
+                return cuda_error(e, "workspace cudaMalloc");
+        }
+        for (int b = 0; b < 2; ++b)
+            if ((e = alloc(&w.cand_v[b], n + 1)) || (e = alloc(&w.cand_pre[b], n + 1)) ||
+                (e = alloc(&w.cand_beg[b], n + 1)) || (e = alloc(&w.cand_tiles[b], cand_tiles)))
+                return cuda_error(e, "workspace cudaMalloc");
+        if ((e = alloc(&w.bc_part, n))) return cuda_error(e, "workspace cudaMalloc");
+        if ((e = cudaMemsetAsync(w.depth, 0xff, sizeof(int32_t) * n, s)) ||
+            (e = cudaMemsetAsync(w.sigma, 0, sizeof(double) * n, s)) ||
+            (e = cudaMemsetAsync(w.du, 0, sizeof(double) * n, s)) ||
+            (e = cudaMemsetAsync(w.gacc, 0, sizeof(double) * n, s)) ||
+            (e = cudaMemsetAsync(w.bc_part, 0, sizeof(double) * n, s)) ||
+            (e = cudaMemsetAsync(w.ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s)))
+            return cuda_error(e, "workspace init");
+    }
+    return TBC_OK;
+}
+
+void engine_free(tbc_graph *g) {
+    for (int i = 0; i < g->ws_count; ++i) {
+        Workspace &w = g->ws[i];
+        cudaFree(w.depth);
+        cudaFree(w.sigma);
+        cudaFree(w.du);
+        cudaFree(w.gacc);
+        cudaFree(w.list_v);
+        cudaFree(w.list_pre);
+        cudaFree(w.list_beg);
+        cudaFree(w.tiles);
+        cudaFree(w.ilist_v);
+        cudaFree(w.ilist_pre);
+        cudaFree(w.ilist_beg);
+        cudaFree(w.itiles);
+        for (int b = 0; b < 2; ++b) {
+            cudaFree(w.cand_v[b]);
+            cudaFree(w.cand_pre[b]);
+            cudaFree(w.cand_beg[b]);
+            cudaFree(w.cand_tiles[b]);
+        }
+        cudaFree(w.lvl);
+        cudaFree(w.ctr);
+        cudaFree(w.bc_part);
+        w = Workspace{};
+    }
+    g->ws_count = 0;
+    cudaFree(g->gctr);
+    cudaFree(g->trace);
+    g->gctr = nullptr;
+    g->trace = nullptr;
+}
+
+tbc_status engine_setup(tbc_graph *g) {
+    const int64_t n = g->n, m = g->m;
+    cudaStream_t s = g->stream;
+    cudaError_t e;
     // packed counters: high bits count (<= n), low bits edge sum (<= m)
     int cbits = 1;
     while ((1ll << cbits) <= n) ++cbits;
     g->ebits = 64 - cbits;
     if (g->ebits < 63 && (m >> g->ebits) != 0)
         return set_error(TBC_ERR_UNSUPPORTED, "nnz %lld too large for n %lld", (long long)m, (long long)n);
-    const int64_t list_tiles = (n + m) / kWT + n + 2;
-    const int64_t cand_tiles = (n + m) / kWT + 2;
-    if ((e = alloc(&g->depth, n)) || (e = alloc(&g->sigma, n)) || (e = alloc(&g->du, n)) ||
-        (e = alloc(&g->gacc, n)) || (e = alloc(&g->list_v, n + 1)) || (e = alloc(&g->list_pre, n + 1)) ||
-        (e = alloc(&g->list_beg, n + 1)) ||
-        (e = alloc(&g->tiles, list_tiles)) || (e = alloc(&g->lvl, kLvlWords * (n + 2))) || (e = alloc(&g->ctr, 1)) ||
-        (e = alloc(&g->trace, 8 * kTraceCap)))
+    if (m >= (1ll << 32))  // warp_append sums degrees of distinct vertices in 32 bits
+        return set_error(TBC_ERR_UNSUPPORTED, "nnz %lld >= 2^32", (long long)m);
+    if ((e = cudaMalloc(&g->gctr, sizeof(Ctrs))) || (e = cudaMalloc(&g->trace, sizeof(int64_t) * 8 * kTraceCap)))
         return cuda_error(e, "workspace cudaMalloc");
-    if (g->directed && g->engine == TBC_ENGINE_CSC) {
-        if ((e = alloc(&g->ilist_v, n + 1)) || (e = alloc(&g->ilist_pre, n + 1)) ||
-            (e = alloc(&g->ilist_beg, n + 1)) || (e = alloc(&g->itiles, list_tiles)))
-            return cuda_error(e, "workspace cudaMalloc");
-    }
-    {
-        for (int b = 0; b < 2; ++b)
-            if ((e = alloc(&g->cand_v[b], n + 1)) || (e = alloc(&g->cand_pre[b], n + 1)) ||
-                (e = alloc(&g->cand_beg[b], n + 1)) ||
-                (e = alloc(&g->cand_tiles[b], cand_tiles)))
-                return cuda_error(e, "workspace cudaMalloc");
-    }
-    if ((e = cudaMemsetAsync(g->depth, 0xff, sizeof(int32_t) * n, s)) ||
-        (e = cudaMemsetAsync(g->sigma, 0, sizeof(double) * n, s)) ||
-        (e = cudaMemsetAsync(g->du, 0, sizeof(double) * n, s)) ||
-        (e = cudaMemsetAsync(g->gacc, 0, sizeof(double) * n, s)) ||
-        (e = cudaMemsetAsync(g->ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s)))
-        return cuda_error(e, "workspace init");
+    g->device_bytes += sizeof(Ctrs) + sizeof(int64_t) * 8 * kTraceCap;
+    if ((e = cudaMemsetAsync(g->gctr, 0, sizeof(Ctrs), s))) return cuda_error(e, "workspace init");
+    tbc_status st = engine_workspaces(g, 1);
+    if (st != TBC_OK) return st;
     {  // vertices that can have in-edges: [0, n_scan); count of in-degree > 0 (scan cost model)
         unsigned long long *d_cnt = nullptr;
         if ((e = cudaMalloc(&d_cnt, 2 * sizeof(unsigned long long))) ||
@@ -1183,64 +1273,83 @@ tbc_status engine_setup(tbc_graph *g) {
 
 tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
                       int bfs_only) {
-    Params P{};
-    P.n = g->n;
-    P.m = g->m;
-    P.in_ptr = g->in_ptr;
-    P.in_idx = g->in_idx;
-    P.out_ptr = g->out_ptr;
-    P.out_idx = g->out_idx;
-    P.deg2 = g->deg2;
-    P.depth = g->depth;
-    P.sigma = g->sigma;
-    P.du = g->du;
-    P.gacc = g->gacc;
-    P.list_v = g->list_v;
-    P.list_pre = g->list_pre;
-    P.list_beg = g->list_beg;
-    P.directed = g->directed;
-    P.coot = g->engine == TBC_ENGINE_COOT;
-    P.in_col = g->in_col;
-    P.out_row = g->out_row;
-    P.fmt_mode = g->fmt_mode;
-    P.c_list = g->c_list;
-    P.c_stream = g->c_stream;
-    P.c_atom = g->c_atom;
-    P.c_vert = g->c_vert;
-    P.tiles = g->tiles;
-    P.in_list = g->ilist_v != nullptr;
-    P.ilist_v = P.in_list ? g->ilist_v : g->list_v;
-    P.ilist_pre = P.in_list ? g->ilist_pre : g->list_pre;
-    P.ilist_beg = P.in_list ? g->ilist_beg : g->list_beg;
-    P.itiles = P.in_list ? g->itiles : g->tiles;
-    P.n_scan = g->n_scan;
-    P.n_in = g->n_in;
-    P.c_scan = g->c_scan;
-    P.c_bpush = g->c_bpush;
-    P.bwd_mode = g->bwd_mode;
-    for (int b = 0; b < 2; ++b) {
-        P.cand_v[b] = g->cand_v[b];
-        P.cand_pre[b] = g->cand_pre[b];
-        P.cand_beg[b] = g->cand_beg[b];
-        P.cand_tiles[b] = g->cand_tiles[b];
+    // SM partitions: never more than the sources (a partition without sources only waits)
+    int np = g->nparts;
+    if (bfs_only || k < 1) np = 1;
+    if (np > k) np = (int)k;
+    if (np > g->grid) np = g->grid;
+    if (np < 1) np = 1;
+    tbc_status st = engine_workspaces(g, np);
+    if (st != TBC_OK) return st;
+    static_assert(sizeof(ParamSet) <= 32000, "kernel parameter space");
+    ParamSet S{};
+    S.nparts = np;
+    S.cta_per_part = g->grid / np;
+    S.gctr = g->gctr;
+    S.bc_out = d_bc;
+    for (int q = 0; q < np; ++q) {
+        const Workspace &w = g->ws[q];
+        Params &P = S.p[q];
+        P.n = g->n;
+        P.m = g->m;
+        P.in_ptr = g->in_ptr;
+        P.in_idx = g->in_idx;
+        P.out_ptr = g->out_ptr;
+        P.out_idx = g->out_idx;
+        P.deg2 = g->deg2;
+        P.depth = w.depth;
+        P.sigma = w.sigma;
+        P.du = w.du;
+        P.gacc = w.gacc;
+        P.list_v = w.list_v;
+        P.list_pre = w.list_pre;
+        P.list_beg = w.list_beg;
+        P.directed = g->directed;
+        P.coot = g->engine == TBC_ENGINE_COOT;
+        P.in_col = g->in_col;
+        P.out_row = g->out_row;
+        P.fmt_mode = g->fmt_mode;
+        P.c_list = g->c_list;
+        P.c_stream = g->c_stream;
+        P.c_atom = g->c_atom;
+        P.c_vert = g->c_vert;
+        P.tiles = w.tiles;
+        P.in_list = w.ilist_v != nullptr;
+        P.ilist_v = P.in_list ? w.ilist_v : w.list_v;
+        P.ilist_pre = P.in_list ? w.ilist_pre : w.list_pre;
+        P.ilist_beg = P.in_list ? w.ilist_beg : w.list_beg;
+        P.itiles = P.in_list ? w.itiles : w.tiles;
+        P.n_scan = g->n_scan;
+        P.n_in = g->n_in;
+        P.c_scan = g->c_scan;
+        P.c_bpush = g->c_bpush;
+        P.bwd_mode = g->bwd_mode;
+        for (int b = 0; b < 2; ++b) {
+            P.cand_v[b] = w.cand_v[b];
+            P.cand_pre[b] = w.cand_pre[b];
+            P.cand_beg[b] = w.cand_beg[b];
+            P.cand_tiles[b] = w.cand_tiles[b];
+        }
+        P.lvl = w.lvl;
+        P.ctr = w.ctr;
+        P.gctr = g->gctr;
+        P.cta_base = q * S.cta_per_part;
+        P.bc = np > 1 ? w.bc_part : d_bc;
+        P.perm = g->perm;
+        P.inv = g->inv;
+        P.sources = d_sources;
+        P.k = k;
+        P.bc_scale = g->directed ? 1.0 : 0.5;
+        P.ebits = g->ebits;
+        P.bfs_only = bfs_only;
+        P.dir_mode = g->dir_mode;
+        P.trace = g->trace;
+        P.trace_cap = g->trace ? kTraceCap : 0;
+        P.trace_src = g->trace_src;
     }
-    P.lvl = g->lvl;
-    P.ctr = g->ctr;
-    P.bc = d_bc;
-    P.perm = g->perm;
-    P.inv = g->inv;
-    P.sources = d_sources;
-    P.k = k;
-    P.bc_scale = g->directed ? 1.0 : 0.5;
-    P.ebits = g->ebits;
-    P.bfs_only = bfs_only;
-    P.dir_mode = g->dir_mode;
-    P.trace = g->trace;
-    P.trace_cap = g->trace ? kTraceCap : 0;
-    P.trace_src = g->trace_src;
-    void *args[] = {&P};
-    cudaError_t e = cudaLaunchCooperativeKernel((const void *)k_bc, dim3(g->grid), dim3(kBlock), args, kSmemBytes,
-                                                stream);
+    void *args[] = {&S};
+    cudaError_t e = cudaLaunchCooperativeKernel((const void *)k_bc, dim3(S.cta_per_part * np), dim3(kBlock), args,
+                                                kSmemBytes, stream);
     if (e != cudaSuccess) return cuda_error(e, "cudaLaunchCooperativeKernel(k_bc)");
     return TBC_OK;
 }

@@ -60,8 +60,11 @@ struct Params {
     int64_t *cand_beg[2];
     int32_t *cand_tiles[2];
     int64_t *lvl;                         // per level: p0, N, e0, E, tile_base, ie0, IE, itile_base
-    Ctrs *ctr;
-    double *bc;                           // indexed by caller labels
+    Ctrs *ctr;                            // this partition's counters and barrier
+    Ctrs *gctr;                           // shared: full-grid barrier, trace counter
+    int cta_base;                         // first CTA of this SM partition
+    double *bc;                           // indexed by caller labels (a partition's partial bc
+                                          // when the launch has several partitions)
     const int32_t *sources;               // caller labels
     const int32_t *__restrict__ perm;     // caller -> internal label (nullptr: identity)
     const int32_t *__restrict__ inv;      // internal -> caller label
@@ -85,6 +88,30 @@ struct Params {
 
 }  // namespace tbc
 
+namespace tbc {
+// per-SM-partition workspace: each partition runs its own sources with these arrays
+struct Workspace {
+    int32_t *depth = nullptr;
+    double *sigma = nullptr, *du = nullptr, *gacc = nullptr;
+    int32_t *list_v = nullptr;
+    int64_t *list_pre = nullptr;
+    int64_t *list_beg = nullptr;
+    int32_t *tiles = nullptr;
+    int32_t *ilist_v = nullptr;   // in-degree list (directed CSC engine only)
+    int64_t *ilist_pre = nullptr;
+    int64_t *ilist_beg = nullptr;
+    int32_t *itiles = nullptr;
+    int32_t *cand_v[2] = {nullptr, nullptr};
+    int64_t *cand_pre[2] = {nullptr, nullptr};
+    int64_t *cand_beg[2] = {nullptr, nullptr};
+    int32_t *cand_tiles[2] = {nullptr, nullptr};
+    int64_t *lvl = nullptr;
+    Ctrs *ctr = nullptr;
+    double *bc_part = nullptr;    // partial bc of this partition (zero between calls)
+};
+constexpr int kMaxPartitions = 8;
+}  // namespace tbc
+
 struct tbc_graph {
     int device = 0;
     int64_t n = 0, m = 0;
@@ -101,24 +128,12 @@ struct tbc_graph {
     int32_t *inv = nullptr;      // internal label -> caller label
     int32_t *in_col = nullptr;   // column (owner) of every CSC entry: with in_idx, the COOC arrays
     int32_t *out_row = nullptr;  // row (owner) of every CSR entry (== in_col when undirected)
-    // workspace (device)
-    int32_t *depth = nullptr;
-    double *sigma = nullptr, *du = nullptr, *gacc = nullptr;
-    int32_t *list_v = nullptr;
-    int64_t *list_pre = nullptr;
-    int64_t *list_beg = nullptr;
-    int32_t *tiles = nullptr;
-    int32_t *ilist_v = nullptr;   // in-degree list (directed CSC engine only)
-    int64_t *ilist_pre = nullptr;
-    int64_t *ilist_beg = nullptr;
-    int32_t *itiles = nullptr;
+    // workspaces (device), one per SM partition; ws_count allocated so far
+    tbc::Workspace ws[tbc::kMaxPartitions];
+    int ws_count = 0;
+    int nparts = 8;               // TBC_OPT_PARTITIONS
+    tbc::Ctrs *gctr = nullptr;    // shared counters: full-grid barrier, trace
     int64_t n_scan = 0, n_in = 0;
-    int32_t *cand_v[2] = {nullptr, nullptr};
-    int64_t *cand_pre[2] = {nullptr, nullptr};
-    int64_t *cand_beg[2] = {nullptr, nullptr};
-    int32_t *cand_tiles[2] = {nullptr, nullptr};
-    int64_t *lvl = nullptr;
-    tbc::Ctrs *ctr = nullptr;
     double *bc_tmp = nullptr;
     int32_t *src_tmp = nullptr;
     int64_t src_cap = 0;
@@ -141,6 +156,8 @@ tbc_status set_error(tbc_status s, const char *fmt, ...);
 tbc_status cuda_error(cudaError_t e, const char *what);
 // engine entry points (tbc_engine.cu)
 tbc_status engine_setup(tbc_graph *g);
+tbc_status engine_workspaces(tbc_graph *g, int count);  // allocate partitions [ws_count, count)
+void engine_free(tbc_graph *g);                          // workspaces + shared counters
 tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc,
                       cudaStream_t stream, int bfs_only);
 }  // namespace tbc

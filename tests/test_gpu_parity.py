@@ -94,6 +94,26 @@ def test_random_small_graphs_many(directed):
             assert_bc(G.bc(src), want)
 
 
+@pytest.mark.parametrize("directed", [False, True])
+def test_sm_partitions(directed):
+    """1..8 SM partitions give the oracle's bc (repeat runs agree to rounding: the fp64 atomics of
+    split owners and backward pushes add in a run-dependent order)."""
+    g = gg.kronecker(13, 16, seed=4, directed=directed, device="cuda")
+    src = gg.sources(g, 37, seed=3)
+    want = oracle.bc(g.col_ptr, g.row_idx, directed, src)
+    with gpu_graph(g) as G:
+        for parts in (1, 2, 3, 4, 8):
+            G.set_partitions(parts)
+            a = G.bc(src)
+            assert_bc(a, want)
+            assert_bc(G.bc(src), a, rel=1e-12)
+        G.set_partitions(8)
+        assert_bc(G.bc(src[:3]), oracle.bc(g.col_ptr, g.row_idx, directed, src[:3]))  # fewer sources than parts
+        assert_bfs(g, G, src[5])
+        with pytest.raises(tbc.TBCError):
+            G.set_partitions(9)
+
+
 def test_grid_sigma_crosses_2_53():
     g = gg.grid(40, 40)
     with gpu_graph(g) as G:

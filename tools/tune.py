@@ -33,7 +33,9 @@ for setting in a.settings.split(";"):
     kv = dict(x.split("=") for x in setting.split(",") if x)
     G.set_format(int(kv.get("fmt", 0)))
     G.set_direction(int(kv.get("dir", 0)))
-    G.set_cost(**{k: float(v) for k, v in kv.items() if k in ("list", "stream", "atomic", "vertex")})
+    G.set_bwd_direction(int(kv.get("bwd", 0)))
+    G.set_partitions(int(kv.get("parts", 4)))
+    G.set_cost(**{k: float(v) for k, v in kv.items() if k in ("list", "stream", "atomic", "vertex", "scan", "bpush")})
     G.bc_device(s_d, bc, st)  # warm-up
     torch.cuda.synchronize()
     G.reset_stats()
@@ -56,5 +58,5 @@ for setting in a.settings.split(";"):
         for r in G.trace():
             print("TRACE " + json.dumps({"setting": setting, "src": t, **r}), flush=True)
         G.set_trace(-1)
-    G.set_cost(list=12, stream=4, atomic=18, vertex=10)
+    G.set_cost(list=12, stream=4, atomic=18, vertex=10, scan=3, bpush=6)
 G.close()

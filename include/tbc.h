@@ -174,6 +174,14 @@ tbc_status tbc_stats_reset(tbc_graph *g);
  *   count: receives the number of entries recorded (<= 65536).  Synchronises the device. */
 tbc_status tbc_trace_get(tbc_graph *g, int64_t *out, int64_t cap, int64_t *count);
 
+/* Diagnostic region profile (libraries built with -DTBC_PROF only; TBC_ERR_UNSUPPORTED otherwise):
+ * warp-cycles spent per code region of the persistent kernel since the last call, summed over
+ * warps (lane 0 clock64 deltas).  out: host uint64[cap]; count receives 32.  Entry 0 grid
+ * barriers, 1 + 4*mode + {window, index issue, gather/op, tail} for list passes (mode 0 push,
+ * 1 pull, 2 backward pull, 3 backward push), 17 + mode stream passes, 20 pull owner pass,
+ * 21 candidate scan, 22 backward owner pass, 23 the rest.  Reading resets the counters. */
+tbc_status tbc_profile_get(tbc_graph *g, uint64_t *out, int64_t cap, int64_t *count);
+
 /* Free everything the handle owns.  NULL is a no-op. */
 tbc_status tbc_destroy(tbc_graph *g);
 

@@ -33,7 +33,7 @@ STATUS = {0: "TBC_OK", 1: "TBC_ERR_INVALID", 2: "TBC_ERR_OOM", 3: "TBC_ERR_CUDA"
 # every symbol include/tbc.h declares (checked by tests/test_abi.py)
 SYMBOLS = ["tbc_graph_create_csc", "tbc_graph_create_coo", "tbc_bc", "tbc_bc_device", "tbc_bfs",
            "tbc_graph_info", "tbc_graph_set_option", "tbc_stats_get", "tbc_stats_reset", "tbc_trace_get",
-           "tbc_destroy", "tbc_status_string", "tbc_last_error"]
+           "tbc_profile_get", "tbc_destroy", "tbc_status_string", "tbc_last_error"]
 
 
 class TBCError(RuntimeError):
@@ -74,11 +74,12 @@ def lib():
         L.tbc_stats_get.argtypes = [vp, P(Stats)]
         L.tbc_stats_reset.argtypes = [vp]
         L.tbc_trace_get.argtypes = [vp, P(i64), i64, P(i64)]
+        L.tbc_profile_get.argtypes = [vp, P(ctypes.c_uint64), i64, P(i64)]
         L.tbc_destroy.argtypes = [vp]
         L.tbc_status_string.argtypes = [ctypes.c_int]
         L.tbc_status_string.restype = ctypes.c_char_p
         L.tbc_last_error.restype = ctypes.c_char_p
-        for name in SYMBOLS[:11]:
+        for name in SYMBOLS[:12]:
             getattr(L, name).restype = ctypes.c_int
         _LIB = L
     return _LIB
@@ -193,6 +194,18 @@ class Graph:
             out.append({"kind": names[int(r[1])], "level": int(r[2]), "N": int(r[3]), "E": int(r[4]),
                         "a": int(r[5]), "b": int(r[6]), "dt_us": dt / 1e3})
         return out
+
+    PROFILE_REGIONS = (["barrier"] + [f"{m}_{r}" for m in ("push", "pull", "bwd", "bpush")
+                                      for r in ("window", "index", "gather", "tail")]
+                       + ["stream_push", "stream_pull", "stream_bwd", "pull_owner", "scan", "bwd_owner", "other"])
+
+    def profile(self) -> dict:
+        """Region profile of a -DTBC_PROF library (warp-cycles per region; resets on read)."""
+        buf = np.zeros(32, dtype=np.uint64)
+        cnt = ctypes.c_int64()
+        _check(lib().tbc_profile_get(self._h, buf.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), 32,
+                                     ctypes.byref(cnt)))
+        return {k: int(v) for k, v in zip(self.PROFILE_REGIONS, buf)}
 
     def stats(self) -> dict:
         st = Stats()

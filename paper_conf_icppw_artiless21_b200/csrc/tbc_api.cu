@@ -657,6 +657,26 @@ fail:
     return st;
 }
 
+tbc_status tbc_profile_get(tbc_graph *g, uint64_t *out, int64_t cap, int64_t *count) {
+    if (!g || !count || (cap > 0 && !out)) return set_error(TBC_ERR_INVALID, "NULL pointer");
+#ifndef TBC_PROF
+    *count = 0;
+    return set_error(TBC_ERR_UNSUPPORTED, "library built without TBC_PROF");
+#else
+    tbc_status st = TBC_OK;
+    Ctrs c;
+    TBC_CUDA(cudaSetDevice(g->device));
+    TBC_CUDA(cudaDeviceSynchronize());
+    TBC_CUDA(cudaMemcpy(&c, g->gctr, sizeof c, cudaMemcpyDeviceToHost));
+    *count = 32;
+    for (int64_t i = 0; i < cap && i < 32; ++i) out[i] = c.prof[i];
+    TBC_CUDA(cudaMemset(g->gctr->prof, 0, sizeof c.prof));
+    return TBC_OK;
+fail:
+    return st;
+#endif
+}
+
 tbc_status tbc_stats_reset(tbc_graph *g) {
     if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
     tbc_status st = TBC_OK;

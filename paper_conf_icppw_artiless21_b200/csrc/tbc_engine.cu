@@ -60,6 +60,28 @@ struct __align__(16) WarpSmem {
 };
 constexpr size_t kSmemBytes = sizeof(WarpSmem) * kWarpsPerBlock;
 
+// ------------------------------------------------------------------ region profiler (TBC_PROF)
+// Diagnostic builds only: lane 0 of every warp adds clock64 deltas per code region into a
+// per-warp shared-memory row; the rows are summed into gctr->prof at the end of the kernel.
+enum {
+    PR_BARRIER = 0, PR_EDGE = 1,  // PR_EDGE + 4 * MODE + {0 window, 1 index issue, 2 gather/op, 3 tail}
+    PR_STREAM = 17,               // + MODE (PUSH, PULL, BWD)
+    PR_PULL_OWNER = 20, PR_SCAN = 21, PR_BWD_OWNER = 22, PR_OTHER = 23, PR_SLOTS = 24
+};
+#ifdef TBC_PROF
+__shared__ unsigned long long tbc_sprof[kWarpsPerBlock][PR_SLOTS];
+#define PROF_START() unsigned long long _pt = clock64()
+#define PROF(slot)                                                              \
+    do {                                                                        \
+        const unsigned long long _n = clock64();                                \
+        if ((threadIdx.x & 31) == 0) tbc_sprof[threadIdx.x >> 5][(slot)] += _n - _pt; \
+        _pt = _n;                                                               \
+    } while (0)
+#else
+#define PROF_START() ((void)0)
+#define PROF(slot) ((void)0)
+#endif
+
 // ------------------------------------------------------------------ memory-model helpers
 
 __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
@@ -137,6 +159,7 @@ constexpr unsigned long long kWatchdogNs = 20ull * 1000 * 1000 * 1000;  // 20 s 
 // the last arriver bumps the generation; waiters acquire it.  The acquire-side gpu fence also
 // invalidates this SM's L1, so plain loads after the barrier see other CTAs' writes.
 __device__ __forceinline__ void grid_sync(Ctrs *c, unsigned &gen, unsigned nblocks) {
+    PROF_START();
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned g0 = gen;
@@ -157,6 +180,7 @@ __device__ __forceinline__ void grid_sync(Ctrs *c, unsigned &gen, unsigned nbloc
     }
     gen += 1;
     __syncthreads();
+    PROF(PR_BARRIER);
 }
 
 // ------------------------------------------------------------------ warp-aggregated append
@@ -209,24 +233,16 @@ __device__ __forceinline__ void warp_append(const bool (&take)[kLaneItems], cons
             const uint32_t t = __shfl_up_sync(FULL, inc, k);
             if (lane >= k) inc += t;
         }
-        const int64_t pp = p + __popc(msk & lt);
-        const int64_t ee = e + (int64_t)(inc - x);
-        const int64_t k0 = (ee - o.e0) + (pp - o.p0);
-        const int64_t t0 = (k0 + kWT - 1) / kWT, t1 = (k0 + x) / kWT;
-        const bool wide = take[i] && t1 - t0 >= 8;  // a hub: the whole warp writes its tile starts
         if (take[i]) {
+            const int64_t pp = p + __popc(msk & lt);
+            const int64_t ee = e + (int64_t)(inc - x);
             TBC_CHECK(v[i] >= 0, "append v %d", v[i]);
             o.v[pp] = v[i];
             o.pre[pp] = ee;
             o.beg[pp] = bg[i];
-            if (!wide)
-                for (int64_t t = t0; t <= t1; ++t) o.tiles[t] = (int32_t)(pp - o.p0);
-        }
-        for (unsigned wm = __ballot_sync(FULL, wide); wm; wm &= wm - 1) {
-            const int src = __ffs(wm) - 1;
-            const int64_t a = __shfl_sync(FULL, t0, src), b = __shfl_sync(FULL, t1, src);
-            const int32_t val = (int32_t)(__shfl_sync(FULL, pp, src) - o.p0);
-            for (int64_t t = a + lane; t <= b; t += 32) o.tiles[t] = val;
+            const int64_t k0 = (ee - o.e0) + (pp - o.p0);
+            const int64_t k1 = k0 + x;
+            for (int64_t t = (k0 + kWT - 1) / kWT; t <= k1 / kWT; ++t) o.tiles[t] = (int32_t)(pp - o.p0);
         }
         p += __popc(msk);
         e += __shfl_sync(FULL, inc, 31);
@@ -276,6 +292,7 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
     const int64_t K = N + E;
     const int64_t ntiles = ceil_div(K, kWT);
     const uint64_t pol_stream = policy_evict_first();
+    PROF_START();
     for (int64_t tile = gwarp; tile < ntiles; tile += nwarps) {
         const int64_t ks = tile * kWT;
         const int64_t ke = min(ks + (int64_t)kWT, K);
@@ -345,6 +362,7 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
         }
         __syncwarp();
 
+        PROF(PR_EDGE + 4 * MODE + 0);
         // ---- edges in coalesced order: slot = i*32 + lane (consecutive lanes -> consecutive entries)
         int xs[kLaneItems];
         int js[kLaneItems];
@@ -362,6 +380,7 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
                           (long long)(ws.beg[j] + (sl - ws.first[j])));
             }
         }
+        PROF(PR_EDGE + 4 * MODE + 1);
         if (MODE == MODE_PUSH) {
             // masked scatter f_t(x) += f(u) for x on levels {-1, d} (Alg.1 l.19-25 as a push).
             // sigma is 0 off the current BFS, so the atomic that lifts sigma(x) from 0 is the
@@ -375,6 +394,7 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
                 olds[i] = 1.0;
                 if (dxs[i] == -1 || dxs[i] == d) olds[i] = atomicAdd(&P.sigma[xs[i]], ws.val[js[i]]);
             }
+            PROF(PR_EDGE + 4 * MODE + 2);
             bool claim[kLaneItems];
             uint32_t cdg[kLaneItems];
             int64_t cbg[kLaneItems];
@@ -405,6 +425,7 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i)
                 if (dxs[i] == d) atomicAdd(&P.gacc[xs[i]], ws.val[js[i]]);
+            PROF(PR_EDGE + 4 * MODE + 2);
         } else {
             double vals[kLaneItems];
             if (MODE == MODE_PULL) {
@@ -423,6 +444,7 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
                     vals[i] = want > 0.0 ? want : 0.0;
                 }
             }
+            PROF(PR_EDGE + 4 * MODE + 2);
             // transpose the values to lane-contiguous slots through shared memory (beg[] is dead)
             double *vb = reinterpret_cast<double *>(ws.beg);
             __syncwarp();
@@ -468,7 +490,7 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
             const int next_head = __shfl_down_sync(FULL, head_o, 1);
             if (tail_o >= 0 && (lane == 31 || next_head != tail_o)) ws.val[tail_o] = S;
             __syncwarp();
-            // ---- hand each owner's sum to the owner pass
+            // ---- hand each owner's sum to the owner pass (this and the reduction: region 3)
             for (int j = lane; j < nwin; j += 32) {
                 const double t = ws.val[j];
                 if (t == 0.0) continue;
@@ -478,6 +500,7 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
             }
         }
         __syncwarp();
+        PROF(PR_EDGE + 4 * MODE + 3);
     }
 }
 
@@ -532,6 +555,7 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
     const int64_t nchunks = ceil_div(m, kWT);
     const int64_t mine = gwarp < nchunks ? (nchunks - 1 - gwarp) / nwarps + 1 : 0;
     if (mine == 0) return;
+    PROF_START();
     __syncwarp();  // every lane is done with the previous contents of the warp slice
     auto issue = [&](int64_t j) {  // lane 0 only
         const int st = (int)(j % kStages);
@@ -718,6 +742,7 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
     if (lane == 0)
         for (int st = 0; st < kStages; ++st) mbar_inval(&bar[st]);
     __syncwarp();
+    PROF(PR_STREAM + MODE);
 }
 
 // ------------------------------------------------------------------ owner passes
@@ -895,6 +920,11 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamS
     const int64_t gtid = (int64_t)lcta * kBlock + tid;
     Ctrs *C = P.ctr;
     unsigned gen_all = (tid == 0) ? ld_acquire(&S.gctr->bar_gen) : 0u;
+#ifdef TBC_PROF
+    for (int i = tid; i < kWarpsPerBlock * PR_SLOTS; i += kBlock) (&tbc_sprof[0][0])[i] = 0;
+    __syncthreads();
+    const unsigned long long t_kernel0 = clock64();
+#endif
     // barrier generation: only thread 0 uses it (the first barrier cannot complete before
     // every CTA has read the current value, so reading it here is race-free)
     unsigned gen = (tid == 0) ? ld_acquire(&C->bar_gen) : 0u;
@@ -992,7 +1022,11 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamS
                 if (choice == 4) {
                     // candidate list cb is empty here (reset by the push level before its barrier)
                     const ListOut sc{&C->cand[cb], P.cand_v[cb], P.cand_pre[cb], P.cand_beg[cb], P.cand_tiles[cb], 0, 0};
-                    cand_scan_pass(P, gwarp, nwarps, sc);
+                    {
+                        PROF_START();
+                        cand_scan_pass(P, gwarp, nwarps, sc);
+                        PROF(PR_SCAN);
+                    }
                     grid_sync(C, gen, ncta);
                     const unsigned long long cv = ld_volatile_u64(&C->cand[cb]);
                     candN = (int64_t)(cv >> P.ebits);
@@ -1014,7 +1048,11 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamS
                 grid_sync(C, gen, ncta);
                 trace(P, tr, TR_PULL, d, candN, candE, stream, 0);
                 // owner pass: the survivors of a stream pull are all undiscovered vertices
-                pull_owner_pass(P, stream ? nullptr : P.cand_v[cb], candN, d, gwarp, nwarps, lo, li, co);
+                {
+                    PROF_START();
+                    pull_owner_pass(P, stream ? nullptr : P.cand_v[cb], candN, d, gwarp, nwarps, lo, li, co);
+                    PROF(PR_PULL_OWNER);
+                }
                 fwd_edges += candE;
                 ++pulls;
                 cand_valid = !P.coot;
@@ -1113,7 +1151,11 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamS
                 grid_sync(C, gen, ncta);
                 trace(P, tr, TR_BWD, L, lv.N, lv.E, bsel, 0);
             }
-            bwd_owner_pass(P, P.list_v + lv.p0, lv.N, L, gtid, nthreads);
+            {
+                PROF_START();
+                bwd_owner_pass(P, P.list_v + lv.p0, lv.N, L, gtid, nthreads);
+                PROF(PR_BWD_OWNER);
+            }
             grid_sync(C, gen, ncta);
             trace(P, tr, TR_OWNER, L, lv.N, lv.E, 1, 0);
             up = lv;
@@ -1125,6 +1167,14 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamS
         P.depth[prev_s] = -1;
         P.sigma[prev_s] = 0.0;
     }
+#ifdef TBC_PROF
+    if ((tid & 31) == 0) {
+        unsigned long long busy = 0;
+        for (int r = 0; r < PR_OTHER; ++r) busy += tbc_sprof[tid >> 5][r];
+        tbc_sprof[tid >> 5][PR_OTHER] = clock64() - t_kernel0 - busy;  // the rest: control, init, idle
+        for (int r = 0; r < PR_SLOTS; ++r) atomicAdd(&S.gctr->prof[r], tbc_sprof[tid >> 5][r]);
+    }
+#endif
     if (S.nparts > 1 && !P.bfs_only) {
         // every partition done: bc_out += the partitions' partial bc in partition order
         // (deterministic), and the partials return to zero for the next call

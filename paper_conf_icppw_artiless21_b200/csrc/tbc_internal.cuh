@@ -29,6 +29,7 @@ struct Ctrs {
     // accumulated statistics (tbc_stats)
     long long st_sources, st_reached, st_reached_edges, st_fwd_edges, st_bwd_edges, st_levels, st_pull_levels,
         st_scans, st_max_depth;
+    unsigned long long prof[32];  // TBC_PROF builds: warp-cycles per code region (gctr only)
 };
 
 struct Params {

@@ -39,6 +39,9 @@ for setting in a.settings.split(";"):
     G.bc_device(s_d, bc, st)  # warm-up
     torch.cuda.synchronize()
     G.reset_stats()
+    prof = "TBC_PROF" in os.environ.get("TBC_VARIANT", "")
+    if prof:
+        G.profile()  # reset
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(st)
     for _ in range(a.reps):
@@ -52,6 +55,10 @@ for setting in a.settings.split(";"):
                       "fwd_edges_per_src": s["fwd_edges"] / max(s["sources"], 1),
                       "bwd_edges_per_src": s["bwd_edges"] / max(s["sources"], 1),
                       "pull_levels": s["pull_levels"] / max(s["sources"], 1)}), flush=True)
+    if prof:
+        pr = G.profile()
+        tot = sum(pr.values()) or 1
+        print("PROFILE " + setting + " " + " ".join(f"{k}={100 * v / tot:.1f}" for k, v in pr.items() if v), flush=True)
     for t in [int(x) for x in a.trace.split(",") if x]:
         G.set_trace(t)
         G.bc(src[: t + 1])

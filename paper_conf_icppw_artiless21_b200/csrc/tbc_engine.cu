@@ -50,6 +50,7 @@ constexpr int kLaneItems = TBC_LANE_ITEMS;  // items per lane per warp tile
 constexpr int kWT = 32 * kLaneItems;   // diagonal items per warp tile
 constexpr int kWarpsPerBlock = kBlock / 32;
 
+constexpr int kListPad = 8;  // spare entries at the end of every list array
 // per-warp slice of shared memory (owner window of one tile; reused as append buffers)
 struct __align__(16) WarpSmem {
     int64_t beg[kWT + 2];    // adjacency position of the owner's first in-tile edge
@@ -190,8 +191,8 @@ __device__ __forceinline__ void grid_sync(Ctrs *c, unsigned &gen, unsigned nbloc
 struct ListOut {
     unsigned long long *ctr;
     int32_t *v;
-    int64_t *pre;
-    int64_t *beg;
+    uint32_t *pre;
+    uint32_t *beg;
     int32_t *tiles;  // already offset to this level's tile base
     int64_t p0, e0;  // level start within the list (list position, edge prefix)
 };
@@ -205,7 +206,7 @@ struct ListOut {
 // one warp scan per item.  Degrees of distinct vertices sum to <= m < 2^32 (engine_setup).
 // All 32 lanes call this (warp-uniform control flow).
 __device__ __forceinline__ void warp_append(const bool (&take)[kLaneItems], const int32_t (&v)[kLaneItems],
-                                            const uint32_t (&dg)[kLaneItems], const int64_t (&bg)[kLaneItems],
+                                            const uint32_t (&dg)[kLaneItems], const uint32_t (&bg)[kLaneItems],
                                             const ListOut &o, int ebits) {
     const int lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
@@ -238,7 +239,7 @@ __device__ __forceinline__ void warp_append(const bool (&take)[kLaneItems], cons
             const int64_t ee = e + (int64_t)(inc - x);
             TBC_CHECK(v[i] >= 0, "append v %d", v[i]);
             o.v[pp] = v[i];
-            o.pre[pp] = ee;
+            o.pre[pp] = (uint32_t)ee;
             o.beg[pp] = bg[i];
             const int64_t k0 = (ee - o.e0) + (pp - o.p0);
             const int64_t k1 = k0 + x;
@@ -250,9 +251,10 @@ __device__ __forceinline__ void warp_append(const bool (&take)[kLaneItems], cons
 }
 
 // degree and adjacency begin of v in a pointer array (CSC in_ptr or CSR out_ptr)
-__device__ __forceinline__ void adj_span(const int64_t *ptr, int32_t v, uint32_t &dg, int64_t &bg) {
-    bg = ptr[v];
-    dg = (uint32_t)(ptr[v + 1] - bg);
+__device__ __forceinline__ void adj_span(const int64_t *ptr, int32_t v, uint32_t &dg, uint32_t &bg) {
+    const int64_t b = ptr[v];
+    bg = (uint32_t)b;
+    dg = (uint32_t)(ptr[v + 1] - b);
 }
 
 // ------------------------------------------------------------------ level descriptors
@@ -283,8 +285,8 @@ __device__ __forceinline__ int64_t ceil_div(int64_t a, int64_t b) { return (a + 
 // must NOT be declared __restrict__ const, or the compiler may read them through the
 // non-coherent (ld.global.nc) path and see stale lines.
 template <int MODE>
-__device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const int32_t *ov, const int64_t *opre,
-                                          const int64_t *obeg, const int32_t *otiles, int64_t N, int64_t E,
+__device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const int32_t *ov, const uint32_t *opre,
+                                          const uint32_t *obeg, const int32_t *otiles, int64_t N, int64_t E,
                                           int64_t e0, const int64_t *__restrict__ adj_ptr,
                                           const int32_t *__restrict__ adj_idx, int d, int64_t gwarp, int64_t nwarps,
                                           ListOut out, ListOut out_in) {
@@ -308,13 +310,13 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
         // ---- owner window (three coalesced list reads): first in-tile slot, its adjacency position
         bool start0 = true;
         for (int j = lane; j < nwin; j += 32) {
-            const int64_t pre = opre[ps + j] - e0;
+            const int64_t pre = (int64_t)opre[ps + j] - e0;
             const int64_t f = max(pre, es);
             const int32_t v = ov[ps + j];
             TBC_CHECK(v >= 0 && v < P.n && f - es >= 0 && f - es <= kWT, "mode %d v %d f-es %lld", MODE, v,
                       (long long)(f - es));
             ws.first[j] = (int32_t)(f - es);
-            ws.beg[j] = obeg[ps + j] + (f - pre);
+            ws.beg[j] = (int64_t)obeg[ps + j] + (f - pre);
             ws.v[j] = v;
             ws.own[j] = -1;
             if (MODE == MODE_PUSH) {
@@ -397,7 +399,7 @@ __device__ __forceinline__ void edge_pass(const Params &P, WarpSmem &ws, const i
             PROF(PR_EDGE + 4 * MODE + 2);
             bool claim[kLaneItems];
             uint32_t cdg[kLaneItems];
-            int64_t cbg[kLaneItems];
+            uint32_t cbg[kLaneItems];
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
                 claim[i] = olds[i] == 0.0;
@@ -650,7 +652,7 @@ __device__ __forceinline__ void stream_pass(const Params &P, WarpSmem &ws, const
             }
             bool claim[kLaneItems];
             uint32_t cdg[kLaneItems];
-            int64_t cbg[kLaneItems];
+            uint32_t cbg[kLaneItems];
 #pragma unroll
             for (int i = 0; i < kLaneItems; ++i) {
                 claim[i] = olds[i] == 0.0;
@@ -771,7 +773,7 @@ __device__ __forceinline__ void pull_owner_pass(const Params &P, const int32_t *
         }
         bool take[kLaneItems];
         uint32_t dg[kLaneItems];
-        int64_t bg[kLaneItems];
+        uint32_t bg[kLaneItems];
 #pragma unroll
         for (int i = 0; i < kLaneItems; ++i) {
             take[i] = vv[i] >= 0 && tot[i] > 0.0;
@@ -816,7 +818,7 @@ __device__ __forceinline__ void cand_scan_pass(const Params &P, int64_t gwarp, i
         bool take[kLaneItems];
         int32_t vv[kLaneItems];
         uint32_t dg[kLaneItems];
-        int64_t bg[kLaneItems];
+        uint32_t bg[kLaneItems];
 #pragma unroll
         for (int i = 0; i < kLaneItems; ++i) {
             const int64_t v = base + i * 32 + lane;
@@ -955,12 +957,12 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamS
                 P.du[s] = 0.0;
                 P.list_v[0] = s;
                 P.list_pre[0] = 0;
-                P.list_beg[0] = P.out_ptr ? P.out_ptr[s] : 0;
+                P.list_beg[0] = P.out_ptr ? (uint32_t)P.out_ptr[s] : 0u;
                 C->list = (1ull << P.ebits) | (unsigned long long)dego;
                 if (P.in_list) {
                     P.ilist_v[0] = s;
                     P.ilist_pre[0] = 0;
-                    P.ilist_beg[0] = P.in_ptr[s];
+                    P.ilist_beg[0] = (uint32_t)P.in_ptr[s];
                     C->ilist = (1ull << P.ebits) | (unsigned long long)degi;
                 }
                 C->cand[0] = 0;
@@ -1141,8 +1143,8 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamS
                     bwd_edges += lv.E;
                 } else {
                     const int32_t *iv = P.in_list ? P.ilist_v : P.list_v;
-                    const int64_t *ip = P.in_list ? P.ilist_pre : P.list_pre;
-                    const int64_t *ib = P.in_list ? P.ilist_beg : P.list_beg;
+                    const uint32_t *ip = P.in_list ? P.ilist_pre : P.list_pre;
+                    const uint32_t *ib = P.in_list ? P.ilist_beg : P.list_beg;
                     const int32_t *it = P.in_list ? P.itiles + up.itbase : P.tiles + up.tbase;
                     edge_pass<MODE_BPUSH>(P, ws, iv + up.p0, ip + up.p0, ib + up.p0, it, up.N, up.IE, up.ie0,
                                           P.in_ptr, P.in_idx, L, gwarp, nwarps, none, none);
@@ -1215,24 +1217,24 @@ tbc_status engine_workspaces(tbc_graph *g, int count) {
         if (r == cudaSuccess) g->device_bytes += bytes;
         return r;
     };
-    const int64_t list_tiles = (n + m) / kWT + n + 2;
-    const int64_t cand_tiles = (n + m) / kWT + 2;
+    const int64_t list_tiles = (n + m) / kWT + n + 2 + kListPad;
+    const int64_t cand_tiles = (n + m) / kWT + 2 + kListPad;
     for (int i = g->ws_count; i < count; ++i) {
         Workspace &w = g->ws[i];
         g->ws_count = i + 1;  // engine_free releases whatever of it was allocated
         if ((e = alloc(&w.depth, n)) || (e = alloc(&w.sigma, n)) || (e = alloc(&w.du, n)) ||
-            (e = alloc(&w.gacc, n)) || (e = alloc(&w.list_v, n + 1)) || (e = alloc(&w.list_pre, n + 1)) ||
-            (e = alloc(&w.list_beg, n + 1)) || (e = alloc(&w.tiles, list_tiles)) ||
+            (e = alloc(&w.gacc, n)) || (e = alloc(&w.list_v, n + kListPad)) || (e = alloc(&w.list_pre, n + kListPad)) ||
+            (e = alloc(&w.list_beg, n + kListPad)) || (e = alloc(&w.tiles, list_tiles)) ||
             (e = alloc(&w.lvl, kLvlWords * (n + 2))) || (e = alloc(&w.ctr, 1)))
             return cuda_error(e, "workspace cudaMalloc");
         if (g->directed && g->engine == TBC_ENGINE_CSC) {
-            if ((e = alloc(&w.ilist_v, n + 1)) || (e = alloc(&w.ilist_pre, n + 1)) ||
-                (e = alloc(&w.ilist_beg, n + 1)) || (e = alloc(&w.itiles, list_tiles)))
+            if ((e = alloc(&w.ilist_v, n + kListPad)) || (e = alloc(&w.ilist_pre, n + kListPad)) ||
+                (e = alloc(&w.ilist_beg, n + kListPad)) || (e = alloc(&w.itiles, list_tiles)))
                 return cuda_error(e, "workspace cudaMalloc");
         }
         for (int b = 0; b < 2; ++b)
-            if ((e = alloc(&w.cand_v[b], n + 1)) || (e = alloc(&w.cand_pre[b], n + 1)) ||
-                (e = alloc(&w.cand_beg[b], n + 1)) || (e = alloc(&w.cand_tiles[b], cand_tiles)))
+            if ((e = alloc(&w.cand_v[b], n + kListPad)) || (e = alloc(&w.cand_pre[b], n + kListPad)) ||
+                (e = alloc(&w.cand_beg[b], n + kListPad)) || (e = alloc(&w.cand_tiles[b], cand_tiles)))
                 return cuda_error(e, "workspace cudaMalloc");
         if ((e = alloc(&w.bc_part, n))) return cuda_error(e, "workspace cudaMalloc");
         if ((e = cudaMemsetAsync(w.depth, 0xff, sizeof(int32_t) * n, s)) ||

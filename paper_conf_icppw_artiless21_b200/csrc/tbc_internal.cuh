@@ -44,21 +44,21 @@ struct Params {
     double *du;                           // signed delta_u, sign = parity of the level
     double *gacc;                         // per-owner sums handed from edge to owner pass (0 between)
     int32_t *list_v;                      // BFS-order vertex list (levels concatenated)
-    int64_t *list_pre;                    // exclusive out-degree prefix along list_v
-    int64_t *list_beg;                    // out_ptr[v] of each list entry (written at append)
+    uint32_t *list_pre;                   // exclusive out-degree prefix along list_v (< m < 2^32)
+    uint32_t *list_beg;                   // out_ptr[v] of each list entry (written at append)
     int32_t *tiles;                       // per level: owner index starting each tile
     // in-degree list (directed CSC engine): the same vertices per level as list_*, keyed by
     // in-degree (prefix over in_ptr) -- the owners of the backward push pass; == list_* otherwise
     int32_t *ilist_v;
-    int64_t *ilist_pre;
-    int64_t *ilist_beg;
+    uint32_t *ilist_pre;
+    uint32_t *ilist_beg;
     int32_t *itiles;
     int in_list;                          // 1: ilist_* is a separate list appended beside list_*
     int64_t n_scan;                       // vertices [0, n_scan) can have in-edges (degree-sorted labels)
     int64_t n_in;                         // vertices with in-degree > 0
     int32_t *cand_v[2];                   // pull candidate buffers
-    int64_t *cand_pre[2];
-    int64_t *cand_beg[2];
+    uint32_t *cand_pre[2];
+    uint32_t *cand_beg[2];
     int32_t *cand_tiles[2];
     int64_t *lvl;                         // per level: p0, N, e0, E, tile_base, ie0, IE, itile_base
     Ctrs *ctr;                            // this partition's counters and barrier
@@ -95,16 +95,16 @@ struct Workspace {
     int32_t *depth = nullptr;
     double *sigma = nullptr, *du = nullptr, *gacc = nullptr;
     int32_t *list_v = nullptr;
-    int64_t *list_pre = nullptr;
-    int64_t *list_beg = nullptr;
+    uint32_t *list_pre = nullptr;
+    uint32_t *list_beg = nullptr;
     int32_t *tiles = nullptr;
     int32_t *ilist_v = nullptr;   // in-degree list (directed CSC engine only)
-    int64_t *ilist_pre = nullptr;
-    int64_t *ilist_beg = nullptr;
+    uint32_t *ilist_pre = nullptr;
+    uint32_t *ilist_beg = nullptr;
     int32_t *itiles = nullptr;
     int32_t *cand_v[2] = {nullptr, nullptr};
-    int64_t *cand_pre[2] = {nullptr, nullptr};
-    int64_t *cand_beg[2] = {nullptr, nullptr};
+    uint32_t *cand_pre[2] = {nullptr, nullptr};
+    uint32_t *cand_beg[2] = {nullptr, nullptr};
     int32_t *cand_tiles[2] = {nullptr, nullptr};
     int64_t *lvl = nullptr;
     Ctrs *ctr = nullptr;

@@ -9,10 +9,10 @@
 namespace tbc {
 
 #ifndef TBC_BLOCK
-#define TBC_BLOCK 512
+#define TBC_BLOCK 1024
 #endif
 #ifndef TBC_LANE_ITEMS
-#define TBC_LANE_ITEMS 8
+#define TBC_LANE_ITEMS 4
 #endif
 constexpr int kBlock = TBC_BLOCK;  // threads per CTA of the persistent kernel (one CTA per SM)
 constexpr int64_t kTraceCap = 65536; // trace entries (one per barrier of the traced source)

@@ -1,3 +1,4 @@
-timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
-timeout 900 python tools/tune.py --config 3 --sources 512 --settings "parts=8;parts=4" --trace 0 > gpurun_out/tune9.log 2>&1
-tail -2 gpurun_out/pytest_gpu.log; grep -v TRACE gpurun_out/tune9.log | cut -c1-150
+for v in "-DTBC_BLOCK=768 -DTBC_LANE_ITEMS=4" "-DTBC_BLOCK=640 -DTBC_LANE_ITEMS=4" "-DTBC_BLOCK=1024 -DTBC_LANE_ITEMS=4" "-DTBC_BLOCK=512 -DTBC_LANE_ITEMS=4" "-DTBC_BLOCK=768 -DTBC_LANE_ITEMS=8"; do
+  echo "== $v"
+  TBC_VARIANT="$v" timeout 600 python tools/tune.py --config 3 --sources 512 --reps 1 --settings "parts=8;parts=4" 2>&1 | grep -v TRACE | cut -c1-110
+done

@@ -159,6 +159,10 @@ constexpr unsigned long long kWatchdogNs = 20ull * 1000 * 1000 * 1000;  // 20 s 
 // Grid-wide barrier of the cooperative (co-resident) grid: release fence + arrival atomic,
 // the last arriver bumps the generation; waiters acquire it.  The acquire-side gpu fence also
 // invalidates this SM's L1, so plain loads after the barrier see other CTAs' writes.
+// The last arriver also snapshots the list / candidate counters into c->snap (every CTA's
+// appends are complete then): after the barrier CTAs read the snapshot, which nobody writes
+// before the next barrier, while the live counters may already move (a CTA released early
+// starts the next push level's appends or resets the candidate counters).
 __device__ __forceinline__ void grid_sync(Ctrs *c, unsigned &gen, unsigned nblocks) {
     PROF_START();
     __syncthreads();
@@ -168,6 +172,13 @@ __device__ __forceinline__ void grid_sync(Ctrs *c, unsigned &gen, unsigned nbloc
         const unsigned arrived = atomicAdd(&c->bar_count, 1u);
         if (arrived == nblocks - 1) {
             c->bar_count = 0;
+            fence_acq_rel();
+            const unsigned long long s0 = ld_volatile_u64(&c->list), s1 = ld_volatile_u64(&c->ilist),
+                                     s2 = ld_volatile_u64(&c->cand[0]), s3 = ld_volatile_u64(&c->cand[1]);
+            c->snap[0] = s0;
+            c->snap[1] = s1;
+            c->snap[2] = s2;
+            c->snap[3] = s3;
             fence_acq_rel();
             atomicExch(&c->bar_gen, g0 + 1);
         } else {
@@ -932,8 +943,6 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamS
     unsigned gen = (tid == 0) ? ld_acquire(&C->bar_gen) : 0u;
     const unsigned long long emask = (1ull << P.ebits) - 1ull;
     int32_t prev_s = -1;
-    // the in-degree list: a separate list for directed graphs, the out-list itself otherwise
-    unsigned long long *ictr = P.in_list ? &C->ilist : &C->list;
 
     for (int64_t si = part; si < P.k; si += S.nparts) {
         const int32_t s_caller = P.sources[si];
@@ -1030,7 +1039,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamS
                         PROF(PR_SCAN);
                     }
                     grid_sync(C, gen, ncta);
-                    const unsigned long long cv = ld_volatile_u64(&C->cand[cb]);
+                    const unsigned long long cv = ld_volatile_u64(&C->snap[2 + cb]);
                     candN = (int64_t)(cv >> P.ebits);
                     candE = (int64_t)(cv & emask);
                     ++scans;
@@ -1074,15 +1083,15 @@ __global__ void __launch_bounds__(kBlock, 1) k_bc(const __grid_constant__ ParamS
             }
             grid_sync(C, gen, ncta);
             {
-                const unsigned long long lv = ld_volatile_u64(&C->list);
+                const unsigned long long lv = ld_volatile_u64(&C->snap[0]);
                 nxt.N = (int64_t)(lv >> P.ebits) - nxt.p0;
                 nxt.E = (int64_t)(lv & emask) - nxt.e0;
-                const unsigned long long il = ld_volatile_u64(ictr);
+                const unsigned long long il = ld_volatile_u64(&C->snap[P.in_list ? 1 : 0]);
                 nxt.IE = (int64_t)(il & emask) - nxt.ie0;
             }
             trace(P, tr, pull ? TR_OWNER : TR_PUSH, d, nxt.N, nxt.E, choice, pull ? candE : cur.E);
             if (pull) {
-                const unsigned long long cv = ld_volatile_u64(&C->cand[cb ^ 1]);
+                const unsigned long long cv = ld_volatile_u64(&C->snap[2 + (cb ^ 1)]);
                 candN = (int64_t)(cv >> P.ebits);
                 candE = (int64_t)(cv & emask);
                 if (cta0 && tid == 0) C->cand[cb] = 0;  // consumed; next append target after cb flips

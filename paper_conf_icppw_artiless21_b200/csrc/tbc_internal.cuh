@@ -24,6 +24,10 @@ struct Ctrs {
     unsigned long long ilist;     // packed (count << ebits) | in-edge sum of the in-degree list (directed)
     unsigned int bar_count;       // grid barrier arrival counter
     unsigned int bar_gen;         // grid barrier generation
+    // {list, ilist, cand[0], cand[1]} as the last arriver of the latest barrier saw them: CTAs
+    // read the level sizes from here, never from the live counters, which a faster CTA may
+    // already be appending to (next push level) or zeroing (candidate reset)
+    unsigned long long snap[4];
     unsigned long long bad_sources;
     unsigned long long trace_n;   // entries written to the trace buffer
     // accumulated statistics (tbc_stats)

@@ -85,12 +85,20 @@ enum {
     TBC_OPT_COST_VERTEX = 8, /*   vertex of a whole-graph owner pass (default 10) */
     TBC_OPT_COST_SCAN = 9,   /*   vertex of a candidate scan before a pull that follows a push (default 3) */
     TBC_OPT_COST_BPUSH = 10, /*   extra per in-edge of a backward push level over a list item (default 6) */
-    TBC_OPT_PARTITIONS = 11  /* SM partitions (1..8, default 8): the source list is dealt round-robin
+    TBC_OPT_PARTITIONS = 11, /* SM partitions (1..8, default 8): the source list is dealt round-robin
                                 to this many disjoint groups of SMs, each running its sources with its
                                 own workspace and partition-local barriers; the partial bc vectors
                                 are summed in partition order at the end of the call (deterministic
                                 for a given value).  Costs one workspace (~50 B/vertex + 8 B/edge/64)
-                                per partition. */
+                                per partition.  Per-source engine only. */
+    TBC_OPT_BATCH = 12,      /* bc engine: 1 (default) batched -- 32 sources per sweep, one per warp
+                                lane, A^T times an n x 32 frontier block; 0 the
+                                per-source engine.  tbc_bfs and TBC_ENGINE_COOT always use the
+                                per-source engine.  The batched workspace holds 2 x 256 B/vertex of
+                                (sigma, delta_u) rows plus level lists of <= 32 entries per vertex. */
+    TBC_OPT_BATCH_PULL = 13  /* batched engine: a forward level is pulled (candidates' in-edges)
+                                when the frontier's out-edges x this value > nnz, else pushed
+                                (default 8; must be >= 0) */
 };
 
 /* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since

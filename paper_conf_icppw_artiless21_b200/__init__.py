@@ -25,6 +25,7 @@ __all__ = ["Graph", "TBCError", "lib", "ENGINE_CSC", "ENGINE_COOT", "DIR_AUTO", 
 ENGINE_CSC, ENGINE_COOT = 0, 1
 FLAG_ONE_FORMAT, FLAG_NO_VALIDATE, FLAG_NO_REORDER = 1, 2, 4
 OPT_DIRECTION, OPT_BWD_DIRECTION, OPT_TRACE, OPT_FORMAT, OPT_PARTITIONS = 1, 2, 3, 4, 11
+OPT_BATCH, OPT_BATCH_PULL = 12, 13
 OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8, "scan": 9, "bpush": 10}
 FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
 DIR_AUTO, DIR_PUSH, DIR_PULL = 0, 1, 2
@@ -162,6 +163,14 @@ class Graph:
     def set_bwd_direction(self, mode: int):
         """Backward levels: 0 auto, 1 pull over level L's out-edges only, 2 push from level L+1 when possible."""
         _check(lib().tbc_graph_set_option(self._h, OPT_BWD_DIRECTION, float(mode)))
+
+    def set_batch(self, on: int):
+        """bc engine: 1 batched (32 sources per sweep, default), 0 per source (TBC_OPT_BATCH)."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_BATCH, float(on)))
+
+    def set_batch_pull(self, ratio: float):
+        """Batched engine: pull a level when frontier out-edges x ratio > nnz (TBC_OPT_BATCH_PULL)."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_BATCH_PULL, float(ratio)))
 
     def set_partitions(self, parts: int):
         """Number of SM partitions running sources concurrently (1..8; TBC_OPT_PARTITIONS)."""

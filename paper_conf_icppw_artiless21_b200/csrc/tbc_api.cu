@@ -525,6 +525,17 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->bwd_mode = v;
         return TBC_OK;
     }
+    if (key == TBC_OPT_BATCH) {
+        int v = (int)value;
+        if (v < 0 || v > 1 || (double)v != value) return set_error(TBC_ERR_INVALID, "batch %g", value);
+        g->batch = v;
+        return TBC_OK;
+    }
+    if (key == TBC_OPT_BATCH_PULL) {
+        if (!(value >= 0)) return set_error(TBC_ERR_INVALID, "batch pull ratio %g", value);
+        g->batch_pull = value;
+        return TBC_OK;
+    }
     if (key >= TBC_OPT_COST_LIST && key <= TBC_OPT_COST_BPUSH) {
         if (!(value >= 0)) return set_error(TBC_ERR_INVALID, "cost %g", value);
         double *c[] = {&g->c_list, &g->c_stream, &g->c_atom, &g->c_vert, &g->c_scan, &g->c_bpush};
@@ -622,8 +633,10 @@ tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
     TBC_CUDA(cudaSetDevice(g->device));
     TBC_CUDA(cudaDeviceSynchronize());
     *out = tbc_stats{};
-    for (int i = 0; i < g->ws_count; ++i) {  // summed over the SM partitions' counters
-        TBC_CUDA(cudaMemcpy(&c, g->ws[i].ctr, sizeof c, cudaMemcpyDeviceToHost));
+    for (int i = 0; i <= g->ws_count; ++i) {  // summed over the SM partitions' and the batch counters
+        Ctrs *src = i < g->ws_count ? g->ws[i].ctr : g->bws.ctr;
+        if (!src) continue;
+        TBC_CUDA(cudaMemcpy(&c, src, sizeof c, cudaMemcpyDeviceToHost));
         out->sources += c.st_sources;
         out->reached += c.st_reached;
         out->reached_edges += c.st_reached_edges;
@@ -684,6 +697,7 @@ tbc_status tbc_stats_reset(tbc_graph *g) {
     TBC_CUDA(cudaDeviceSynchronize());
     for (int i = 0; i < g->ws_count; ++i)
         TBC_CUDA(cudaMemset(&g->ws[i].ctr->st_sources, 0, sizeof(long long) * 9));
+    if (g->bws.ctr) TBC_CUDA(cudaMemset(&g->bws.ctr->st_sources, 0, sizeof(long long) * 9));
     return TBC_OK;
 fail:
     return st;

@@ -1,0 +1,722 @@
+// tbc_batch.cu -- the batched multi-source engine (north star (c)): Algorithm 1
+// of PAPER.md for 32 sources at once, one source per warp lane.  The per-source
+// SpMV f_t = A^T f of l.19 becomes the product of A^T with a tall-skinny n x 32 frontier block
+// (sparse times tall-skinny, still CUDA cores: irregular gathers, not a dense contraction), and
+// the backward SpMV of l.37 (A delta_u, R1) likewise.  One stream of the adjacency
+// serves all 32 sources of a level, and the per-level fixed costs (barriers, small levels,
+// tails) are paid once per 32 sources instead of once per source.
+//
+// State (vertex-major, source-minor, so a warp's 32 lanes touch one 256-byte row):
+//   sig[v][s]  sigma_s(v)             (fp64, exact integers < 2^53)
+//   du[v][s]   delta_u_s(v) = (1 + delta_s(v)) / sigma_s(v) = 1/sigma_s(v) + acc_s(v)  (l.35)
+//   vis[v]     lanes s with depth_s(v) <= the current level
+//   fr[p][v]   lanes s with depth_s(v) = d, for the levels d of parity p in flight
+//   level list d: vertices with any lane on level d, with that lane mask (M_d) and their
+//              out-degree prefix, plus per-warp-tile start owners (merge path, as tbc_engine.cu)
+//
+// Forward level d+1 (Alg.1 l.19-27):
+//   PUSH  owners = level list d; lanes M_d(u) & ~vis(x) of each out-edge u->x:
+//         sig[x][s] += sig[u][s] (fp64 atomic), fr[x] |= lanes; the atomicOr that lifts fr[x]
+//         from 0 appends x to level list d+1.
+//   PULL  owners = candidates w (any active lane unvisited); lanes M_d(u) & ~vis(w) of each
+//         in-edge u->w: acc[s] += sig[u][s]; discovered lanes = acc > 0 (the mask of l.20-25).
+//   then an owner phase: list_m = M_{d+1}, vis |= M_{d+1}, retire M_d's dense masks.
+// Backward level L = D..1 (Alg.1 l.29-47): owners = level list L; lanes M_L(v) & M_{L+1}(w) of
+// each out-edge v->w: acc[s] += du[w][s]; then bc(v) += scale * sum_s sigma_s(v) acc_s
+// (l.39, l.45, 1/2 if undirected P:180) and du[v][s] = 1/sigma_s(v) + acc_s.  A vertex whose
+// out-edges span several warp tiles is "split": its partial sums are added with fp64 atomics
+// (both bc and du are linear in acc), the tile holding its first item adds the 1/sigma term.
+#include <cstdio>
+
+#include "tbc_internal.cuh"
+#include "tbc_device.cuh"
+
+namespace tbc {
+namespace {
+
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int kBB = 1024;        // threads per CTA (one CTA per SM)
+constexpr int kBWarps = kBB / 32;
+constexpr int kBI = 2;           // tile items per lane (window / index phases)
+constexpr int kBT = 32 * kBI;    // diagonal items (owner end items + edges) per warp tile
+constexpr int kPad = 8;
+
+enum { B_PUSH = 0, B_PULL = 1, B_BWD = 2 };
+
+struct BParams {
+    int64_t n, m;
+    const int64_t *__restrict__ in_ptr;
+    const int32_t *__restrict__ in_idx;
+    const int64_t *__restrict__ out_ptr;
+    const int32_t *__restrict__ out_idx;
+    const int2 *__restrict__ deg2;
+    double *sig, *du;
+    uint32_t *vis;
+    uint32_t *fr0, *fr1;
+    int32_t *list_v;
+    uint32_t *list_pre, *list_beg, *list_m;
+    int32_t *tiles;
+    int32_t *cand_v;
+    uint32_t *cand_pre, *cand_beg;
+    int32_t *cand_tiles;
+    int64_t *lvl;
+    Ctrs *ctr;
+    double *bc;
+    const int32_t *sources;
+    const int32_t *__restrict__ perm;
+    const int32_t *__restrict__ inv;
+    int64_t k, n_scan, list_cap, tiles_cap, cand_tiles_cap;
+    double bc_scale, pull_ratio;
+    int ebits, dir_mode;
+};
+
+struct __align__(16) BWarpSmem {
+    uint32_t beg[kBT + 2];   // adjacency position of the owner's first in-tile edge
+    int32_t first[kBT + 2];  // slot of that edge (+ sentinel ne)
+    int32_t v[kBT + 2];      // owner vertex
+    uint32_t msk[kBT + 2];   // owner lanes
+    int32_t fl[kBT + 2];     // bit 0: the tile holds the owner's first item; bit 1: whole owner
+    int32_t own[kBT + 2];    // owner (window index) of each slot
+    int32_t x[kBT];          // other end of each slot
+    uint32_t em[kBT];        // lanes of each slot
+    int32_t claim[kBT + 2];  // vertices discovered by this tile (PULL)
+};
+constexpr size_t kBSmem = sizeof(BWarpSmem) * kBWarps;
+
+struct Lv {
+    int64_t p0, N, E, tb;
+};
+
+__device__ __forceinline__ int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// grid barrier (as tbc_engine.cu): the last arriver snapshots {list, active, cand} counters
+__device__ __forceinline__ void bsync(Ctrs *c, unsigned &gen, unsigned nblocks) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const unsigned g0 = gen;
+        fence_acq_rel();
+        const unsigned arrived = atomicAdd(&c->bar_count, 1u);
+        if (arrived == nblocks - 1) {
+            c->bar_count = 0;
+            fence_acq_rel();
+            const unsigned long long s0 = ld_volatile_u64(&c->list), s1 = ld_volatile_u64(&c->ilist),
+                                     s2 = ld_volatile_u64(&c->cand[0]);
+            c->snap[0] = s0;
+            c->snap[1] = s1;
+            c->snap[2] = s2;
+            fence_acq_rel();
+            atomicExch(&c->bar_gen, g0 + 1);
+        } else {
+            const unsigned long long t0 = globaltimer_ns();
+            while (ld_acquire(&c->bar_gen) == g0) {
+                __nanosleep(20);
+                if (globaltimer_ns() - t0 > kWatchdogNs) __trap();
+            }
+        }
+        fence_acq_rel();
+    }
+    gen += 1;
+    __syncthreads();
+}
+
+// a list being appended to: relative packed counter (count << ebits) | degree sum, arrays
+// offset to the level start, capacities left
+struct BOut {
+    unsigned long long *ctr;
+    int32_t *v;
+    uint32_t *pre, *beg;
+    int32_t *tiles;
+    int64_t cap, tcap;
+};
+
+// warp-aggregated append of the entries lanes hold (item i of lane l: v[i], degree dg[i],
+// adjacency begin bg[i] if take[i]); one packed atomic per warp; the appender of an owner writes
+// the start owner of every tile whose first item lies in its merge-path span (tbc_engine.cu)
+__device__ __forceinline__ void bappend(const bool (&take)[kBI], const int32_t (&v)[kBI], const uint32_t (&dg)[kBI],
+                                        const uint32_t (&bg)[kBI], const BOut &o, int ebits) {
+    const int lane = threadIdx.x & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    unsigned cnt = 0;
+    unsigned long long esum = 0;
+#pragma unroll
+    for (int i = 0; i < kBI; ++i) {
+        cnt += __popc(__ballot_sync(FULL, take[i]));
+        esum += __reduce_add_sync(FULL, take[i] ? dg[i] : 0u);
+    }
+    if (cnt == 0) return;
+    unsigned long long old = 0;
+    if (lane == 0) old = atomicAdd(o.ctr, ((unsigned long long)cnt << ebits) + esum);
+    old = __shfl_sync(FULL, old, 0);
+    int64_t p = (int64_t)(old >> ebits);
+    int64_t e = (int64_t)(old & ((1ull << ebits) - 1ull));
+#pragma unroll
+    for (int i = 0; i < kBI; ++i) {
+        const unsigned msk = __ballot_sync(FULL, take[i]);
+        if (msk == 0) continue;
+        const uint32_t x = take[i] ? dg[i] : 0u;
+        uint32_t inc = x;
+#pragma unroll
+        for (int k = 1; k < 32; k <<= 1) {
+            const uint32_t t = __shfl_up_sync(FULL, inc, k);
+            if (lane >= k) inc += t;
+        }
+        if (take[i]) {
+            const int64_t pp = p + __popc(msk & lt);
+            const int64_t ee = e + (int64_t)(inc - x);
+            if (pp < o.cap) {  // capacities are sufficient by construction (batch_alloc)
+                o.v[pp] = v[i];
+                o.pre[pp] = (uint32_t)ee;
+                o.beg[pp] = bg[i];
+                const int64_t k0 = ee + pp, k1 = k0 + x;
+                for (int64_t t = (k0 + kBT - 1) / kBT; t <= k1 / kBT && t < o.tcap; ++t) o.tiles[t] = (int32_t)pp;
+            }
+        }
+        p += __popc(msk);
+        e += __shfl_sync(FULL, inc, 31);
+    }
+}
+
+__device__ __forceinline__ void span(const int64_t *ptr, int32_t v, uint32_t &dg, uint32_t &bg) {
+    const int64_t b = ptr[v];
+    bg = (uint32_t)b;
+    dg = (uint32_t)(ptr[v + 1] - b);
+}
+
+__device__ __forceinline__ uint64_t slot_range(int s0, int s1) {
+    if (s0 >= 64 || s1 <= s0) return 0ull;
+    const uint64_t hi = s1 >= 64 ? ~0ull : ((1ull << s1) - 1ull);
+    return hi & ~((1ull << s0) - 1ull);
+}
+
+// One merge-path pass over an owner list (ov/opre/obeg/omsk/otiles, N owners, E edges):
+//   PUSH: frontier owners, out-edges;  PULL: candidates, in-edges;  BWD: level-L owners, out-edges.
+// emsk: per-vertex lane mask of the other end (PULL: M_d, BWD: M_{L+1}; PUSH uses ~vis).
+// fr_out: PUSH/PULL the next level's dense mask, BWD the owners' level (scattered M_L).
+template <int MODE>
+__device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int32_t *ov, const uint32_t *opre,
+                                      const uint32_t *obeg, const uint32_t *omsk, const int32_t *otiles, int64_t N,
+                                      int64_t E, const int32_t *__restrict__ adj_idx, const uint32_t *emsk,
+                                      uint32_t *fr_out, uint32_t active, int64_t gwarp, int64_t nwarps, const BOut &out) {
+    const int lane = threadIdx.x & 31;
+    const int64_t K = N + E;
+    const int64_t ntiles = cdiv(K, kBT);
+    const uint64_t pol = policy_evict_first();
+    double *const sig = P.sig;
+    for (int64_t tile = gwarp; tile < ntiles; tile += nwarps) {
+        const int64_t ks = tile * kBT;
+        const int64_t ke = min(ks + (int64_t)kBT, K);
+        const int64_t ps = otiles[tile];
+        const int64_t pe = (tile + 1 < ntiles) ? (int64_t)otiles[tile + 1] : N;
+        const int64_t es = ks - ps, ee = ke - pe;
+        const int nwin = (int)(min(pe, N - 1) - ps + 1);
+        const int ne = (int)(ee - es);
+        // ---- owner window
+        for (int j = lane; j < nwin; j += 32) {
+            const int64_t p = ps + j;
+            const int64_t pre = (int64_t)opre[p];
+            const int64_t f = max(pre, es);
+            const int32_t v = ov[p];
+            ws.first[j] = (int32_t)(f - es);
+            ws.beg[j] = obeg[p] + (uint32_t)(f - pre);
+            ws.v[j] = v;
+            const int64_t kf = pre + p;  // the owner's first diagonal item
+            const bool isf = kf >= ks && kf < ke;
+            const bool whole = isf && p < pe;
+            ws.msk[j] = (MODE == B_PULL) ? (~P.vis[v] & active) : omsk[p];
+            ws.fl[j] = (isf ? 1 : 0) | (whole ? 2 : 0);
+        }
+        for (int sl = lane; sl < kBT; sl += 32) ws.own[sl] = -1;
+        if (lane == 0) ws.first[nwin] = ne;
+        __syncwarp();
+        for (int j = lane; j < nwin; j += 32)
+            if (ws.first[j] < ws.first[j + 1]) ws.own[ws.first[j]] = j;
+        __syncwarp();
+        {  // owner of every slot: running max of the head marks over lane-contiguous slots
+            int o[kBI];
+            int run = -1;
+#pragma unroll
+            for (int i = 0; i < kBI; ++i) {
+                const int sl = lane * kBI + i;
+                run = max(run, sl < ne ? ws.own[sl] : -1);
+                o[i] = run;
+            }
+            int incl = run;
+#pragma unroll
+            for (int k = 1; k < 32; k <<= 1) {
+                const int t = __shfl_up_sync(FULL, incl, k);
+                if (lane >= k) incl = max(incl, t);
+            }
+            int prev = __shfl_up_sync(FULL, incl, 1);
+            if (lane == 0) prev = -1;
+            __syncwarp();
+#pragma unroll
+            for (int i = 0; i < kBI; ++i) {
+                const int sl = lane * kBI + i;
+                if (sl < ne) ws.own[sl] = max(prev, o[i]);
+            }
+        }
+        __syncwarp();
+        // ---- edges, coalesced (slot = i*32 + lane): other end and its lanes
+        int xs[kBI];
+        uint32_t ems[kBI];
+        uint64_t act = 0;
+#pragma unroll
+        for (int i = 0; i < kBI; ++i) {
+            const int sl = i * 32 + lane;
+            xs[i] = 0;
+            ems[i] = 0;
+            if (sl < ne) {
+                const int j = ws.own[sl];
+                xs[i] = ld_stream(adj_idx + ws.beg[j] + (uint32_t)(sl - ws.first[j]), pol);
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < kBI; ++i) {
+            const int sl = i * 32 + lane;
+            if (sl < ne) {
+                const uint32_t g = (MODE == B_PUSH) ? ~P.vis[xs[i]] : emsk[xs[i]];
+                ems[i] = g & ws.msk[ws.own[sl]];
+            }
+            ws.x[sl] = xs[i];
+            ws.em[sl] = ems[i];
+            act |= (uint64_t)__ballot_sync(FULL, ems[i] != 0u) << (32 * i);
+        }
+        if (MODE == B_PUSH) {
+            // claims: the atomicOr that lifts fr_out[x] from 0 appends x to the next level
+            bool cl[kBI];
+            uint32_t cdg[kBI], cbg[kBI];
+#pragma unroll
+            for (int i = 0; i < kBI; ++i) {
+                cl[i] = false;
+                cdg[i] = 0;
+                cbg[i] = 0;
+                if (ems[i] != 0u) cl[i] = atomicOr(&fr_out[xs[i]], ems[i]) == 0u;
+                if (cl[i]) span(P.out_ptr, xs[i], cdg[i], cbg[i]);
+            }
+            bappend(cl, xs, cdg, cbg, out, P.ebits);
+        }
+        __syncwarp();
+        int nc = 0;  // PULL: discovered owners of this tile
+        for (int j = 0; j < nwin; ++j) {
+            uint64_t bits = act & slot_range(ws.first[j], ws.first[j + 1]);
+            const int fl = ws.fl[j];
+            if (MODE != B_BWD && bits == 0) continue;
+            if (MODE == B_BWD && bits == 0 && !(fl & 1)) continue;
+            const int32_t v = ws.v[j];
+            const uint32_t m = ws.msk[j];
+            const bool in = (m >> lane) & 1u;
+            if (MODE == B_PUSH) {
+                const double su = in ? sig[(int64_t)v * kBatch + lane] : 0.0;
+                while (bits) {
+                    const int sl = __ffsll((long long)bits) - 1;
+                    bits &= bits - 1;
+                    if ((ws.em[sl] >> lane) & 1u) atomicAdd(&sig[(int64_t)ws.x[sl] * kBatch + lane], su);
+                }
+                continue;
+            }
+            const double *src = (MODE == B_PULL) ? sig : P.du;
+            const double sv = (MODE == B_BWD && in) ? sig[(int64_t)v * kBatch + lane] : 1.0;
+            double acc = 0.0;
+            while (bits) {  // four slots in flight per lane
+                int sl[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    sl[q] = -1;
+                    if (bits) {
+                        sl[q] = __ffsll((long long)bits) - 1;
+                        bits &= bits - 1;
+                    }
+                }
+                double a[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    a[q] = 0.0;
+                    if (sl[q] >= 0 && ((ws.em[sl[q]] >> lane) & 1u)) a[q] = src[(int64_t)ws.x[sl[q]] * kBatch + lane];
+                }
+                acc += (a[0] + a[1]) + (a[2] + a[3]);
+            }
+            if (MODE == B_PULL) {
+                // Alg.1 l.20-25: lanes with a non-zero masked sum are discovered on this level
+                const unsigned newm = __ballot_sync(FULL, acc > 0.0);
+                if (newm == 0u) continue;
+                bool claimed;
+                if (fl & 2) {
+                    if (acc > 0.0) sig[(int64_t)v * kBatch + lane] = acc;
+                    if (lane == 0) fr_out[v] = newm;
+                    claimed = true;
+                } else {
+                    if (acc > 0.0) atomicAdd(&sig[(int64_t)v * kBatch + lane], acc);
+                    unsigned old = 0;
+                    if (lane == 0) old = atomicOr(&fr_out[v], newm);
+                    claimed = __shfl_sync(FULL, old, 0) == 0u;
+                }
+                if (claimed) {
+                    if (lane == 0) ws.claim[nc] = v;
+                    ++nc;
+                }
+            } else {
+                // Alg.1 l.38-39, l.45 (x 1/2 undirected) and l.35
+                double c = in ? sv * acc : 0.0;
+#pragma unroll
+                for (int k = 16; k >= 1; k >>= 1) c += __shfl_xor_sync(FULL, c, k);
+                if (fl & 2) {
+                    if (in) P.du[(int64_t)v * kBatch + lane] = 1.0 / sv + acc;
+                } else {
+                    const double t = acc + ((fl & 1) ? 1.0 / sv : 0.0);
+                    if (in && t != 0.0) atomicAdd(&P.du[(int64_t)v * kBatch + lane], t);
+                }
+                if (lane == 0) {
+                    if (c != 0.0) atomicAdd(&P.bc[P.inv ? P.inv[v] : v], c * P.bc_scale);
+                    if (fl & 1) atomicOr(&fr_out[v], m);
+                }
+            }
+        }
+        if (MODE == B_PULL) {
+            __syncwarp();
+            bool cl[kBI];
+            int32_t cv[kBI];
+            uint32_t cdg[kBI], cbg[kBI];
+#pragma unroll
+            for (int i = 0; i < kBI; ++i) {
+                const int q = i * 32 + lane;
+                cl[i] = q < nc;
+                cv[i] = cl[i] ? ws.claim[q] : 0;
+                cdg[i] = 0;
+                cbg[i] = 0;
+                if (cl[i]) span(P.out_ptr, cv[i], cdg[i], cbg[i]);
+            }
+            bappend(cl, cv, cdg, cbg, out, P.ebits);
+        }
+        __syncwarp();
+    }
+}
+
+// zero the (vertex, lane) state of a level list's entries: sigma, delta_u, visited lanes and
+// the dense mask of its parity (atomicAnd: a concurrent scatter of another level may share the word)
+__device__ __forceinline__ void bclear(const BParams &P, const Lv &l, uint32_t *fr, int64_t gwarp, int64_t nwarps) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t base = gwarp * 32; base < l.N; base += nwarps * 32) {
+        const int64_t p = base + lane;
+        int32_t v = -1;
+        uint32_t m = 0;
+        if (p < l.N) {
+            v = P.list_v[l.p0 + p];
+            m = P.list_m[l.p0 + p];
+            atomicAnd(&fr[v], ~m);
+            P.vis[v] = 0u;
+        }
+        const int cnt = (int)min((int64_t)32, l.N - base);
+        for (int q = 0; q < cnt; ++q) {
+            const int32_t vq = __shfl_sync(FULL, v, q);
+            const uint32_t mq = __shfl_sync(FULL, m, q);
+            if ((mq >> lane) & 1u) {
+                P.sig[(int64_t)vq * kBatch + lane] = 0.0;
+                P.du[(int64_t)vq * kBatch + lane] = 0.0;
+            }
+        }
+    }
+}
+
+__global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams P) {
+    extern __shared__ __align__(16) unsigned char bsm[];
+    BWarpSmem &ws = reinterpret_cast<BWarpSmem *>(bsm)[threadIdx.x >> 5];
+    const int tid = threadIdx.x, lane = tid & 31;
+    const bool cta0 = blockIdx.x == 0;
+    const unsigned ncta = gridDim.x;
+    const int64_t nwarps = (int64_t)ncta * kBWarps;
+    const int64_t gwarp = (int64_t)blockIdx.x * kBWarps + (tid >> 5);
+    const int64_t nthreads = (int64_t)ncta * kBB;
+    const int64_t gtid = (int64_t)blockIdx.x * kBB + tid;
+    Ctrs *C = P.ctr;
+    unsigned gen = (tid == 0) ? ld_acquire(&C->bar_gen) : 0u;
+    const unsigned long long emask = (1ull << P.ebits) - 1ull;
+    uint32_t *fr[2] = {P.fr0, P.fr1};
+    const int64_t nb = (P.k + kBatch - 1) / kBatch;
+
+    for (int64_t b = 0; b < nb; ++b) {
+        // ---------------- level 0: the batch's sources (Alg.1 l.15-18), lane s <- sources[32b+s]
+        if (cta0 && tid < 32) {
+            const int64_t si = b * kBatch + lane;
+            int32_t s = -1;
+            if (si < P.k) {
+                const int32_t sc = P.sources[si];
+                if (sc >= 0 && sc < P.n) s = P.perm ? P.perm[sc] : sc;
+                else atomicAdd(&C->bad_sources, 1ull);
+            }
+            if (s >= 0) {
+                atomicOr(&P.fr0[s], 1u << lane);
+                P.sig[(int64_t)s * kBatch + lane] = 1.0;
+            }
+            bool take = s >= 0;
+            for (int l = 0; l < 32; ++l) {  // repeated vertices: the lowest lane appends
+                const int32_t t = __shfl_sync(FULL, s, l);
+                if (l < lane && t == s) take = false;
+            }
+            uint32_t dg = 0, bg = 0;
+            if (take) span(P.out_ptr, s, dg, bg);
+            const unsigned tm = __ballot_sync(FULL, take);
+            uint32_t inc = take ? dg : 0u;
+            for (int k = 1; k < 32; k <<= 1) {
+                const uint32_t t = __shfl_up_sync(FULL, inc, k);
+                if (lane >= k) inc += t;
+            }
+            const uint32_t tot = __shfl_sync(FULL, inc, 31);
+            if (take) {
+                const int pos = __popc(tm & ((1u << lane) - 1u));
+                const uint32_t e0 = inc - dg;
+                P.list_v[pos] = s;
+                P.list_pre[pos] = e0;
+                P.list_beg[pos] = bg;
+                const int64_t k0 = (int64_t)e0 + pos, k1 = k0 + dg;
+                for (int64_t t = (k0 + kBT - 1) / kBT; t <= k1 / kBT; ++t) P.tiles[t] = pos;
+            }
+            const unsigned valid = __ballot_sync(FULL, s >= 0);
+            if (lane == 0) {
+                C->list = ((unsigned long long)__popc(tm) << P.ebits) | tot;
+                C->ilist = 0;
+                C->cand[0] = 0;
+                C->st_sources += __popc(valid);
+            }
+        }
+        bsync(C, gen, ncta);
+        Lv cur{0, (int64_t)(ld_volatile_u64(&C->snap[0]) >> P.ebits), (int64_t)(ld_volatile_u64(&C->snap[0]) & emask), 0};
+        if (cur.N == 0) continue;  // every lane invalid: nothing was written
+        if (cta0 && tid == 0) {
+            int64_t *l = P.lvl;
+            l[0] = cur.p0; l[1] = cur.N; l[2] = cur.E; l[3] = cur.tb;
+        }
+        Lv prev{0, 0, 0, 0};
+        int d = 0;
+        uint32_t active = 0xffffffffu;
+        int64_t fwd_edges = 0, pulls = 0;
+        for (;;) {
+            // direction of level d+1 (uniform: every CTA computes it from the same snapshot)
+            const bool pull = d + 1 >= 2 && P.dir_mode != 1 &&
+                              (P.dir_mode == 2 || (double)cur.E * P.pull_ratio > (double)P.m);
+            // ---- B(d): lanes of level d -> list masks and visited; retire M_{d-1}; candidates
+            if (cta0 && tid == 0) C->list = 0;  // relative counter of level d+1 (snapshot already taken)
+            {
+                uint32_t orr = 0;
+                long long rc = 0, re = 0;
+                uint32_t *frd = fr[d & 1];
+                for (int64_t p = gtid; p < cur.N; p += nthreads) {
+                    const int32_t v = P.list_v[cur.p0 + p];
+                    const uint32_t m = frd[v];
+                    P.list_m[cur.p0 + p] = m;
+                    P.vis[v] |= m;
+                    orr |= m;
+                    rc += __popc(m);
+                    re += (long long)__popc(m) * P.deg2[v].x;
+                }
+                orr = __reduce_or_sync(FULL, orr);
+                rc = __reduce_add_sync(FULL, (unsigned)rc);
+                for (int k = 16; k >= 1; k >>= 1) re += __shfl_xor_sync(FULL, re, k);
+                if (lane == 0) {
+                    if (orr) atomicOr((unsigned long long *)&C->ilist, (unsigned long long)orr);
+                    if (rc) atomicAdd((unsigned long long *)&C->st_reached, (unsigned long long)rc);
+                    if (re) atomicAdd((unsigned long long *)&C->st_reached_edges, (unsigned long long)re);
+                }
+                if (d >= 1) {
+                    uint32_t *frp = fr[(d + 1) & 1];
+                    for (int64_t p = gtid; p < prev.N; p += nthreads) frp[P.list_v[prev.p0 + p]] = 0u;
+                }
+                if (pull) {  // candidates: vertices with in-edges and an unvisited active lane
+                    const BOut co{&C->cand[0], P.cand_v, P.cand_pre, P.cand_beg, P.cand_tiles, P.n + kPad,
+                                  P.cand_tiles_cap};
+                    for (int64_t base = gwarp * kBT; base < P.n_scan; base += nwarps * kBT) {
+                        bool tk[kBI];
+                        int32_t vv[kBI];
+                        uint32_t dg[kBI], bg[kBI];
+#pragma unroll
+                        for (int i = 0; i < kBI; ++i) {
+                            const int64_t w = base + i * 32 + lane;
+                            vv[i] = (int32_t)w;
+                            tk[i] = w < P.n_scan && (~P.vis[w] & active) != 0u;
+                            dg[i] = 0;
+                            bg[i] = 0;
+                            if (tk[i]) {
+                                span(P.in_ptr, vv[i], dg[i], bg[i]);
+                                tk[i] = dg[i] > 0;
+                            }
+                        }
+                        bappend(tk, vv, dg, bg, co, P.ebits);
+                    }
+                }
+            }
+            bsync(C, gen, ncta);
+            active = (uint32_t)ld_volatile_u64(&C->snap[1]);
+            const unsigned long long cs = ld_volatile_u64(&C->snap[2]);
+            // ---- A(d+1)
+            if (cta0 && tid == 0) {
+                C->cand[0] = 0;
+                C->ilist = 0;
+            }
+            Lv nxt{cur.p0 + cur.N, 0, 0, cur.tb + cdiv(cur.N + cur.E, kBT)};
+            const BOut lo{&C->list, P.list_v + nxt.p0, P.list_pre + nxt.p0, P.list_beg + nxt.p0, P.tiles + nxt.tb,
+                          P.list_cap - nxt.p0, P.tiles_cap - nxt.tb};
+            uint32_t *fro = fr[(d + 1) & 1];
+            if (pull) {
+                const int64_t cN = (int64_t)(cs >> P.ebits), cE = (int64_t)(cs & emask);
+                bpass<B_PULL>(P, ws, P.cand_v, P.cand_pre, P.cand_beg, nullptr, P.cand_tiles, cN, cE, P.in_idx,
+                              fr[d & 1], fro, active, gwarp, nwarps, lo);
+                fwd_edges += cE;
+                ++pulls;
+            } else {
+                bpass<B_PUSH>(P, ws, P.list_v + cur.p0, P.list_pre + cur.p0, P.list_beg + cur.p0, P.list_m + cur.p0,
+                              P.tiles + cur.tb, cur.N, cur.E, P.out_idx, nullptr, fro, 0u, gwarp, nwarps, lo);
+                fwd_edges += cur.E;
+            }
+            bsync(C, gen, ncta);
+            {
+                const unsigned long long lv = ld_volatile_u64(&C->snap[0]);
+                nxt.N = (int64_t)(lv >> P.ebits);
+                nxt.E = (int64_t)(lv & emask);
+            }
+            if (nxt.N == 0) break;
+            ++d;
+            if (cta0 && tid == 0) {
+                int64_t *l = P.lvl + 4 * (int64_t)d;
+                l[0] = nxt.p0; l[1] = nxt.N; l[2] = nxt.E; l[3] = nxt.tb;
+            }
+            if (d > P.n + 1) __trap();  // impossible for a correct BFS: fail loudly, never spin
+            prev = cur;
+            cur = nxt;
+        }
+        const int D = d;  // deepest non-empty level of the batch
+        if (cta0 && tid == 0) {
+            C->st_levels += D + 2;
+            C->st_pull_levels += pulls;
+            C->st_fwd_edges += fwd_edges;
+            if (D > C->st_max_depth) C->st_max_depth = D;
+        }
+        // ---------------- backward, L = D..1 (Alg.1 l.29-47); level L+2 retired on the way
+        int64_t bwd_edges = 0;
+        for (int L = D; L >= 1; --L) {
+            const int64_t *l = P.lvl + 4 * (int64_t)L;
+            const Lv lv{l[0], l[1], l[2], l[3]};
+            const BOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0};
+            bpass<B_BWD>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.list_beg + lv.p0, P.list_m + lv.p0,
+                         P.tiles + lv.tb, lv.N, lv.E, P.out_idx, fr[(L + 1) & 1], fr[L & 1], 0u, gwarp, nwarps, none);
+            bwd_edges += lv.E;
+            if (L + 2 <= D) {
+                const int64_t *l2 = P.lvl + 4 * (int64_t)(L + 2);
+                bclear(P, Lv{l2[0], l2[1], l2[2], l2[3]}, fr[L & 1], gwarp, nwarps);
+            }
+            bsync(C, gen, ncta);
+        }
+        // retire levels 0..min(2, D)
+        for (int L = 0; L <= min(2, D); ++L) {
+            const int64_t *l = P.lvl + 4 * (int64_t)L;
+            bclear(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps);
+        }
+        if (cta0 && tid == 0) {
+            C->st_bwd_edges += bwd_edges;
+            C->st_scans += pulls;
+        }
+        bsync(C, gen, ncta);
+    }
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ host side
+
+static tbc_status batch_alloc(tbc_graph *g) {
+    BatchWorkspace &w = g->bws;
+    if (w.ready) return TBC_OK;
+    const int64_t n = g->n, m = g->m;
+    cudaStream_t s = g->stream;
+    cudaError_t e = cudaSuccess;
+    auto alloc = [&](auto **p, size_t cnt) -> cudaError_t {
+        size_t bytes = sizeof(**p) * (cnt > 0 ? cnt : 1);
+        cudaError_t r = cudaMalloc((void **)p, bytes);
+        if (r == cudaSuccess) g->device_bytes += bytes;
+        return r;
+    };
+    // every (vertex, level) pair of a batch has at least one lane: <= 32 n list entries, and the
+    // levels' tiles sum to <= (32 n + 32 m) / kBT + (levels <= n + 1)
+    w.list_cap = (int64_t)kBatch * n + kPad;
+    w.tiles_cap = ((int64_t)kBatch * (n + m)) / kBT + n + 2 + kPad;
+    w.cand_tiles_cap = (n + m) / kBT + 2 + kPad;
+    if ((e = alloc(&w.sig, (size_t)n * kBatch)) || (e = alloc(&w.du, (size_t)n * kBatch)) || (e = alloc(&w.vis, n)) ||
+        (e = alloc(&w.fr[0], n)) || (e = alloc(&w.fr[1], n)) || (e = alloc(&w.list_v, w.list_cap)) ||
+        (e = alloc(&w.list_pre, w.list_cap)) || (e = alloc(&w.list_beg, w.list_cap)) ||
+        (e = alloc(&w.list_m, w.list_cap)) || (e = alloc(&w.tiles, w.tiles_cap)) ||
+        (e = alloc(&w.cand_v, n + kPad)) || (e = alloc(&w.cand_pre, n + kPad)) || (e = alloc(&w.cand_beg, n + kPad)) ||
+        (e = alloc(&w.cand_tiles, w.cand_tiles_cap)) || (e = alloc(&w.lvl, 4 * (n + 2))) || (e = alloc(&w.ctr, 1)))
+        return cuda_error(e, "batch workspace cudaMalloc");
+    if ((e = cudaMemsetAsync(w.sig, 0, sizeof(double) * n * kBatch, s)) ||
+        (e = cudaMemsetAsync(w.du, 0, sizeof(double) * n * kBatch, s)) ||
+        (e = cudaMemsetAsync(w.vis, 0, sizeof(uint32_t) * n, s)) ||
+        (e = cudaMemsetAsync(w.fr[0], 0, sizeof(uint32_t) * n, s)) ||
+        (e = cudaMemsetAsync(w.fr[1], 0, sizeof(uint32_t) * n, s)) ||
+        (e = cudaMemsetAsync(w.ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s)))
+        return cuda_error(e, "batch workspace init");
+    int per_sm = 0, sms = 0;
+    if ((e = cudaFuncSetAttribute(k_bcb, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmem)) ||
+        (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_bcb, kBB, kBSmem)) ||
+        (e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device)))
+        return cuda_error(e, "batch occupancy query");
+    if (per_sm < 1) return set_error(TBC_ERR_CUDA, "k_bcb cannot be resident (occupancy 0)");
+    g->bgrid = per_sm * sms;
+    w.ready = true;
+    return TBC_OK;
+}
+
+void batch_free(tbc_graph *g) {
+    BatchWorkspace &w = g->bws;
+    void *ps[] = {w.sig, w.du, w.vis, w.fr[0], w.fr[1], w.list_v, w.list_pre, w.list_beg, w.list_m, w.tiles,
+                  w.cand_v, w.cand_pre, w.cand_beg, w.cand_tiles, w.lvl, w.ctr};
+    for (void *p : ps) cudaFree(p);
+    w = BatchWorkspace{};
+}
+
+tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream) {
+    tbc_status st = batch_alloc(g);
+    if (st != TBC_OK) return st;
+    const BatchWorkspace &w = g->bws;
+    BParams P{};
+    P.n = g->n;
+    P.m = g->m;
+    P.in_ptr = g->in_ptr;
+    P.in_idx = g->in_idx;
+    P.out_ptr = g->out_ptr;
+    P.out_idx = g->out_idx;
+    P.deg2 = g->deg2;
+    P.sig = w.sig;
+    P.du = w.du;
+    P.vis = w.vis;
+    P.fr0 = w.fr[0];
+    P.fr1 = w.fr[1];
+    P.list_v = w.list_v;
+    P.list_pre = w.list_pre;
+    P.list_beg = w.list_beg;
+    P.list_m = w.list_m;
+    P.tiles = w.tiles;
+    P.cand_v = w.cand_v;
+    P.cand_pre = w.cand_pre;
+    P.cand_beg = w.cand_beg;
+    P.cand_tiles = w.cand_tiles;
+    P.lvl = w.lvl;
+    P.ctr = w.ctr;
+    P.bc = d_bc;
+    P.sources = d_sources;
+    P.perm = g->perm;
+    P.inv = g->inv;
+    P.k = k;
+    P.n_scan = g->n_scan;
+    P.list_cap = w.list_cap;
+    P.tiles_cap = w.tiles_cap;
+    P.cand_tiles_cap = w.cand_tiles_cap;
+    P.bc_scale = g->directed ? 1.0 : 0.5;
+    P.pull_ratio = g->batch_pull;
+    P.ebits = g->ebits;
+    P.dir_mode = g->dir_mode;
+    void *args[] = {&P};
+    cudaError_t e =
+        cudaLaunchCooperativeKernel((const void *)k_bcb, dim3(g->bgrid), dim3(kBB), args, kBSmem, stream);
+    if (e != cudaSuccess) return cuda_error(e, "cudaLaunchCooperativeKernel(k_bcb)");
+    return TBC_OK;
+}
+
+}  // namespace tbc

@@ -23,6 +23,7 @@
 #include <cstdio>
 
 #include "tbc_internal.cuh"
+#include "tbc_device.cuh"
 
 namespace tbc {
 namespace {
@@ -85,27 +86,6 @@ __shared__ unsigned long long tbc_sprof[kWarpsPerBlock][PR_SLOTS];
 
 // ------------------------------------------------------------------ memory-model helpers
 
-__device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
-    unsigned v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-
-__device__ __forceinline__ void fence_acq_rel() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
-
-__device__ __forceinline__ uint64_t policy_evict_first() {
-    uint64_t p;
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
-
-// streaming read of graph indices: read-only for the whole kernel, L1 no-allocate, L2 evict-first
-__device__ __forceinline__ int ld_stream(const int32_t *ptr, uint64_t pol) {
-    int v;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(ptr), "l"(pol));
-    return v;
-}
-
 // ---- TMA bulk copies (cp.async.bulk) completing on an mbarrier: the edge-stream pipeline
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -143,18 +123,6 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned by
 
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
-
-__device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned long long *p) {
-    return *(volatile const unsigned long long *)p;
-}
-
-__device__ __forceinline__ unsigned long long globaltimer_ns() {
-    unsigned long long t;
-    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
-    return t;
-}
-
-constexpr unsigned long long kWatchdogNs = 20ull * 1000 * 1000 * 1000;  // 20 s at one barrier
 
 // Grid-wide barrier of the cooperative (co-resident) grid: release fence + arrival atomic,
 // the last arriver bumps the generation; waiters acquire it.  The acquire-side gpu fence also
@@ -1284,6 +1252,7 @@ void engine_free(tbc_graph *g) {
         w = Workspace{};
     }
     g->ws_count = 0;
+    batch_free(g);
     cudaFree(g->gctr);
     cudaFree(g->trace);
     g->gctr = nullptr;
@@ -1334,6 +1303,8 @@ tbc_status engine_setup(tbc_graph *g) {
 
 tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
                       int bfs_only) {
+    // the batched engine (tbc_batch.cu) runs every bc call of the CSC engine unless TBC_OPT_BATCH = 0
+    if (!bfs_only && g->batch && g->engine == TBC_ENGINE_CSC) return batch_run(g, d_sources, k, d_bc, stream);
     // SM partitions: never more than the sources (a partition without sources only waits)
     int np = g->nparts;
     if (bfs_only || k < 1) np = 1;

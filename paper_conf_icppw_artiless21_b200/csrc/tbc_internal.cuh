@@ -115,6 +115,28 @@ struct Workspace {
     double *bc_part = nullptr;    // partial bc of this partition (zero between calls)
 };
 constexpr int kMaxPartitions = 8;
+
+// workspace of the batched engine (tbc_batch.cu): 32 sources per sweep, one per warp lane
+constexpr int kBatch = 32;
+struct BatchWorkspace {
+    double *sig = nullptr;       // [n][32] sigma of (vertex, lane)
+    double *du = nullptr;        // [n][32] delta_u of (vertex, lane) (backward)
+    uint32_t *vis = nullptr;     // [n] lanes that have reached the vertex
+    uint32_t *fr[2] = {nullptr, nullptr};  // [n] dense level masks, by level parity
+    int32_t *list_v = nullptr;   // level lists (levels concatenated), capacity list_cap
+    uint32_t *list_pre = nullptr;  // out-degree prefix, relative to the level
+    uint32_t *list_beg = nullptr;  // out_ptr of the entry
+    uint32_t *list_m = nullptr;    // lanes on this level
+    int32_t *tiles = nullptr;      // per level: owner starting each warp tile, capacity tiles_cap
+    int32_t *cand_v = nullptr;     // pull candidates (in-degree prefix)
+    uint32_t *cand_pre = nullptr;
+    uint32_t *cand_beg = nullptr;
+    int32_t *cand_tiles = nullptr;
+    int64_t *lvl = nullptr;        // per level: p0, N, E, tile base
+    Ctrs *ctr = nullptr;
+    int64_t list_cap = 0, tiles_cap = 0, cand_tiles_cap = 0;
+    bool ready = false;
+};
 }  // namespace tbc
 
 struct tbc_graph {
@@ -149,6 +171,10 @@ struct tbc_graph {
     int bwd_mode = 0;
     int fmt_mode = 0;
     double c_list = 12.0, c_stream = 4.0, c_atom = 18.0, c_vert = 10.0, c_scan = 3.0, c_bpush = 6.0;
+    int batch = 1;                // TBC_OPT_BATCH: 1 batched engine (32 sources per sweep), 0 per source
+    double batch_pull = 8.0;      // TBC_OPT_BATCH_PULL: pull when frontier out-edges x this > m
+    tbc::BatchWorkspace bws;
+    int bgrid = 0;
     int64_t *trace = nullptr;     // device, 8 * kTraceCap int64
     int64_t trace_src = -1;       // index in the next call's source list to trace (-1: off)
     cudaStream_t stream = nullptr;  // internal stream for the synchronous host API
@@ -165,4 +191,7 @@ tbc_status engine_workspaces(tbc_graph *g, int count);  // allocate partitions [
 void engine_free(tbc_graph *g);                          // workspaces + shared counters
 tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc,
                       cudaStream_t stream, int bfs_only);
+// batched engine (tbc_batch.cu)
+tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream);
+void batch_free(tbc_graph *g);
 }  // namespace tbc

@@ -16,15 +16,18 @@ pytestmark = pytest.mark.gpu
 # (forward direction, format, backward direction) triples: every forward/backward pass kind
 # gets exercised -- (PULL, LIST) forces the candidate scan + list pull after the first push
 # level; backward 1 = pull over level L's out-edges only, 2 = push from level L+1 (in-edges)
-MODES = [(tbc.DIR_AUTO, tbc.FMT_AUTO, 0), (tbc.DIR_PUSH, tbc.FMT_LIST, 1), (tbc.DIR_PUSH, tbc.FMT_STREAM, 0),
-         (tbc.DIR_PULL, tbc.FMT_AUTO, 0), (tbc.DIR_PULL, tbc.FMT_STREAM, 0), (tbc.DIR_PULL, tbc.FMT_LIST, 2),
-         (tbc.DIR_AUTO, tbc.FMT_LIST, 2)]
+# the 4th element selects the engine: 1 batched (32 sources per sweep, the default), 0 per source
+MODES = [(tbc.DIR_AUTO, tbc.FMT_AUTO, 0, 1), (tbc.DIR_PUSH, tbc.FMT_AUTO, 0, 1), (tbc.DIR_PULL, tbc.FMT_AUTO, 0, 1),
+         (tbc.DIR_AUTO, tbc.FMT_AUTO, 0, 0), (tbc.DIR_PUSH, tbc.FMT_LIST, 1, 0), (tbc.DIR_PUSH, tbc.FMT_STREAM, 0, 0),
+         (tbc.DIR_PULL, tbc.FMT_AUTO, 0, 0), (tbc.DIR_PULL, tbc.FMT_STREAM, 0, 0), (tbc.DIR_PULL, tbc.FMT_LIST, 2, 0),
+         (tbc.DIR_AUTO, tbc.FMT_LIST, 2, 0)]
 
 
 def set_mode(G, mode):
     G.set_direction(mode[0])
     G.set_format(mode[1])
     G.set_bwd_direction(mode[2] if len(mode) > 2 else 0)
+    G.set_batch(mode[3] if len(mode) > 3 else 1)
 
 
 def assert_bc(got, want, rel=1e-9):
@@ -61,7 +64,7 @@ SMALL = [gg.star(7), gg.star(7, directed_both=True), gg.path(7), gg.path(7, dire
 
 
 @pytest.mark.parametrize("engine", ENGINES)
-@pytest.mark.parametrize("mode", MODES, ids=lambda m: f"dir{m[0]}fmt{m[1]}bwd{m[2]}")
+@pytest.mark.parametrize("mode", MODES, ids=lambda m: f"dir{m[0]}fmt{m[1]}bwd{m[2]}b{m[3]}")
 @pytest.mark.parametrize("g", SMALL, ids=lambda g: g.name)
 def test_small_graphs_all_sources(g, mode, engine):
     with gpu_graph(g, engine=engine, reorder=(mode[1] != tbc.FMT_LIST)) as G:
@@ -102,6 +105,7 @@ def test_sm_partitions(directed):
     src = gg.sources(g, 37, seed=3)
     want = oracle.bc(g.col_ptr, g.row_idx, directed, src)
     with gpu_graph(g) as G:
+        G.set_batch(0)
         for parts in (1, 2, 3, 4, 8):
             G.set_partitions(parts)
             a = G.bc(src)
@@ -112,6 +116,27 @@ def test_sm_partitions(directed):
         assert_bfs(g, G, src[5])
         with pytest.raises(tbc.TBCError):
             G.set_partitions(9)
+
+
+@pytest.mark.parametrize("directed", [False, True])
+@pytest.mark.parametrize("pull", [0.0, 8.0, 1e9])
+def test_batched_engine(directed, pull):
+    """Batched engine: several sweeps (full and ragged last batch of 32), repeated sources inside a
+    batch and across batches, push-only / auto / pull-from-level-2 forward levels; repeat runs agree
+    to rounding (fp64 atomics of split owners)."""
+    g = gg.kronecker(13, 16, seed=4, directed=directed, device="cuda")
+    src = gg.sources(g, 77, seed=3)
+    src = np.concatenate([src, src[:5], src[10:12], src[10:12]]).astype(np.int32)
+    want = oracle.bc(g.col_ptr, g.row_idx, directed, src)
+    with gpu_graph(g) as G:
+        G.set_batch(1)
+        G.set_batch_pull(pull)
+        a = G.bc(src)
+        assert_bc(a, want)
+        assert_bc(G.bc(src), a, rel=1e-12)
+        assert_bc(G.bc(src[:1]), oracle.bc(g.col_ptr, g.row_idx, directed, src[:1]))
+        st = G.stats()
+        assert st["sources"] == len(src) * 2 + 1
 
 
 def test_grid_sigma_crosses_2_53():

@@ -34,7 +34,9 @@ for setting in a.settings.split(";"):
     G.set_format(int(kv.get("fmt", 0)))
     G.set_direction(int(kv.get("dir", 0)))
     G.set_bwd_direction(int(kv.get("bwd", 0)))
-    G.set_partitions(int(kv.get("parts", 4)))
+    G.set_partitions(int(kv.get("parts", 8)))
+    G.set_batch(int(kv.get("batch", 1)))
+    G.set_batch_pull(float(kv.get("bpull", 8)))
     G.set_cost(**{k: float(v) for k, v in kv.items() if k in ("list", "stream", "atomic", "vertex", "scan", "bpush")})
     G.bc_device(s_d, bc, st)  # warm-up
     torch.cuda.synchronize()
@@ -54,7 +56,8 @@ for setting in a.settings.split(";"):
                       "gteps": a.sources * g.nnz / (ms / 1e3) / 1e9,
                       "fwd_edges_per_src": s["fwd_edges"] / max(s["sources"], 1),
                       "bwd_edges_per_src": s["bwd_edges"] / max(s["sources"], 1),
-                      "pull_levels": s["pull_levels"] / max(s["sources"], 1)}), flush=True)
+                      "pull_levels": s["pull_levels"] / max(s["sources"], 1),
+                      "levels": s["levels"], "reached_per_src": s["reached"] / max(s["sources"], 1)}), flush=True)
     if prof:
         pr = G.profile()
         tot = sum(pr.values()) or 1

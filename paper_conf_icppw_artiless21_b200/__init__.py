@@ -206,7 +206,9 @@ class Graph:
 
     PROFILE_REGIONS = (["barrier"] + [f"{m}_{r}" for m in ("push", "pull", "bwd", "bpush")
                                       for r in ("window", "index", "gather", "tail")]
-                       + ["stream_push", "stream_pull", "stream_bwd", "pull_owner", "scan", "bwd_owner", "other"])
+                       + ["stream_push", "stream_pull", "stream_bwd", "pull_owner", "scan", "bwd_owner", "other"]
+                       + ["b_push_slots", "b_push_pairs", "b_pull_slots", "b_pull_pairs", "b_bwd_slots", "b_bwd_pairs",
+                          "b_edge_slots", "b_owners"])
 
     def profile(self) -> dict:
         """Region profile of a -DTBC_PROF library (warp-cycles per region; resets on read)."""

@@ -40,6 +40,10 @@ constexpr int kBWarps = kBB / 32;
 constexpr int kBI = 2;           // tile items per lane (window / index phases)
 constexpr int kBT = 32 * kBI;    // diagonal items (owner end items + edges) per warp tile
 constexpr int kPad = 8;
+#ifndef TBC_BUNROLL
+#define TBC_BUNROLL 4
+#endif
+constexpr int kBU = TBC_BUNROLL;  // gathers in flight per lane in the slot loop
 
 enum { B_PUSH = 0, B_PULL = 1, B_BWD = 2 };
 
@@ -61,6 +65,7 @@ struct BParams {
     int32_t *cand_tiles;
     int64_t *lvl;
     Ctrs *ctr;
+    Ctrs *gctr;  // TBC_PROF builds: slot statistics in gctr->prof[24..31]
     double *bc;
     const int32_t *sources;
     const int32_t *__restrict__ perm;
@@ -78,7 +83,6 @@ struct __align__(16) BWarpSmem {
     int32_t fl[kBT + 2];     // bit 0: the tile holds the owner's first item; bit 1: whole owner
     int32_t own[kBT + 2];    // owner (window index) of each slot
     int32_t x[kBT];          // other end of each slot
-    uint32_t em[kBT];        // lanes of each slot
     int32_t claim[kBT + 2];  // vertices discovered by this tile (PULL)
 };
 constexpr size_t kBSmem = sizeof(BWarpSmem) * kBWarps;
@@ -182,6 +186,20 @@ __device__ __forceinline__ void span(const int64_t *ptr, int32_t v, uint32_t &dg
     dg = (uint32_t)(ptr[v + 1] - b);
 }
 
+// 32 x 32 bit transpose across the warp: lane l holds row l (bit c = column c); afterwards lane c
+// holds column c (bit l = row l).  Five rounds of block swaps with the partner lane l ^ j.
+__device__ __forceinline__ uint32_t transpose32(uint32_t x) {
+    const int lane = threadIdx.x & 31;
+    constexpr uint32_t hi[5] = {0xFFFF0000u, 0xFF00FF00u, 0xF0F0F0F0u, 0xCCCCCCCCu, 0xAAAAAAAAu};
+#pragma unroll
+    for (int r = 0; r < 5; ++r) {
+        const int j = 16 >> r;
+        const uint32_t y = __shfl_xor_sync(FULL, x, j);
+        x = (lane & j) ? ((x & hi[r]) | ((y >> j) & ~hi[r])) : ((x & ~hi[r]) | ((y << j) & hi[r]));
+    }
+    return x;
+}
+
 __device__ __forceinline__ uint64_t slot_range(int s0, int s1) {
     if (s0 >= 64 || s1 <= s0) return 0ull;
     const uint64_t hi = s1 >= 64 ? ~0ull : ((1ull << s1) - 1ull);
@@ -278,9 +296,25 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                 ems[i] = g & ws.msk[ws.own[sl]];
             }
             ws.x[sl] = xs[i];
-            ws.em[sl] = ems[i];
             act |= (uint64_t)__ballot_sync(FULL, ems[i] != 0u) << (32 * i);
         }
+        // this lane's (source's) slots: the transpose of the slots' lane masks
+        static_assert(kBI == 2, "64 slots per tile: two 32 x 32 transposes");
+        const uint64_t lm = (uint64_t)transpose32(ems[0]) | ((uint64_t)transpose32(ems[1]) << 32);
+#ifdef TBC_PROF
+        {
+            unsigned pairs = 0;
+#pragma unroll
+            for (int i = 0; i < kBI; ++i) pairs += __popc(ems[i]);
+            pairs = __reduce_add_sync(FULL, pairs);
+            if (lane == 0) {
+                atomicAdd(&P.gctr->prof[24 + 2 * MODE], (unsigned long long)__popcll(act));
+                atomicAdd(&P.gctr->prof[25 + 2 * MODE], (unsigned long long)pairs);
+                atomicAdd(&P.gctr->prof[30], (unsigned long long)ne);
+                atomicAdd(&P.gctr->prof[31], (unsigned long long)nwin);
+            }
+        }
+#endif
         if (MODE == B_PUSH) {
             // claims: the atomicOr that lifts fr_out[x] from 0 appends x to the next level
             bool cl[kBI];
@@ -305,35 +339,36 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             const int32_t v = ws.v[j];
             const uint32_t m = ws.msk[j];
             const bool in = (m >> lane) & 1u;
+            // each lane walks only its own source's slots of this owner (divergent loop, no
+            // collectives inside): warp iterations = the busiest lane's count, not the slots'
+            uint64_t mine = lm & bits;
             if (MODE == B_PUSH) {
                 const double su = in ? sig[(int64_t)v * kBatch + lane] : 0.0;
-                while (bits) {
-                    const int sl = __ffsll((long long)bits) - 1;
-                    bits &= bits - 1;
-                    if ((ws.em[sl] >> lane) & 1u) atomicAdd(&sig[(int64_t)ws.x[sl] * kBatch + lane], su);
+                while (mine) {
+                    const int sl = __ffsll((long long)mine) - 1;
+                    mine &= mine - 1;
+                    atomicAdd(&sig[(int64_t)ws.x[sl] * kBatch + lane], su);
                 }
                 continue;
             }
             const double *src = (MODE == B_PULL) ? sig : P.du;
             const double sv = (MODE == B_BWD && in) ? sig[(int64_t)v * kBatch + lane] : 1.0;
             double acc = 0.0;
-            while (bits) {  // four slots in flight per lane
-                int sl[4];
+            while (mine) {  // kBU gathers in flight per lane
+                int sl[kBU];
 #pragma unroll
-                for (int q = 0; q < 4; ++q) {
+                for (int q = 0; q < kBU; ++q) {
                     sl[q] = -1;
-                    if (bits) {
-                        sl[q] = __ffsll((long long)bits) - 1;
-                        bits &= bits - 1;
+                    if (mine) {
+                        sl[q] = __ffsll((long long)mine) - 1;
+                        mine &= mine - 1;
                     }
                 }
-                double a[4];
+                double a[kBU];
 #pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    a[q] = 0.0;
-                    if (sl[q] >= 0 && ((ws.em[sl[q]] >> lane) & 1u)) a[q] = src[(int64_t)ws.x[sl[q]] * kBatch + lane];
-                }
-                acc += (a[0] + a[1]) + (a[2] + a[3]);
+                for (int q = 0; q < kBU; ++q) a[q] = sl[q] >= 0 ? src[(int64_t)ws.x[sl[q]] * kBatch + lane] : 0.0;
+#pragma unroll
+                for (int q = 0; q < kBU; ++q) acc += a[q];
             }
             if (MODE == B_PULL) {
                 // Alg.1 l.20-25: lanes with a non-zero masked sum are discovered on this level
@@ -699,6 +734,7 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
     P.cand_tiles = w.cand_tiles;
     P.lvl = w.lvl;
     P.ctr = w.ctr;
+    P.gctr = g->gctr;
     P.bc = d_bc;
     P.sources = d_sources;
     P.perm = g->perm;

@@ -61,7 +61,10 @@ for setting in a.settings.split(";"):
     if prof:
         pr = G.profile()
         tot = sum(pr.values()) or 1
-        print("PROFILE " + setting + " " + " ".join(f"{k}={100 * v / tot:.1f}" for k, v in pr.items() if v), flush=True)
+        reg = {k: v for k, v in pr.items() if not k.startswith("b_")}
+        tot = sum(reg.values()) or 1
+        print("PROFILE " + setting + " " + " ".join(f"{k}={100 * v / tot:.1f}" for k, v in reg.items() if v), flush=True)
+        print("COUNTS " + setting + " " + " ".join(f"{k}={v}" for k, v in pr.items() if k.startswith("b_")), flush=True)
     for t in [int(x) for x in a.trace.split(",") if x]:
         G.set_trace(t)
         G.bc(src[: t + 1])

@@ -41,7 +41,7 @@ constexpr int kBI = 2;           // tile items per lane (window / index phases)
 constexpr int kBT = 32 * kBI;    // diagonal items (owner end items + edges) per warp tile
 constexpr int kPad = 8;
 #ifndef TBC_BUNROLL
-#define TBC_BUNROLL 4
+#define TBC_BUNROLL 6
 #endif
 constexpr int kBU = TBC_BUNROLL;  // gathers in flight per lane in the slot loop
 
@@ -73,6 +73,8 @@ struct BParams {
     int64_t k, n_scan, list_cap, tiles_cap, cand_tiles_cap;
     double bc_scale, pull_ratio;
     int ebits, dir_mode;
+    int64_t *trace;  // per-phase timeline of batch trace_b (TBC_OPT_TRACE: source index / 32)
+    int64_t trace_cap, trace_b;
 };
 
 struct __align__(16) BWarpSmem {
@@ -92,6 +94,18 @@ struct Lv {
 };
 
 __device__ __forceinline__ int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// timeline entry {t_ns, kind, level, N, E, a, b, 0} after a barrier (CTA 0, thread 0; traced batch)
+// kinds as tbc_trace_get: 0 init, 1 level masks + candidates (B phase), 2 push, 3 pull, 4 backward
+__device__ __forceinline__ void btrace(const BParams &P, bool on, int kind, int64_t level, int64_t N, int64_t E,
+                                       int64_t a, int64_t b) {
+    if (!on || blockIdx.x != 0 || threadIdx.x != 0) return;
+    const unsigned long long i = P.gctr->trace_n;
+    if ((int64_t)i >= P.trace_cap) return;
+    int64_t *t = P.trace + 8 * i;
+    t[0] = (int64_t)globaltimer_ns(); t[1] = kind; t[2] = level; t[3] = N; t[4] = E; t[5] = a; t[6] = b; t[7] = 0;
+    P.gctr->trace_n = i + 1;
+}
 
 // grid barrier (as tbc_engine.cu): the last arriver snapshots {list, active, cand} counters
 __device__ __forceinline__ void bsync(Ctrs *c, unsigned &gen, unsigned nblocks) {
@@ -344,31 +358,39 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             uint64_t mine = lm & bits;
             if (MODE == B_PUSH) {
                 const double su = in ? sig[(int64_t)v * kBatch + lane] : 0.0;
-                while (mine) {
-                    const int sl = __ffsll((long long)mine) - 1;
-                    mine &= mine - 1;
-                    atomicAdd(&sig[(int64_t)ws.x[sl] * kBatch + lane], su);
+#pragma unroll
+                for (int h = 0; h < kBI; ++h) {
+                    uint32_t mm = (uint32_t)(mine >> (32 * h));
+                    while (mm) {
+                        const int sl = 32 * h + __ffs(mm) - 1;
+                        mm &= mm - 1;
+                        atomicAdd(&sig[(int64_t)ws.x[sl] * kBatch + lane], su);
+                    }
                 }
                 continue;
             }
             const double *src = (MODE == B_PULL) ? sig : P.du;
             const double sv = (MODE == B_BWD && in) ? sig[(int64_t)v * kBatch + lane] : 1.0;
             double acc = 0.0;
-            while (mine) {  // kBU gathers in flight per lane
-                int sl[kBU];
+            // the two 32-slot halves of the tile, kBU gathers in flight per lane; __ffs(0) = 0
+            // marks the exhausted positions
 #pragma unroll
-                for (int q = 0; q < kBU; ++q) {
-                    sl[q] = -1;
-                    if (mine) {
-                        sl[q] = __ffsll((long long)mine) - 1;
-                        mine &= mine - 1;
+            for (int h = 0; h < kBI; ++h) {
+                uint32_t mm = (uint32_t)(mine >> (32 * h));
+                const int32_t *xh = ws.x + 32 * h;
+                while (mm) {
+                    int sl[kBU];
+#pragma unroll
+                    for (int q = 0; q < kBU; ++q) {
+                        sl[q] = __ffs(mm) - 1;
+                        mm &= mm - 1;
                     }
+                    double a[kBU];
+#pragma unroll
+                    for (int q = 0; q < kBU; ++q) a[q] = sl[q] >= 0 ? src[(int64_t)xh[sl[q]] * kBatch + lane] : 0.0;
+#pragma unroll
+                    for (int q = 0; q < kBU; ++q) acc += a[q];
                 }
-                double a[kBU];
-#pragma unroll
-                for (int q = 0; q < kBU; ++q) a[q] = sl[q] >= 0 ? src[(int64_t)ws.x[sl[q]] * kBatch + lane] : 0.0;
-#pragma unroll
-                for (int q = 0; q < kBU; ++q) acc += a[q];
             }
             if (MODE == B_PULL) {
                 // Alg.1 l.20-25: lanes with a non-zero masked sum are discovered on this level
@@ -513,7 +535,10 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
                 C->st_sources += __popc(valid);
             }
         }
+        const bool tr = b == P.trace_b;
+        if (tr && cta0 && tid == 0) P.gctr->trace_n = 0;
         bsync(C, gen, ncta);
+        btrace(P, tr, 0, 0, 0, 0, 0, 0);
         Lv cur{0, (int64_t)(ld_volatile_u64(&C->snap[0]) >> P.ebits), (int64_t)(ld_volatile_u64(&C->snap[0]) & emask), 0};
         if (cur.N == 0) continue;  // every lane invalid: nothing was written
         if (cta0 && tid == 0) {
@@ -579,6 +604,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
                 }
             }
             bsync(C, gen, ncta);
+            btrace(P, tr, 1, d, cur.N, cur.E, pull, 0);
             active = (uint32_t)ld_volatile_u64(&C->snap[1]);
             const unsigned long long cs = ld_volatile_u64(&C->snap[2]);
             // ---- A(d+1)
@@ -607,6 +633,8 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
                 nxt.N = (int64_t)(lv >> P.ebits);
                 nxt.E = (int64_t)(lv & emask);
             }
+            btrace(P, tr, pull ? 3 : 2, d + 1, nxt.N, nxt.E, pull ? (int64_t)(cs >> P.ebits) : cur.N,
+                   pull ? (int64_t)(cs & emask) : cur.E);
             if (nxt.N == 0) break;
             ++d;
             if (cta0 && tid == 0) {
@@ -638,6 +666,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
                 bclear(P, Lv{l2[0], l2[1], l2[2], l2[3]}, fr[L & 1], gwarp, nwarps);
             }
             bsync(C, gen, ncta);
+            btrace(P, tr, 4, L, lv.N, lv.E, 0, 0);
         }
         // retire levels 0..min(2, D)
         for (int L = 0; L <= min(2, D); ++L) {
@@ -649,6 +678,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
             C->st_scans += pulls;
         }
         bsync(C, gen, ncta);
+        btrace(P, tr, 5, 0, 0, 0, 0, 0);
     }
 }
 
@@ -748,6 +778,9 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
     P.pull_ratio = g->batch_pull;
     P.ebits = g->ebits;
     P.dir_mode = g->dir_mode;
+    P.trace = g->trace;
+    P.trace_cap = g->trace ? kTraceCap : 0;
+    P.trace_b = g->trace_src >= 0 ? g->trace_src / kBatch : -1;
     void *args[] = {&P};
     cudaError_t e =
         cudaLaunchCooperativeKernel((const void *)k_bcb, dim3(g->bgrid), dim3(kBB), args, kBSmem, stream);

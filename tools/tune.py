@@ -67,7 +67,7 @@ for setting in a.settings.split(";"):
         print("COUNTS " + setting + " " + " ".join(f"{k}={v}" for k, v in pr.items() if k.startswith("b_")), flush=True)
     for t in [int(x) for x in a.trace.split(",") if x]:
         G.set_trace(t)
-        G.bc(src[: t + 1])
+        G.bc(src[: 32 * (t // 32 + 1)])
         for r in G.trace():
             print("TRACE " + json.dumps({"setting": setting, "src": t, **r}), flush=True)
         G.set_trace(-1)

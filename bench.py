@@ -45,6 +45,7 @@ def parse():
     ap.add_argument("--direction", type=int, default=0)
     ap.add_argument("--format", type=int, default=0, help="0 auto, 1 list passes, 2 edge streams")
     ap.add_argument("--engine", choices=["csc", "coot"], default="csc")
+    ap.add_argument("--batch", type=int, default=1, help="1: batched engine (32 sources per sweep), 0: per source")
     ap.add_argument("--cost", default="", help="cost model overrides, e.g. list=10,stream=2")
     ap.add_argument("--trace", type=int, default=-1, help="print the per-level timeline of this source to stderr")
     return ap.parse_args()
@@ -208,6 +209,9 @@ def main():
     create_s = time.time() - t0
     G.set_direction(args.direction)
     G.set_format(args.format)
+    G.set_batch(args.batch)
+    batched = bool(args.batch) and args.engine == "csc"
+    kname = "k_bcb" if batched else "k_bc"
     if args.cost:
         G.set_cost(**{k: float(v) for k, v in (kv.split("=") for kv in args.cost.split(","))})
     src_d = torch.from_numpy(my_src).to(dev)
@@ -254,7 +258,7 @@ def main():
     gteps = sources_total * g.nnz / (total_ms / 1e3) / 1e9
     ms_per_step = total_ms / args.steps
 
-    # roofline of k_bc (the only kernel of the hot path): SURVEY 8(d) algorithmic bytes
+    # roofline of the hot-path kernel (k_bcb batched, or k_bc per source): SURVEY 8(d) algorithmic bytes
     # B_min = 8 B per out-edge of the reached set (4 B index read once per stage) + 80 B per
     # reached vertex, summed over the launch's sources; / the kernel's event-timed duration.
     alg_bytes_per_launch = (8.0 * st["reached_edges"] + 80.0 * st["reached"]) / args.steps
@@ -262,7 +266,7 @@ def main():
     peak, peak_kind = peaks()
     achieved = alg_bytes_per_launch / k_avg_s / 1e9
     traffic = None
-    tpath = os.path.join(ROOT, "profiles", f"traffic_cfg{args.config}.json")
+    tpath = os.path.join(ROOT, "profiles", f"traffic_cfg{args.config}_{kname}.json")
     if os.path.exists(tpath):
         try:
             tj = json.load(open(tpath))
@@ -303,12 +307,14 @@ def main():
                        "l2": "inputs larger than L2 (CSC+CSR %.0f MB vs 126 MB L2); no flush" %
                              ((8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) / 1e6),
                        "direction": args.direction, "format": args.format, "engine_kind": args.engine,
+                       "engine_mode": "batched, 32 sources per sweep (one per warp lane)" if batched
+                       else "per source, SM partitions",
                        "cost": args.cost},
             "clocks": clocks,
             "gpu_launches": args.steps,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
-                         "kernel": "k_bc", "alg_bytes_per_launch": alg_bytes_per_launch,
+                         "kernel": kname, "alg_bytes_per_launch": alg_bytes_per_launch,
                          "kernel_ms": statistics.mean(kern_ms)},
             "e2e": {"value": e2e_gteps, "unit": "GTEPS", "h2d_bytes_per_step": 4 * len(my_src),
                     "d2h_bytes_per_step": 8 * g.n},

@@ -91,14 +91,17 @@ enum {
                                 are summed in partition order at the end of the call (deterministic
                                 for a given value).  Costs one workspace (~50 B/vertex + 8 B/edge/64)
                                 per partition.  Per-source engine only. */
-    TBC_OPT_BATCH = 12,      /* bc engine: 1 (default) batched -- 32 sources per sweep, one per warp
-                                lane, A^T times an n x 32 frontier block; 0 the
+    TBC_OPT_BATCH = 12,      /* bc engine: 1 (default) batched -- W sources per sweep (W = 32 or 64,
+                                TBC_OPT_BATCH_WIDTH), A^T times an n x W frontier block; 0 the
                                 per-source engine.  tbc_bfs and TBC_ENGINE_COOT always use the
                                 per-source engine.  The batched workspace holds 2 x 256 B/vertex of
                                 (sigma, delta_u) rows plus level lists of <= 32 entries per vertex. */
-    TBC_OPT_BATCH_PULL = 13  /* batched engine: a forward level is pulled (candidates' in-edges)
+    TBC_OPT_BATCH_PULL = 13, /* batched engine: a forward level is pulled (candidates' in-edges)
                                 when the frontier's out-edges x this value > nnz, else pushed
                                 (default 8; must be >= 0) */
+    TBC_OPT_BATCH_WIDTH = 14 /* batched engine: sources per sweep, 32 (one per warp lane) or 64
+                                (two per lane); default 32.  Workspace ~ 2 x 8 W B/vertex of (sigma,
+                                delta_u) rows plus level lists of <= W entries per vertex. */
 };
 
 /* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since

@@ -25,7 +25,7 @@ __all__ = ["Graph", "TBCError", "lib", "ENGINE_CSC", "ENGINE_COOT", "DIR_AUTO", 
 ENGINE_CSC, ENGINE_COOT = 0, 1
 FLAG_ONE_FORMAT, FLAG_NO_VALIDATE, FLAG_NO_REORDER = 1, 2, 4
 OPT_DIRECTION, OPT_BWD_DIRECTION, OPT_TRACE, OPT_FORMAT, OPT_PARTITIONS = 1, 2, 3, 4, 11
-OPT_BATCH, OPT_BATCH_PULL = 12, 13
+OPT_BATCH, OPT_BATCH_PULL, OPT_BATCH_WIDTH = 12, 13, 14
 OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8, "scan": 9, "bpush": 10}
 FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
 DIR_AUTO, DIR_PUSH, DIR_PULL = 0, 1, 2
@@ -58,8 +58,8 @@ def lib():
     """Load libturbobc.so (building it in-tree first if the sources are newer)."""
     global _LIB
     if _LIB is None:
-        path = _build.build(debug=os.environ.get("TBC_DEBUG_LIB") == "1",
-                            variant=os.environ.get("TBC_VARIANT", ""))
+        path = os.environ.get("TBC_LIB_PATH") or _build.build(debug=os.environ.get("TBC_DEBUG_LIB") == "1",
+                                                              variant=os.environ.get("TBC_VARIANT", ""))
         L = ctypes.CDLL(path)
         i64, i32, P = ctypes.c_int64, ctypes.c_int32, ctypes.POINTER
         vp = ctypes.c_void_p
@@ -167,6 +167,10 @@ class Graph:
     def set_batch(self, on: int):
         """bc engine: 1 batched (32 sources per sweep, default), 0 per source (TBC_OPT_BATCH)."""
         _check(lib().tbc_graph_set_option(self._h, OPT_BATCH, float(on)))
+
+    def set_batch_width(self, width: int):
+        """Batched engine: sources per sweep, 32 or 64 (TBC_OPT_BATCH_WIDTH)."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_BATCH_WIDTH, float(width)))
 
     def set_batch_pull(self, ratio: float):
         """Batched engine: pull a level when frontier out-edges x ratio > nnz (TBC_OPT_BATCH_PULL)."""

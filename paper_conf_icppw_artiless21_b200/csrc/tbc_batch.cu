@@ -47,6 +47,29 @@ constexpr int kBU = TBC_BUNROLL;  // gathers in flight per lane in the slot loop
 
 enum { B_PUSH = 0, B_PULL = 1, B_BWD = 2 };
 
+// lane-mask word of a batch of W sources: lane l of a warp holds sources l and (W = 64) l + 32
+template <int W> struct MaskT { using T = uint32_t; };
+template <> struct MaskT<64> { using T = unsigned long long; };
+
+// TBC_PROF builds: lane 0 of every warp sums clock64 deltas per region into gctr->prof[0..15]:
+// 0 barrier, 1 B phase, 2 push pass, 3 pull pass, 4 backward pass, 5 retire, 6 init/other,
+// 8 + {0 window, 1 index+masks, 2 claims/append, 3 owner loop} inside the edge passes
+enum { BR_BAR = 0, BR_BPHASE = 1, BR_PASS = 2, BR_CLEAR = 5, BR_OTHER = 6, BR_WIN = 8, BR_IDX = 9, BR_APP = 10,
+       BR_OWN = 11, BR_SLOTS = 16 };
+#ifdef TBC_PROF
+__shared__ unsigned long long tbc_bprof[kBWarps][BR_SLOTS];
+#define BPROF_START() unsigned long long _bt = clock64()
+#define BPROF(slot)                                                              \
+    do {                                                                         \
+        const unsigned long long _n = clock64();                                 \
+        if ((threadIdx.x & 31) == 0) tbc_bprof[threadIdx.x >> 5][(slot)] += _n - _bt; \
+        _bt = _n;                                                                \
+    } while (0)
+#else
+#define BPROF_START() ((void)0)
+#define BPROF(slot) ((void)0)
+#endif
+
 struct BParams {
     int64_t n, m;
     const int64_t *__restrict__ in_ptr;
@@ -55,10 +78,11 @@ struct BParams {
     const int32_t *__restrict__ out_idx;
     const int2 *__restrict__ deg2;
     double *sig, *du;
-    uint32_t *vis;
-    uint32_t *fr0, *fr1;
+    void *vis;        // MaskT<W>[n]
+    void *fr0, *fr1;  // MaskT<W>[n]
     int32_t *list_v;
-    uint32_t *list_pre, *list_beg, *list_m;
+    uint32_t *list_pre, *list_beg;
+    void *list_m;     // MaskT<W>[list_cap]
     int32_t *tiles;
     int32_t *cand_v;
     uint32_t *cand_pre, *cand_beg;
@@ -81,7 +105,7 @@ struct __align__(16) BWarpSmem {
     uint32_t beg[kBT + 2];   // adjacency position of the owner's first in-tile edge
     int32_t first[kBT + 2];  // slot of that edge (+ sentinel ne)
     int32_t v[kBT + 2];      // owner vertex
-    uint32_t msk[kBT + 2];   // owner lanes
+    unsigned long long msk[kBT + 2];  // owner lanes
     int32_t fl[kBT + 2];     // bit 0: the tile holds the owner's first item; bit 1: whole owner
     int32_t own[kBT + 2];    // owner (window index) of each slot
     int32_t x[kBT];          // other end of each slot
@@ -109,6 +133,7 @@ __device__ __forceinline__ void btrace(const BParams &P, bool on, int kind, int6
 
 // grid barrier (as tbc_engine.cu): the last arriver snapshots {list, active, cand} counters
 __device__ __forceinline__ void bsync(Ctrs *c, unsigned &gen, unsigned nblocks) {
+    BPROF_START();
     __syncthreads();
     if (threadIdx.x == 0) {
         const unsigned g0 = gen;
@@ -135,6 +160,7 @@ __device__ __forceinline__ void bsync(Ctrs *c, unsigned &gen, unsigned nblocks) 
     }
     gen += 1;
     __syncthreads();
+    BPROF(BR_BAR);
 }
 
 // a list being appended to: relative packed counter (count << ebits) | degree sum, arrays
@@ -224,17 +250,27 @@ __device__ __forceinline__ uint64_t slot_range(int s0, int s1) {
 //   PUSH: frontier owners, out-edges;  PULL: candidates, in-edges;  BWD: level-L owners, out-edges.
 // emsk: per-vertex lane mask of the other end (PULL: M_d, BWD: M_{L+1}; PUSH uses ~vis).
 // fr_out: PUSH/PULL the next level's dense mask, BWD the owners' level (scattered M_L).
-template <int MODE>
+template <int MODE, int W>
 __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int32_t *ov, const uint32_t *opre,
-                                      const uint32_t *obeg, const uint32_t *omsk, const int32_t *otiles, int64_t N,
-                                      int64_t E, const int32_t *__restrict__ adj_idx, const uint32_t *emsk,
-                                      uint32_t *fr_out, uint32_t active, int64_t gwarp, int64_t nwarps, const BOut &out) {
+                                      const uint32_t *obeg, const void *omsk_, const int32_t *otiles, int64_t N,
+                                      int64_t E, const int32_t *__restrict__ adj_idx, const void *emsk_,
+                                      void *fr_out_, unsigned long long active_, int64_t gwarp, int64_t nwarps,
+                                      const BOut &out) {
+    using MT = typename MaskT<W>::T;
+    constexpr int NS = W / 32;                 // sources per lane
+    constexpr int U2 = kBU / NS > 0 ? kBU / NS : 1;  // gathers in flight per lane and source
+    const MT *omsk = static_cast<const MT *>(omsk_);
+    const MT *emsk = static_cast<const MT *>(emsk_);
+    MT *fr_out = static_cast<MT *>(fr_out_);
+    const MT *vis = static_cast<const MT *>(P.vis);
+    const MT active = (MT)active_;
     const int lane = threadIdx.x & 31;
     const int64_t K = N + E;
     const int64_t ntiles = cdiv(K, kBT);
     const uint64_t pol = policy_evict_first();
     double *const sig = P.sig;
     for (int64_t tile = gwarp; tile < ntiles; tile += nwarps) {
+        BPROF_START();
         const int64_t ks = tile * kBT;
         const int64_t ke = min(ks + (int64_t)kBT, K);
         const int64_t ps = otiles[tile];
@@ -254,7 +290,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             const int64_t kf = pre + p;  // the owner's first diagonal item
             const bool isf = kf >= ks && kf < ke;
             const bool whole = isf && p < pe;
-            ws.msk[j] = (MODE == B_PULL) ? (~P.vis[v] & active) : omsk[p];
+            ws.msk[j] = (MODE == B_PULL) ? (MT)(~vis[v] & active) : omsk[p];
             ws.fl[j] = (isf ? 1 : 0) | (whole ? 2 : 0);
         }
         for (int sl = lane; sl < kBT; sl += 32) ws.own[sl] = -1;
@@ -288,9 +324,10 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             }
         }
         __syncwarp();
+        BPROF(BR_WIN);
         // ---- edges, coalesced (slot = i*32 + lane): other end and its lanes
         int xs[kBI];
-        uint32_t ems[kBI];
+        MT ems[kBI];
         uint64_t act = 0;
 #pragma unroll
         for (int i = 0; i < kBI; ++i) {
@@ -306,20 +343,24 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
         for (int i = 0; i < kBI; ++i) {
             const int sl = i * 32 + lane;
             if (sl < ne) {
-                const uint32_t g = (MODE == B_PUSH) ? ~P.vis[xs[i]] : emsk[xs[i]];
-                ems[i] = g & ws.msk[ws.own[sl]];
+                const MT g = (MODE == B_PUSH) ? (MT)~vis[xs[i]] : emsk[xs[i]];
+                ems[i] = g & (MT)ws.msk[ws.own[sl]];
             }
             ws.x[sl] = xs[i];
-            act |= (uint64_t)__ballot_sync(FULL, ems[i] != 0u) << (32 * i);
+            act |= (uint64_t)__ballot_sync(FULL, ems[i] != (MT)0) << (32 * i);
         }
-        // this lane's (source's) slots: the transpose of the slots' lane masks
-        static_assert(kBI == 2, "64 slots per tile: two 32 x 32 transposes");
-        const uint64_t lm = (uint64_t)transpose32(ems[0]) | ((uint64_t)transpose32(ems[1]) << 32);
+        // this lane's slots per source: the transpose of the slots' lane masks
+        static_assert(kBI == 2, "64 slots per tile: two 32 x 32 transposes per source word");
+        uint64_t lm[NS];
+#pragma unroll
+        for (int k = 0; k < NS; ++k)
+            lm[k] = (uint64_t)transpose32((uint32_t)(ems[0] >> (32 * k))) |
+                    ((uint64_t)transpose32((uint32_t)(ems[1] >> (32 * k))) << 32);
 #ifdef TBC_PROF
         {
             unsigned pairs = 0;
 #pragma unroll
-            for (int i = 0; i < kBI; ++i) pairs += __popc(ems[i]);
+            for (int i = 0; i < kBI; ++i) pairs += __popcll((unsigned long long)ems[i]);
             pairs = __reduce_add_sync(FULL, pairs);
             if (lane == 0) {
                 atomicAdd(&P.gctr->prof[24 + 2 * MODE], (unsigned long long)__popcll(act));
@@ -329,6 +370,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             }
         }
 #endif
+        BPROF(BR_IDX);
         if (MODE == B_PUSH) {
             // claims: the atomicOr that lifts fr_out[x] from 0 appends x to the next level
             bool cl[kBI];
@@ -338,12 +380,13 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                 cl[i] = false;
                 cdg[i] = 0;
                 cbg[i] = 0;
-                if (ems[i] != 0u) cl[i] = atomicOr(&fr_out[xs[i]], ems[i]) == 0u;
+                if (ems[i] != (MT)0) cl[i] = atomicOr(&fr_out[xs[i]], ems[i]) == (MT)0;
                 if (cl[i]) span(P.out_ptr, xs[i], cdg[i], cbg[i]);
             }
             bappend(cl, xs, cdg, cbg, out, P.ebits);
         }
         __syncwarp();
+        BPROF(BR_APP);
         int nc = 0;  // PULL: discovered owners of this tile
         for (int j = 0; j < nwin; ++j) {
             uint64_t bits = act & slot_range(ws.first[j], ws.first[j + 1]);
@@ -351,61 +394,96 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             if (MODE != B_BWD && bits == 0) continue;
             if (MODE == B_BWD && bits == 0 && !(fl & 1)) continue;
             const int32_t v = ws.v[j];
-            const uint32_t m = ws.msk[j];
-            const bool in = (m >> lane) & 1u;
-            // each lane walks only its own source's slots of this owner (divergent loop, no
-            // collectives inside): warp iterations = the busiest lane's count, not the slots'
-            uint64_t mine = lm & bits;
-            if (MODE == B_PUSH) {
-                const double su = in ? sig[(int64_t)v * kBatch + lane] : 0.0;
+            const MT m = (MT)ws.msk[j];
+            const int64_t row = (int64_t)v * W + lane;  // + 32 k: the lane's word of source k
+            bool in[NS];
+            uint64_t mine[NS];
 #pragma unroll
-                for (int h = 0; h < kBI; ++h) {
-                    uint32_t mm = (uint32_t)(mine >> (32 * h));
-                    while (mm) {
-                        const int sl = 32 * h + __ffs(mm) - 1;
-                        mm &= mm - 1;
-                        atomicAdd(&sig[(int64_t)ws.x[sl] * kBatch + lane], su);
+            for (int k = 0; k < NS; ++k) {
+                in[k] = (m >> (32 * k + lane)) & 1u;
+                // each lane walks only its own sources' slots of this owner (divergent loop, no
+                // collectives inside): warp iterations = the busiest lane's count, not the slots'
+                mine[k] = lm[k] & bits;
+            }
+            if (MODE == B_PUSH) {
+#pragma unroll
+                for (int k = 0; k < NS; ++k) {
+                    const double su = in[k] ? sig[row + 32 * k] : 0.0;
+#pragma unroll
+                    for (int h = 0; h < kBI; ++h) {
+                        uint32_t mm = (uint32_t)(mine[k] >> (32 * h));
+                        while (mm) {
+                            const int sl = 32 * h + __ffs(mm) - 1;
+                            mm &= mm - 1;
+                            atomicAdd(&sig[(int64_t)ws.x[sl] * W + 32 * k + lane], su);
+                        }
                     }
                 }
                 continue;
             }
             const double *src = (MODE == B_PULL) ? sig : P.du;
-            const double sv = (MODE == B_BWD && in) ? sig[(int64_t)v * kBatch + lane] : 1.0;
-            double acc = 0.0;
-            // the two 32-slot halves of the tile, kBU gathers in flight per lane; __ffs(0) = 0
-            // marks the exhausted positions
+            double sv[NS], acc[NS];
+#pragma unroll
+            for (int k = 0; k < NS; ++k) {
+                sv[k] = (MODE == B_BWD && in[k]) ? sig[row + 32 * k] : 1.0;
+                acc[k] = 0.0;
+            }
+            // the two 32-slot halves of the tile, U2 gathers in flight per lane and source;
+            // __ffs(0) = 0 marks the exhausted positions
 #pragma unroll
             for (int h = 0; h < kBI; ++h) {
-                uint32_t mm = (uint32_t)(mine >> (32 * h));
+                uint32_t mm[NS];
+                uint32_t any = 0;
+#pragma unroll
+                for (int k = 0; k < NS; ++k) {
+                    mm[k] = (uint32_t)(mine[k] >> (32 * h));
+                    any |= mm[k];
+                }
                 const int32_t *xh = ws.x + 32 * h;
-                while (mm) {
-                    int sl[kBU];
+                while (any) {
+                    int sl[NS][U2];
+                    double a[NS][U2];
+                    any = 0;
 #pragma unroll
-                    for (int q = 0; q < kBU; ++q) {
-                        sl[q] = __ffs(mm) - 1;
-                        mm &= mm - 1;
+                    for (int k = 0; k < NS; ++k) {
+#pragma unroll
+                        for (int q = 0; q < U2; ++q) {
+                            sl[k][q] = __ffs(mm[k]) - 1;
+                            mm[k] &= mm[k] - 1;
+                        }
+                        any |= mm[k];
                     }
-                    double a[kBU];
 #pragma unroll
-                    for (int q = 0; q < kBU; ++q) a[q] = sl[q] >= 0 ? src[(int64_t)xh[sl[q]] * kBatch + lane] : 0.0;
+                    for (int k = 0; k < NS; ++k)
 #pragma unroll
-                    for (int q = 0; q < kBU; ++q) acc += a[q];
+                        for (int q = 0; q < U2; ++q)
+                            a[k][q] = sl[k][q] >= 0 ? src[(int64_t)xh[sl[k][q]] * W + 32 * k + lane] : 0.0;
+#pragma unroll
+                    for (int k = 0; k < NS; ++k)
+#pragma unroll
+                        for (int q = 0; q < U2; ++q) acc[k] += a[k][q];
                 }
             }
             if (MODE == B_PULL) {
                 // Alg.1 l.20-25: lanes with a non-zero masked sum are discovered on this level
-                const unsigned newm = __ballot_sync(FULL, acc > 0.0);
-                if (newm == 0u) continue;
+                MT newm = 0;
+#pragma unroll
+                for (int k = 0; k < NS; ++k) newm |= (MT)__ballot_sync(FULL, acc[k] > 0.0) << (32 * k);
+                if (newm == (MT)0) continue;
                 bool claimed;
                 if (fl & 2) {
-                    if (acc > 0.0) sig[(int64_t)v * kBatch + lane] = acc;
+#pragma unroll
+                    for (int k = 0; k < NS; ++k)
+                        if (acc[k] > 0.0) sig[row + 32 * k] = acc[k];
                     if (lane == 0) fr_out[v] = newm;
                     claimed = true;
                 } else {
-                    if (acc > 0.0) atomicAdd(&sig[(int64_t)v * kBatch + lane], acc);
-                    unsigned old = 0;
+#pragma unroll
+                    for (int k = 0; k < NS; ++k)
+                        if (acc[k] > 0.0) atomicAdd(&sig[row + 32 * k], acc[k]);
+                    MT old = 0;
                     if (lane == 0) old = atomicOr(&fr_out[v], newm);
-                    claimed = __shfl_sync(FULL, old, 0) == 0u;
+                    claimed = __shfl_sync(FULL, old, 0) == (MT)0;
                 }
                 if (claimed) {
                     if (lane == 0) ws.claim[nc] = v;
@@ -413,14 +491,19 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                 }
             } else {
                 // Alg.1 l.38-39, l.45 (x 1/2 undirected) and l.35
-                double c = in ? sv * acc : 0.0;
+                double c = 0.0;
 #pragma unroll
-                for (int k = 16; k >= 1; k >>= 1) c += __shfl_xor_sync(FULL, c, k);
-                if (fl & 2) {
-                    if (in) P.du[(int64_t)v * kBatch + lane] = 1.0 / sv + acc;
-                } else {
-                    const double t = acc + ((fl & 1) ? 1.0 / sv : 0.0);
-                    if (in && t != 0.0) atomicAdd(&P.du[(int64_t)v * kBatch + lane], t);
+                for (int k = 0; k < NS; ++k) c += in[k] ? sv[k] * acc[k] : 0.0;
+#pragma unroll
+                for (int o = 16; o >= 1; o >>= 1) c += __shfl_xor_sync(FULL, c, o);
+#pragma unroll
+                for (int k = 0; k < NS; ++k) {
+                    if (fl & 2) {
+                        if (in[k]) P.du[row + 32 * k] = 1.0 / sv[k] + acc[k];
+                    } else {
+                        const double t = acc[k] + ((fl & 1) ? 1.0 / sv[k] : 0.0);
+                        if (in[k] && t != 0.0) atomicAdd(&P.du[row + 32 * k], t);
+                    }
                 }
                 if (lane == 0) {
                     if (c != 0.0) atomicAdd(&P.bc[P.inv ? P.inv[v] : v], c * P.bc_scale);
@@ -445,36 +528,49 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             bappend(cl, cv, cdg, cbg, out, P.ebits);
         }
         __syncwarp();
+        BPROF(BR_OWN);
     }
 }
 
-// zero the (vertex, lane) state of a level list's entries: sigma, delta_u, visited lanes and
+// zero the (vertex, source) state of a level list's entries: sigma, delta_u, visited lanes and
 // the dense mask of its parity (atomicAnd: a concurrent scatter of another level may share the word)
-__device__ __forceinline__ void bclear(const BParams &P, const Lv &l, uint32_t *fr, int64_t gwarp, int64_t nwarps) {
+template <int W>
+__device__ __forceinline__ void bclear(const BParams &P, const Lv &l, void *fr_, int64_t gwarp, int64_t nwarps) {
+    using MT = typename MaskT<W>::T;
+    constexpr int NS = W / 32;
+    MT *fr = static_cast<MT *>(fr_);
+    MT *vis = static_cast<MT *>(P.vis);
+    const MT *lm = static_cast<const MT *>(P.list_m);
     const int lane = threadIdx.x & 31;
     for (int64_t base = gwarp * 32; base < l.N; base += nwarps * 32) {
         const int64_t p = base + lane;
         int32_t v = -1;
-        uint32_t m = 0;
+        MT m = 0;
         if (p < l.N) {
             v = P.list_v[l.p0 + p];
-            m = P.list_m[l.p0 + p];
+            m = lm[l.p0 + p];
             atomicAnd(&fr[v], ~m);
-            P.vis[v] = 0u;
+            vis[v] = 0;
         }
         const int cnt = (int)min((int64_t)32, l.N - base);
         for (int q = 0; q < cnt; ++q) {
             const int32_t vq = __shfl_sync(FULL, v, q);
-            const uint32_t mq = __shfl_sync(FULL, m, q);
-            if ((mq >> lane) & 1u) {
-                P.sig[(int64_t)vq * kBatch + lane] = 0.0;
-                P.du[(int64_t)vq * kBatch + lane] = 0.0;
+            const MT mq = __shfl_sync(FULL, m, q);
+#pragma unroll
+            for (int k = 0; k < NS; ++k) {
+                if ((mq >> (32 * k + lane)) & 1u) {
+                    P.sig[(int64_t)vq * W + 32 * k + lane] = 0.0;
+                    P.du[(int64_t)vq * W + 32 * k + lane] = 0.0;
+                }
             }
         }
     }
 }
 
+template <int W>
 __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams P) {
+    using MT = typename MaskT<W>::T;
+    constexpr int NS = W / 32;
     extern __shared__ __align__(16) unsigned char bsm[];
     BWarpSmem &ws = reinterpret_cast<BWarpSmem *>(bsm)[threadIdx.x >> 5];
     const int tid = threadIdx.x, lane = tid & 31;
@@ -487,52 +583,74 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
     Ctrs *C = P.ctr;
     unsigned gen = (tid == 0) ? ld_acquire(&C->bar_gen) : 0u;
     const unsigned long long emask = (1ull << P.ebits) - 1ull;
-    uint32_t *fr[2] = {P.fr0, P.fr1};
-    const int64_t nb = (P.k + kBatch - 1) / kBatch;
+    MT *fr[2] = {static_cast<MT *>(P.fr0), static_cast<MT *>(P.fr1)};
+    MT *vis = static_cast<MT *>(P.vis);
+    MT *list_m = static_cast<MT *>(P.list_m);
+    const int64_t nb = (P.k + W - 1) / W;
 
+#ifdef TBC_PROF
+    for (int i = tid; i < kBWarps * BR_SLOTS; i += kBB) (&tbc_bprof[0][0])[i] = 0;
+    __syncthreads();
+    const unsigned long long t_kernel0 = clock64();
+#endif
     for (int64_t b = 0; b < nb; ++b) {
-        // ---------------- level 0: the batch's sources (Alg.1 l.15-18), lane s <- sources[32b+s]
+        // ---------------- level 0: the batch's sources (Alg.1 l.15-18): source b*W + 32k + l is
+        // lane l's source k; a vertex repeated in the batch is appended once, by its lowest source
         if (cta0 && tid < 32) {
-            const int64_t si = b * kBatch + lane;
-            int32_t s = -1;
-            if (si < P.k) {
-                const int32_t sc = P.sources[si];
-                if (sc >= 0 && sc < P.n) s = P.perm ? P.perm[sc] : sc;
-                else atomicAdd(&C->bad_sources, 1ull);
+            int32_t s[NS];
+            unsigned valid = 0;
+#pragma unroll
+            for (int k = 0; k < NS; ++k) {
+                const int64_t si = b * W + 32 * k + lane;
+                s[k] = -1;
+                if (si < P.k) {
+                    const int32_t sc = P.sources[si];
+                    if (sc >= 0 && sc < P.n) s[k] = P.perm ? P.perm[sc] : sc;
+                    else atomicAdd(&C->bad_sources, 1ull);
+                }
+                if (s[k] >= 0) {
+                    atomicOr(&fr[0][s[k]], (MT)1 << (32 * k + lane));
+                    P.sig[(int64_t)s[k] * W + 32 * k + lane] = 1.0;
+                }
+                valid += __popc(__ballot_sync(FULL, s[k] >= 0));
             }
-            if (s >= 0) {
-                atomicOr(&P.fr0[s], 1u << lane);
-                P.sig[(int64_t)s * kBatch + lane] = 1.0;
+            int pos0 = 0;
+            uint32_t e0 = 0;
+#pragma unroll
+            for (int k = 0; k < NS; ++k) {
+                bool take = s[k] >= 0;
+                for (int l = 0; l < 32; ++l) {
+#pragma unroll
+                    for (int k2 = 0; k2 <= k; ++k2) {
+                        const int32_t t = __shfl_sync(FULL, s[k2], l);
+                        if ((k2 < k || l < lane) && t == s[k]) take = false;
+                    }
+                }
+                uint32_t dg = 0, bg = 0;
+                if (take) span(P.out_ptr, s[k], dg, bg);
+                const unsigned tm = __ballot_sync(FULL, take);
+                uint32_t inc = take ? dg : 0u;
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t t = __shfl_up_sync(FULL, inc, o);
+                    if (lane >= o) inc += t;
+                }
+                if (take) {
+                    const int pos = pos0 + __popc(tm & ((1u << lane) - 1u));
+                    const uint32_t ee = e0 + inc - dg;
+                    P.list_v[pos] = s[k];
+                    P.list_pre[pos] = ee;
+                    P.list_beg[pos] = bg;
+                    const int64_t k0 = (int64_t)ee + pos, k1 = k0 + dg;
+                    for (int64_t t = (k0 + kBT - 1) / kBT; t <= k1 / kBT; ++t) P.tiles[t] = pos;
+                }
+                pos0 += __popc(tm);
+                e0 += __shfl_sync(FULL, inc, 31);
             }
-            bool take = s >= 0;
-            for (int l = 0; l < 32; ++l) {  // repeated vertices: the lowest lane appends
-                const int32_t t = __shfl_sync(FULL, s, l);
-                if (l < lane && t == s) take = false;
-            }
-            uint32_t dg = 0, bg = 0;
-            if (take) span(P.out_ptr, s, dg, bg);
-            const unsigned tm = __ballot_sync(FULL, take);
-            uint32_t inc = take ? dg : 0u;
-            for (int k = 1; k < 32; k <<= 1) {
-                const uint32_t t = __shfl_up_sync(FULL, inc, k);
-                if (lane >= k) inc += t;
-            }
-            const uint32_t tot = __shfl_sync(FULL, inc, 31);
-            if (take) {
-                const int pos = __popc(tm & ((1u << lane) - 1u));
-                const uint32_t e0 = inc - dg;
-                P.list_v[pos] = s;
-                P.list_pre[pos] = e0;
-                P.list_beg[pos] = bg;
-                const int64_t k0 = (int64_t)e0 + pos, k1 = k0 + dg;
-                for (int64_t t = (k0 + kBT - 1) / kBT; t <= k1 / kBT; ++t) P.tiles[t] = pos;
-            }
-            const unsigned valid = __ballot_sync(FULL, s >= 0);
             if (lane == 0) {
-                C->list = ((unsigned long long)__popc(tm) << P.ebits) | tot;
+                C->list = ((unsigned long long)pos0 << P.ebits) | e0;
                 C->ilist = 0;
                 C->cand[0] = 0;
-                C->st_sources += __popc(valid);
+                C->st_sources += valid;
             }
         }
         const bool tr = b == P.trace_b;
@@ -547,38 +665,40 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
         }
         Lv prev{0, 0, 0, 0};
         int d = 0;
-        uint32_t active = 0xffffffffu;
+        MT active = ~(MT)0;
         int64_t fwd_edges = 0, pulls = 0;
         for (;;) {
             // direction of level d+1 (uniform: every CTA computes it from the same snapshot)
             const bool pull = d + 1 >= 2 && P.dir_mode != 1 &&
                               (P.dir_mode == 2 || (double)cur.E * P.pull_ratio > (double)P.m);
             // ---- B(d): lanes of level d -> list masks and visited; retire M_{d-1}; candidates
+            BPROF_START();
             if (cta0 && tid == 0) C->list = 0;  // relative counter of level d+1 (snapshot already taken)
             {
-                uint32_t orr = 0;
+                unsigned long long orr = 0;
                 long long rc = 0, re = 0;
-                uint32_t *frd = fr[d & 1];
+                MT *frd = fr[d & 1];
                 for (int64_t p = gtid; p < cur.N; p += nthreads) {
                     const int32_t v = P.list_v[cur.p0 + p];
-                    const uint32_t m = frd[v];
-                    P.list_m[cur.p0 + p] = m;
-                    P.vis[v] |= m;
-                    orr |= m;
-                    rc += __popc(m);
-                    re += (long long)__popc(m) * P.deg2[v].x;
+                    const MT m = frd[v];
+                    list_m[cur.p0 + p] = m;
+                    vis[v] |= m;
+                    orr |= (unsigned long long)m;
+                    rc += __popcll((unsigned long long)m);
+                    re += (long long)__popcll((unsigned long long)m) * P.deg2[v].x;
                 }
-                orr = __reduce_or_sync(FULL, orr);
+                orr = (unsigned long long)__reduce_or_sync(FULL, (unsigned)orr) |
+                      ((unsigned long long)__reduce_or_sync(FULL, (unsigned)(orr >> 32)) << 32);
                 rc = __reduce_add_sync(FULL, (unsigned)rc);
                 for (int k = 16; k >= 1; k >>= 1) re += __shfl_xor_sync(FULL, re, k);
                 if (lane == 0) {
-                    if (orr) atomicOr((unsigned long long *)&C->ilist, (unsigned long long)orr);
+                    if (orr) atomicOr((unsigned long long *)&C->ilist, orr);
                     if (rc) atomicAdd((unsigned long long *)&C->st_reached, (unsigned long long)rc);
                     if (re) atomicAdd((unsigned long long *)&C->st_reached_edges, (unsigned long long)re);
                 }
                 if (d >= 1) {
-                    uint32_t *frp = fr[(d + 1) & 1];
-                    for (int64_t p = gtid; p < prev.N; p += nthreads) frp[P.list_v[prev.p0 + p]] = 0u;
+                    MT *frp = fr[(d + 1) & 1];
+                    for (int64_t p = gtid; p < prev.N; p += nthreads) frp[P.list_v[prev.p0 + p]] = 0;
                 }
                 if (pull) {  // candidates: vertices with in-edges and an unvisited active lane
                     const BOut co{&C->cand[0], P.cand_v, P.cand_pre, P.cand_beg, P.cand_tiles, P.n + kPad,
@@ -591,7 +711,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
                         for (int i = 0; i < kBI; ++i) {
                             const int64_t w = base + i * 32 + lane;
                             vv[i] = (int32_t)w;
-                            tk[i] = w < P.n_scan && (~P.vis[w] & active) != 0u;
+                            tk[i] = w < P.n_scan && (~vis[w] & active) != (MT)0;
                             dg[i] = 0;
                             bg[i] = 0;
                             if (tk[i]) {
@@ -603,9 +723,10 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
                     }
                 }
             }
+            BPROF(BR_BPHASE);
             bsync(C, gen, ncta);
             btrace(P, tr, 1, d, cur.N, cur.E, pull, 0);
-            active = (uint32_t)ld_volatile_u64(&C->snap[1]);
+            active = (MT)ld_volatile_u64(&C->snap[1]);
             const unsigned long long cs = ld_volatile_u64(&C->snap[2]);
             // ---- A(d+1)
             if (cta0 && tid == 0) {
@@ -615,15 +736,15 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
             Lv nxt{cur.p0 + cur.N, 0, 0, cur.tb + cdiv(cur.N + cur.E, kBT)};
             const BOut lo{&C->list, P.list_v + nxt.p0, P.list_pre + nxt.p0, P.list_beg + nxt.p0, P.tiles + nxt.tb,
                           P.list_cap - nxt.p0, P.tiles_cap - nxt.tb};
-            uint32_t *fro = fr[(d + 1) & 1];
+            MT *fro = fr[(d + 1) & 1];
             if (pull) {
                 const int64_t cN = (int64_t)(cs >> P.ebits), cE = (int64_t)(cs & emask);
-                bpass<B_PULL>(P, ws, P.cand_v, P.cand_pre, P.cand_beg, nullptr, P.cand_tiles, cN, cE, P.in_idx,
-                              fr[d & 1], fro, active, gwarp, nwarps, lo);
+                bpass<B_PULL, W>(P, ws, P.cand_v, P.cand_pre, P.cand_beg, nullptr, P.cand_tiles, cN, cE, P.in_idx,
+                              fr[d & 1], fro, (unsigned long long)active, gwarp, nwarps, lo);
                 fwd_edges += cE;
                 ++pulls;
             } else {
-                bpass<B_PUSH>(P, ws, P.list_v + cur.p0, P.list_pre + cur.p0, P.list_beg + cur.p0, P.list_m + cur.p0,
+                bpass<B_PUSH, W>(P, ws, P.list_v + cur.p0, P.list_pre + cur.p0, P.list_beg + cur.p0, list_m + cur.p0,
                               P.tiles + cur.tb, cur.N, cur.E, P.out_idx, nullptr, fro, 0u, gwarp, nwarps, lo);
                 fwd_edges += cur.E;
             }
@@ -658,12 +779,14 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
             const int64_t *l = P.lvl + 4 * (int64_t)L;
             const Lv lv{l[0], l[1], l[2], l[3]};
             const BOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0};
-            bpass<B_BWD>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.list_beg + lv.p0, P.list_m + lv.p0,
+            bpass<B_BWD, W>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.list_beg + lv.p0, list_m + lv.p0,
                          P.tiles + lv.tb, lv.N, lv.E, P.out_idx, fr[(L + 1) & 1], fr[L & 1], 0u, gwarp, nwarps, none);
             bwd_edges += lv.E;
             if (L + 2 <= D) {
+                BPROF_START();
                 const int64_t *l2 = P.lvl + 4 * (int64_t)(L + 2);
-                bclear(P, Lv{l2[0], l2[1], l2[2], l2[3]}, fr[L & 1], gwarp, nwarps);
+                bclear<W>(P, Lv{l2[0], l2[1], l2[2], l2[3]}, fr[L & 1], gwarp, nwarps);
+                BPROF(BR_CLEAR);
             }
             bsync(C, gen, ncta);
             btrace(P, tr, 4, L, lv.N, lv.E, 0, 0);
@@ -671,7 +794,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
         // retire levels 0..min(2, D)
         for (int L = 0; L <= min(2, D); ++L) {
             const int64_t *l = P.lvl + 4 * (int64_t)L;
-            bclear(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps);
+            bclear<W>(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps);
         }
         if (cta0 && tid == 0) {
             C->st_bwd_edges += bwd_edges;
@@ -680,46 +803,62 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
         bsync(C, gen, ncta);
         btrace(P, tr, 5, 0, 0, 0, 0, 0);
     }
+#ifdef TBC_PROF
+    if ((tid & 31) == 0) {
+        unsigned long long busy = 0;
+        for (int r = 0; r < BR_OTHER; ++r) busy += tbc_bprof[tid >> 5][r];
+        for (int r = BR_WIN; r <= BR_OWN; ++r) busy += tbc_bprof[tid >> 5][r];
+        tbc_bprof[tid >> 5][BR_OTHER] = clock64() - t_kernel0 - busy;
+        for (int r = 0; r < BR_SLOTS; ++r) atomicAdd(&P.gctr->prof[r], tbc_bprof[tid >> 5][r]);
+    }
+#endif
 }
 
 }  // namespace
 
 // ------------------------------------------------------------------ host side
 
-static tbc_status batch_alloc(tbc_graph *g) {
+static tbc_status batch_alloc(tbc_graph *g, int W) {
     BatchWorkspace &w = g->bws;
-    if (w.ready) return TBC_OK;
+    if (w.ready && w.width == W) return TBC_OK;
+    if (w.ready) batch_free(g);  // other width: reallocate
     const int64_t n = g->n, m = g->m;
+    const int64_t nw = W / 32;  // 32-bit words per mask
     cudaStream_t s = g->stream;
     cudaError_t e = cudaSuccess;
     auto alloc = [&](auto **p, size_t cnt) -> cudaError_t {
         size_t bytes = sizeof(**p) * (cnt > 0 ? cnt : 1);
         cudaError_t r = cudaMalloc((void **)p, bytes);
-        if (r == cudaSuccess) g->device_bytes += bytes;
+        if (r == cudaSuccess) w.bytes += bytes;
         return r;
     };
-    // every (vertex, level) pair of a batch has at least one lane: <= 32 n list entries, and the
-    // levels' tiles sum to <= (32 n + 32 m) / kBT + (levels <= n + 1)
-    w.list_cap = (int64_t)kBatch * n + kPad;
-    w.tiles_cap = ((int64_t)kBatch * (n + m)) / kBT + n + 2 + kPad;
+    // every (vertex, level) pair of a batch has at least one source: <= W n list entries, and the
+    // levels' tiles sum to <= (W n + W m) / kBT + (levels <= n + 1)
+    w.width = W;
+    w.list_cap = (int64_t)W * n + kPad;
+    w.tiles_cap = ((int64_t)W * (n + m)) / kBT + n + 2 + kPad;
     w.cand_tiles_cap = (n + m) / kBT + 2 + kPad;
-    if ((e = alloc(&w.sig, (size_t)n * kBatch)) || (e = alloc(&w.du, (size_t)n * kBatch)) || (e = alloc(&w.vis, n)) ||
-        (e = alloc(&w.fr[0], n)) || (e = alloc(&w.fr[1], n)) || (e = alloc(&w.list_v, w.list_cap)) ||
+    if ((e = alloc(&w.sig, (size_t)n * W)) || (e = alloc(&w.du, (size_t)n * W)) || (e = alloc(&w.vis, n * nw)) ||
+        (e = alloc(&w.fr[0], n * nw)) || (e = alloc(&w.fr[1], n * nw)) || (e = alloc(&w.list_v, w.list_cap)) ||
         (e = alloc(&w.list_pre, w.list_cap)) || (e = alloc(&w.list_beg, w.list_cap)) ||
-        (e = alloc(&w.list_m, w.list_cap)) || (e = alloc(&w.tiles, w.tiles_cap)) ||
+        (e = alloc(&w.list_m, w.list_cap * nw)) || (e = alloc(&w.tiles, w.tiles_cap)) ||
         (e = alloc(&w.cand_v, n + kPad)) || (e = alloc(&w.cand_pre, n + kPad)) || (e = alloc(&w.cand_beg, n + kPad)) ||
-        (e = alloc(&w.cand_tiles, w.cand_tiles_cap)) || (e = alloc(&w.lvl, 4 * (n + 2))) || (e = alloc(&w.ctr, 1)))
+        (e = alloc(&w.cand_tiles, w.cand_tiles_cap)) || (e = alloc(&w.lvl, 4 * (n + 2))) || (e = alloc(&w.ctr, 1))) {
+        g->device_bytes += w.bytes;
         return cuda_error(e, "batch workspace cudaMalloc");
-    if ((e = cudaMemsetAsync(w.sig, 0, sizeof(double) * n * kBatch, s)) ||
-        (e = cudaMemsetAsync(w.du, 0, sizeof(double) * n * kBatch, s)) ||
-        (e = cudaMemsetAsync(w.vis, 0, sizeof(uint32_t) * n, s)) ||
-        (e = cudaMemsetAsync(w.fr[0], 0, sizeof(uint32_t) * n, s)) ||
-        (e = cudaMemsetAsync(w.fr[1], 0, sizeof(uint32_t) * n, s)) ||
+    }
+    g->device_bytes += w.bytes;
+    if ((e = cudaMemsetAsync(w.sig, 0, sizeof(double) * n * W, s)) ||
+        (e = cudaMemsetAsync(w.du, 0, sizeof(double) * n * W, s)) ||
+        (e = cudaMemsetAsync(w.vis, 0, sizeof(uint32_t) * n * nw, s)) ||
+        (e = cudaMemsetAsync(w.fr[0], 0, sizeof(uint32_t) * n * nw, s)) ||
+        (e = cudaMemsetAsync(w.fr[1], 0, sizeof(uint32_t) * n * nw, s)) ||
         (e = cudaMemsetAsync(w.ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s)))
         return cuda_error(e, "batch workspace init");
+    const void *fn = W == 64 ? (const void *)k_bcb<64> : (const void *)k_bcb<32>;
     int per_sm = 0, sms = 0;
-    if ((e = cudaFuncSetAttribute(k_bcb, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmem)) ||
-        (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_bcb, kBB, kBSmem)) ||
+    if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmem)) ||
+        (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kBB, kBSmem)) ||
         (e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device)))
         return cuda_error(e, "batch occupancy query");
     if (per_sm < 1) return set_error(TBC_ERR_CUDA, "k_bcb cannot be resident (occupancy 0)");
@@ -733,11 +872,13 @@ void batch_free(tbc_graph *g) {
     void *ps[] = {w.sig, w.du, w.vis, w.fr[0], w.fr[1], w.list_v, w.list_pre, w.list_beg, w.list_m, w.tiles,
                   w.cand_v, w.cand_pre, w.cand_beg, w.cand_tiles, w.lvl, w.ctr};
     for (void *p : ps) cudaFree(p);
+    g->device_bytes -= w.bytes;
     w = BatchWorkspace{};
 }
 
 tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream) {
-    tbc_status st = batch_alloc(g);
+    const int W = g->batch_width;
+    tbc_status st = batch_alloc(g, W);
     if (st != TBC_OK) return st;
     const BatchWorkspace &w = g->bws;
     BParams P{};
@@ -780,10 +921,10 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
     P.dir_mode = g->dir_mode;
     P.trace = g->trace;
     P.trace_cap = g->trace ? kTraceCap : 0;
-    P.trace_b = g->trace_src >= 0 ? g->trace_src / kBatch : -1;
+    P.trace_b = g->trace_src >= 0 ? g->trace_src / W : -1;
     void *args[] = {&P};
-    cudaError_t e =
-        cudaLaunchCooperativeKernel((const void *)k_bcb, dim3(g->bgrid), dim3(kBB), args, kBSmem, stream);
+    const void *fn = W == 64 ? (const void *)k_bcb<64> : (const void *)k_bcb<32>;
+    cudaError_t e = cudaLaunchCooperativeKernel(fn, dim3(g->bgrid), dim3(kBB), args, kBSmem, stream);
     if (e != cudaSuccess) return cuda_error(e, "cudaLaunchCooperativeKernel(k_bcb)");
     return TBC_OK;
 }

@@ -116,17 +116,19 @@ struct Workspace {
 };
 constexpr int kMaxPartitions = 8;
 
-// workspace of the batched engine (tbc_batch.cu): 32 sources per sweep, one per warp lane
-constexpr int kBatch = 32;
+// workspace of the batched engine (tbc_batch.cu): W = 32 or 64 sources per sweep, lane l of a
+// warp holding sources l (and l + 32); masks are W-bit words (W / 32 uint32 words)
 struct BatchWorkspace {
-    double *sig = nullptr;       // [n][32] sigma of (vertex, lane)
-    double *du = nullptr;        // [n][32] delta_u of (vertex, lane) (backward)
-    uint32_t *vis = nullptr;     // [n] lanes that have reached the vertex
-    uint32_t *fr[2] = {nullptr, nullptr};  // [n] dense level masks, by level parity
+    int width = 0;               // W the workspace was sized for
+    size_t bytes = 0;
+    double *sig = nullptr;       // [n][W] sigma of (vertex, source)
+    double *du = nullptr;        // [n][W] delta_u of (vertex, source) (backward)
+    uint32_t *vis = nullptr;     // [n] sources that have reached the vertex (W-bit words)
+    uint32_t *fr[2] = {nullptr, nullptr};  // [n] dense level masks, by level parity (W-bit words)
     int32_t *list_v = nullptr;   // level lists (levels concatenated), capacity list_cap
     uint32_t *list_pre = nullptr;  // out-degree prefix, relative to the level
     uint32_t *list_beg = nullptr;  // out_ptr of the entry
-    uint32_t *list_m = nullptr;    // lanes on this level
+    uint32_t *list_m = nullptr;    // sources on this level (W-bit words)
     int32_t *tiles = nullptr;      // per level: owner starting each warp tile, capacity tiles_cap
     int32_t *cand_v = nullptr;     // pull candidates (in-degree prefix)
     uint32_t *cand_pre = nullptr;
@@ -171,7 +173,8 @@ struct tbc_graph {
     int bwd_mode = 0;
     int fmt_mode = 0;
     double c_list = 12.0, c_stream = 4.0, c_atom = 18.0, c_vert = 10.0, c_scan = 3.0, c_bpush = 6.0;
-    int batch = 1;                // TBC_OPT_BATCH: 1 batched engine (32 sources per sweep), 0 per source
+    int batch = 1;                // TBC_OPT_BATCH: 1 batched engine, 0 per source
+    int batch_width = 32;         // TBC_OPT_BATCH_WIDTH: sources per sweep (32 or 64)
     double batch_pull = 8.0;      // TBC_OPT_BATCH_PULL: pull when frontier out-edges x this > m
     tbc::BatchWorkspace bws;
     int bgrid = 0;

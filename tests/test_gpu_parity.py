@@ -16,8 +16,10 @@ pytestmark = pytest.mark.gpu
 # (forward direction, format, backward direction) triples: every forward/backward pass kind
 # gets exercised -- (PULL, LIST) forces the candidate scan + list pull after the first push
 # level; backward 1 = pull over level L's out-edges only, 2 = push from level L+1 (in-edges)
-# the 4th element selects the engine: 1 batched (32 sources per sweep, the default), 0 per source
+# the 4th element selects the engine: 1 batched (the default), 0 per source; the 5th the batch
+# width (sources per sweep, 32 default, or 64)
 MODES = [(tbc.DIR_AUTO, tbc.FMT_AUTO, 0, 1), (tbc.DIR_PUSH, tbc.FMT_AUTO, 0, 1), (tbc.DIR_PULL, tbc.FMT_AUTO, 0, 1),
+         (tbc.DIR_AUTO, tbc.FMT_AUTO, 0, 1, 64), (tbc.DIR_PULL, tbc.FMT_AUTO, 0, 1, 64),
          (tbc.DIR_AUTO, tbc.FMT_AUTO, 0, 0), (tbc.DIR_PUSH, tbc.FMT_LIST, 1, 0), (tbc.DIR_PUSH, tbc.FMT_STREAM, 0, 0),
          (tbc.DIR_PULL, tbc.FMT_AUTO, 0, 0), (tbc.DIR_PULL, tbc.FMT_STREAM, 0, 0), (tbc.DIR_PULL, tbc.FMT_LIST, 2, 0),
          (tbc.DIR_AUTO, tbc.FMT_LIST, 2, 0)]
@@ -28,6 +30,7 @@ def set_mode(G, mode):
     G.set_format(mode[1])
     G.set_bwd_direction(mode[2] if len(mode) > 2 else 0)
     G.set_batch(mode[3] if len(mode) > 3 else 1)
+    G.set_batch_width(mode[4] if len(mode) > 4 else 32)
 
 
 def assert_bc(got, want, rel=1e-9):
@@ -64,7 +67,7 @@ SMALL = [gg.star(7), gg.star(7, directed_both=True), gg.path(7), gg.path(7, dire
 
 
 @pytest.mark.parametrize("engine", ENGINES)
-@pytest.mark.parametrize("mode", MODES, ids=lambda m: f"dir{m[0]}fmt{m[1]}bwd{m[2]}b{m[3]}")
+@pytest.mark.parametrize("mode", MODES, ids=lambda m: f"dir{m[0]}fmt{m[1]}bwd{m[2]}b{m[3]}w{m[4] if len(m) > 4 else 32}")
 @pytest.mark.parametrize("g", SMALL, ids=lambda g: g.name)
 def test_small_graphs_all_sources(g, mode, engine):
     with gpu_graph(g, engine=engine, reorder=(mode[1] != tbc.FMT_LIST)) as G:
@@ -118,18 +121,20 @@ def test_sm_partitions(directed):
             G.set_partitions(9)
 
 
+@pytest.mark.parametrize("width", [32, 64])
 @pytest.mark.parametrize("directed", [False, True])
 @pytest.mark.parametrize("pull", [0.0, 8.0, 1e9])
-def test_batched_engine(directed, pull):
+def test_batched_engine(directed, pull, width):
     """Batched engine: several sweeps (full and ragged last batch of 32), repeated sources inside a
     batch and across batches, push-only / auto / pull-from-level-2 forward levels; repeat runs agree
     to rounding (fp64 atomics of split owners)."""
     g = gg.kronecker(13, 16, seed=4, directed=directed, device="cuda")
-    src = gg.sources(g, 77, seed=3)
-    src = np.concatenate([src, src[:5], src[10:12], src[10:12]]).astype(np.int32)
+    src = gg.sources(g, 150, seed=3)
+    src = np.concatenate([src, src[:5], src[10:12], src[10:12], src[40:41], src[100:101]]).astype(np.int32)
     want = oracle.bc(g.col_ptr, g.row_idx, directed, src)
     with gpu_graph(g) as G:
         G.set_batch(1)
+        G.set_batch_width(width)
         G.set_batch_pull(pull)
         a = G.bc(src)
         assert_bc(a, want)

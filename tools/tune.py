@@ -36,6 +36,7 @@ for setting in a.settings.split(";"):
     G.set_bwd_direction(int(kv.get("bwd", 0)))
     G.set_partitions(int(kv.get("parts", 8)))
     G.set_batch(int(kv.get("batch", 1)))
+    G.set_batch_width(int(kv.get("width", 32)))
     G.set_batch_pull(float(kv.get("bpull", 8)))
     G.set_cost(**{k: float(v) for k, v in kv.items() if k in ("list", "stream", "atomic", "vertex", "scan", "bpush")})
     G.bc_device(s_d, bc, st)  # warm-up
@@ -61,6 +62,11 @@ for setting in a.settings.split(";"):
     if prof:
         pr = G.profile()
         tot = sum(pr.values()) or 1
+        if int(kv.get("batch", 1)):
+            names = ["barrier", "bphase", "r2", "r3", "r4", "retire", "other", "r7",
+                     "tile_window", "tile_index", "tile_append", "tile_owners"]
+            pr = {**{n: v for n, v in zip(names, pr.values()) if not n.startswith("r")},
+                  **{k: v for k, v in pr.items() if k.startswith("b_")}}
         reg = {k: v for k, v in pr.items() if not k.startswith("b_")}
         tot = sum(reg.values()) or 1
         print("PROFILE " + setting + " " + " ".join(f"{k}={100 * v / tot:.1f}" for k, v in reg.items() if v), flush=True)

@@ -29,7 +29,11 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "BC GTEPS and sec/source at 1/2/4/8 B200; HBM GB/s fraction of peak"
-SOURCES_PER_GPU = {1: 1024, 2: 1024, 3: 4096, 4: 1024, 5: 1024}
+SOURCES_PER_GPU = {1: 1024, 2: 1024, 3: 4096, 4: 1024, 5: 1024, 6: None, 7: 1024}
+# the paper's printed figure for the SAME workload (context: Titan Xp), GTEPS
+PAPER_GTEPS = {6: (10.257, "Table 5 P:452: exact BC of mycielski16, 159.8 s, 10,257 MTEPs on a Titan Xp"),
+               7: (18.470, "Table 3 P:380: one source of mycielski19, 48.9 ms, 18,470 MTEPs on a Titan Xp")}
+EXACT = (6,)  # configs whose step is exact BC over all n sources, split across the ranks
 
 
 def parse():
@@ -45,7 +49,8 @@ def parse():
     ap.add_argument("--direction", type=int, default=0)
     ap.add_argument("--format", type=int, default=0, help="0 auto, 1 list passes, 2 edge streams")
     ap.add_argument("--engine", choices=["csc", "coot"], default="csc")
-    ap.add_argument("--batch", type=int, default=1, help="1: batched engine (32 sources per sweep), 0: per source")
+    ap.add_argument("--batch", type=int, default=1, help="1: batched engine, 0: per source")
+    ap.add_argument("--width", type=int, default=32, help="batched engine: sources per sweep (32 or 64)")
     ap.add_argument("--cost", default="", help="cost model overrides, e.g. list=10,stream=2")
     ap.add_argument("--trace", type=int, default=-1, help="print the per-level timeline of this source to stderr")
     return ap.parse_args()
@@ -143,8 +148,11 @@ def run_reference(args):
         return
     import oracle
     g, _ = make_graph(args.config, "cpu" if args.config in (1,) else _gen_device())
-    per_gpu = args.sources or SOURCES_PER_GPU[args.config]
-    srcs = source_list(g, args.config, per_gpu * args.gpus)
+    if args.config in EXACT:
+        srcs = np.arange(g.n, dtype=np.int32)
+    else:
+        per_gpu = args.sources or SOURCES_PER_GPU[args.config]
+        srcs = source_list(g, args.config, per_gpu * args.gpus)
     cores = os.cpu_count() or 1
     k = args.cpu_sample or min(max(cores, 4), 64)
     times = []
@@ -199,10 +207,17 @@ def main():
         dist.init_process_group("nccl", device_id=dev)
 
     g, gen_s = make_graph(args.config, "cuda")
-    per_gpu = args.sources or SOURCES_PER_GPU[args.config]
-    all_src = source_list(g, args.config, per_gpu * world)
-    lo, hi = rank * per_gpu, (rank + 1) * per_gpu
-    my_src = all_src[lo:hi]
+    if args.config in EXACT:  # exact BC: all n sources per step, split across the ranks
+        all_src = np.arange(g.n, dtype=np.int32)
+        my_src = np.array_split(all_src, world)[rank]
+        per_gpu = len(my_src)
+        n_sources = g.n
+    else:
+        per_gpu = args.sources or SOURCES_PER_GPU[args.config]
+        all_src = source_list(g, args.config, per_gpu * world)
+        lo, hi = rank * per_gpu, (rank + 1) * per_gpu
+        my_src = all_src[lo:hi]
+        n_sources = per_gpu * world
     t0 = time.time()
     engine = tbc.ENGINE_COOT if args.engine == "coot" else tbc.ENGINE_CSC
     G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, engine=engine, device=local)
@@ -210,6 +225,7 @@ def main():
     G.set_direction(args.direction)
     G.set_format(args.format)
     G.set_batch(args.batch)
+    G.set_batch_width(args.width)
     batched = bool(args.batch) and args.engine == "csc"
     kname = "k_bcb" if batched else "k_bc"
     if args.cost:
@@ -254,7 +270,7 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
     st = G.stats()
-    sources_total = per_gpu * world * args.steps
+    sources_total = n_sources * args.steps
     gteps = sources_total * g.nnz / (total_ms / 1e3) / 1e9
     ms_per_step = total_ms / args.steps
 
@@ -289,7 +305,7 @@ def main():
         t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_s = float(t.item())
-    e2e_gteps = per_gpu * world * g.nnz / e2e_s / 1e9
+    e2e_gteps = n_sources * g.nnz / e2e_s / 1e9
 
     if rank == 0:
         cpu = None
@@ -298,8 +314,10 @@ def main():
         clocks = clk.summary()
         line = {
             "metric": METRIC, "value": gteps, "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
-            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "strong" if args.config in EXACT else "weak",
+            "vs_baseline": gteps / PAPER_GTEPS[args.config][0] if args.config in PAPER_GTEPS else None,
+            "dtype": "f64", "data": "synthetic",
             "sec_per_source": total_ms / 1e3 / sources_total,
             "config": {"workload": _workload_name(args.config), "n": g.n, "m": g.nnz,
                        "directed": g.directed, "engine": args.engine, "sources_per_gpu": per_gpu,
@@ -307,8 +325,9 @@ def main():
                        "l2": "inputs larger than L2 (CSC+CSR %.0f MB vs 126 MB L2); no flush" %
                              ((8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) / 1e6),
                        "direction": args.direction, "format": args.format, "engine_kind": args.engine,
-                       "engine_mode": "batched, 32 sources per sweep (one per warp lane)" if batched
+                       "engine_mode": f"batched, {args.width} sources per sweep" if batched
                        else "per source, SM partitions",
+                       "paper": PAPER_GTEPS[args.config][1] if args.config in PAPER_GTEPS else None,
                        "cost": args.cost},
             "clocks": clocks,
             "gpu_launches": args.steps,

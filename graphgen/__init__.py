@@ -225,21 +225,32 @@ def random_tree(n: int, seed: int) -> Graph:
     return from_edges(f"tree{n}_s{seed}", n, e, False)
 
 
-def mycielski(k: int) -> Graph:
+def mycielski(k: int, device: str = "cpu") -> Graph:
     """Mycielski graph M_k (networkx convention: M_1 = K_1, M_2 = K_2); the paper's
-    'mycielski15..19' (Table 3) are M_15..M_19 of SuiteSparse."""
+    'mycielski15..19' (Table 3) are M_15..M_19 of SuiteSparse.  device="cuda" builds
+    the edge list and the CSC with torch on the GPU (M_19 has 903 M stored entries)."""
     if k == 1:
         return from_edges("mycielski1", 1, [], False)
-    eu = np.array([0], dtype=np.int64)
-    ev = np.array([1], dtype=np.int64)
+    xp_cat = np.concatenate if device == "cpu" else torch.cat
+    if device == "cpu":
+        arange = lambda a, b: np.arange(a, b, dtype=np.int64)  # noqa: E731
+        full = lambda c, v: np.full(c, v, dtype=np.int64)  # noqa: E731
+        eu, ev = np.array([0], dtype=np.int64), np.array([1], dtype=np.int64)
+    else:
+        arange = lambda a, b: torch.arange(a, b, dtype=torch.int64, device=device)  # noqa: E731
+        full = lambda c, v: torch.full((c,), v, dtype=torch.int64, device=device)  # noqa: E731
+        eu = torch.tensor([0], dtype=torch.int64, device=device)
+        ev = torch.tensor([1], dtype=torch.int64, device=device)
     n = 2
     for _ in range(k - 2):
         # Mycielskian: copies u_i = i + n adjacent to N(v_i), hub w = 2n adjacent to all u_i
-        ui = np.arange(n, 2 * n, dtype=np.int64)
-        eu, ev = (np.concatenate([eu, eu, eu + n, ui]),
-                  np.concatenate([ev, ev + n, ev, np.full(n, 2 * n, dtype=np.int64)]))
+        ui = arange(n, 2 * n)
+        eu, ev = (xp_cat([eu, eu, eu + n, ui]), xp_cat([ev, ev + n, ev, full(n, 2 * n)]))
         n = 2 * n + 1
-    cp, ri = csc_from_edges(n, eu, ev, directed=False)
+    if device == "cpu":
+        cp, ri = csc_from_edges(n, eu, ev, directed=False)
+    else:
+        cp, ri = csc_from_edges_torch(n, eu, ev, directed=False)
     return Graph(f"mycielski{k}", n, cp, ri, False)
 
 
@@ -264,12 +275,16 @@ CONFIGS = {
     3: dict(name="cfg3_kron22_dir", kind="kron", scale=22, ef=16, seed=3, directed=True, k=4096, src_seed=13),
     4: dict(name="cfg4_road4096", kind="road", side=4096, q=0.10, seed=4, directed=False, k=1024, src_seed=14),
     5: dict(name="cfg5_kron25_undir", kind="kron", scale=25, ef=16, seed=5, directed=False, k=8192, src_seed=15),
+    # the paper's own best-case inputs, reproduced exactly up to vertex labels:
+    # exact BC of mycielski16 (Table 5) and single sources of mycielski19 (Table 3)
+    6: dict(name="cfg6_mycielski16_exact", kind="myc", myc=16, directed=False, k=None, src_seed=None),
+    7: dict(name="cfg7_mycielski19_sources", kind="myc", myc=19, directed=False, k=1024, src_seed=17),
 }
 
 
 def make_config(cfg: int, device: str = "cpu", scale_override: int | None = None,
                 side_override: int | None = None):
-    """(Graph, sources) for config 1..5; overrides shrink the graph for fast tests."""
+    """(Graph, sources) for config 1..7; overrides shrink the graph for fast tests."""
     c = CONFIGS[cfg]
     if c["kind"] == "er":
         g = erdos_renyi(c["n"], c["M"], c["seed"], c["directed"])
@@ -277,6 +292,9 @@ def make_config(cfg: int, device: str = "cpu", scale_override: int | None = None
     elif c["kind"] == "kron":
         g = kronecker(scale_override or c["scale"], c["ef"], c["seed"], c["directed"], device=device)
         src = sources(g, c["k"], c["src_seed"])
+    elif c["kind"] == "myc":
+        g = mycielski(c["myc"], device=device)
+        src = np.arange(g.n, dtype=np.int32) if c["k"] is None else sources(g, c["k"], c["src_seed"])
     else:
         g = road_lattice(side_override or c["side"], c["q"], c["seed"])
         src = sources(g, c["k"], c["src_seed"])

@@ -278,6 +278,10 @@ def main():
     # B_min = 8 B per out-edge of the reached set (4 B index read once per stage) + 80 B per
     # reached vertex, summed over the launch's sources; / the kernel's event-timed duration.
     alg_bytes_per_launch = (8.0 * st["reached_edges"] + 80.0 * st["reached"]) / args.steps
+    # the batched engine's own compulsory traffic: the index stream once per stage per BATCH of W
+    # sources (8 B per reached edge / W per source) + the per-(vertex, source) state (80 B)
+    wdt = args.width if batched else 1
+    alg_bytes_batched = (8.0 * st["reached_edges"] / wdt + 80.0 * st["reached"]) / args.steps
     k_avg_s = statistics.mean(kern_ms) / 1e3
     peak, peak_kind = peaks()
     achieved = alg_bytes_per_launch / k_avg_s / 1e9
@@ -334,6 +338,10 @@ def main():
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
                          "kernel": kname, "alg_bytes_per_launch": alg_bytes_per_launch,
+                         "model": "SURVEY 8(d) B_min = 8 B per reached edge + 80 B per reached vertex, per "
+                                  "source; a batch shares the index stream, so frac may exceed 1",
+                         "achieved_batched_model": alg_bytes_batched / k_avg_s / 1e9,
+                         "frac_batched_model": alg_bytes_batched / k_avg_s / 1e9 / peak,
                          "kernel_ms": statistics.mean(kern_ms)},
             "e2e": {"value": e2e_gteps, "unit": "GTEPS", "h2d_bytes_per_step": 4 * len(my_src),
                     "d2h_bytes_per_step": 8 * g.n},

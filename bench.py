@@ -50,7 +50,7 @@ def parse():
     ap.add_argument("--format", type=int, default=0, help="0 auto, 1 list passes, 2 edge streams")
     ap.add_argument("--engine", choices=["csc", "coot"], default="csc")
     ap.add_argument("--batch", type=int, default=1, help="1: batched engine, 0: per source")
-    ap.add_argument("--width", type=int, default=32, help="batched engine: sources per sweep (32 or 64)")
+    ap.add_argument("--width", type=int, default=0, help="batched engine: sources per sweep (32, 64; 0 auto)")
     ap.add_argument("--cost", default="", help="cost model overrides, e.g. list=10,stream=2")
     ap.add_argument("--trace", type=int, default=-1, help="print the per-level timeline of this source to stderr")
     return ap.parse_args()
@@ -280,7 +280,7 @@ def main():
     alg_bytes_per_launch = (8.0 * st["reached_edges"] + 80.0 * st["reached"]) / args.steps
     # the batched engine's own compulsory traffic: the index stream once per stage per BATCH of W
     # sources (8 B per reached edge / W per source) + the per-(vertex, source) state (80 B)
-    wdt = args.width if batched else 1
+    wdt = (args.width or (64 if g.n * 64 * 16 <= (1 << 30) else 32)) if batched else 1
     alg_bytes_batched = (8.0 * st["reached_edges"] / wdt + 80.0 * st["reached"]) / args.steps
     k_avg_s = statistics.mean(kern_ms) / 1e3
     peak, peak_kind = peaks()
@@ -329,7 +329,7 @@ def main():
                        "l2": "inputs larger than L2 (CSC+CSR %.0f MB vs 126 MB L2); no flush" %
                              ((8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) / 1e6),
                        "direction": args.direction, "format": args.format, "engine_kind": args.engine,
-                       "engine_mode": f"batched, {args.width} sources per sweep" if batched
+                       "engine_mode": f"batched, {wdt} sources per sweep" if batched
                        else "per source, SM partitions",
                        "paper": PAPER_GTEPS[args.config][1] if args.config in PAPER_GTEPS else None,
                        "cost": args.cost},

@@ -100,7 +100,8 @@ enum {
                                 when the frontier's out-edges x this value > nnz, else pushed
                                 (default 8; must be >= 0) */
     TBC_OPT_BATCH_WIDTH = 14 /* batched engine: sources per sweep, 32 (one per warp lane) or 64
-                                (two per lane); default 32.  Workspace ~ 2 x 8 W B/vertex of (sigma,
+                                (two per lane), or 0 (default) = 64 when n x 1 KiB <= 1 GiB, else
+                                32 (measured crossover).  Workspace ~ 2 x 8 W B/vertex of (sigma,
                                 delta_u) rows plus level lists of <= W entries per vertex. */
 };
 

@@ -532,7 +532,8 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         return TBC_OK;
     }
     if (key == TBC_OPT_BATCH_WIDTH) {
-        if (value != 32 && value != 64) return set_error(TBC_ERR_INVALID, "batch width %g not 32 or 64", value);
+        if (value != 0 && value != 32 && value != 64)
+            return set_error(TBC_ERR_INVALID, "batch width %g not 0 (auto), 32 or 64", value);
         g->batch_width = (int)value;
         return TBC_OK;
     }

@@ -876,8 +876,16 @@ void batch_free(tbc_graph *g) {
     w = BatchWorkspace{};
 }
 
+// auto width: 64 sources per sweep while the (sigma, delta_u) rows stay within 1 GiB (measured:
+// faster on RMAT scale 18 and the mycielski graphs), else 32 (faster on Kronecker scale 22, whose
+// rows miss in L2 either way and the wider rows cost more gather locality than they save)
+int batch_width(const tbc_graph *g) {
+    if (g->batch_width) return g->batch_width;
+    return g->n * 64 * 16 <= (1ll << 30) ? 64 : 32;
+}
+
 tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream) {
-    const int W = g->batch_width;
+    const int W = batch_width(g);
     tbc_status st = batch_alloc(g, W);
     if (st != TBC_OK) return st;
     const BatchWorkspace &w = g->bws;

@@ -174,7 +174,7 @@ struct tbc_graph {
     int fmt_mode = 0;
     double c_list = 12.0, c_stream = 4.0, c_atom = 18.0, c_vert = 10.0, c_scan = 3.0, c_bpush = 6.0;
     int batch = 1;                // TBC_OPT_BATCH: 1 batched engine, 0 per source
-    int batch_width = 32;         // TBC_OPT_BATCH_WIDTH: sources per sweep (32 or 64)
+    int batch_width = 0;          // TBC_OPT_BATCH_WIDTH: sources per sweep (32 or 64; 0 auto)
     double batch_pull = 8.0;      // TBC_OPT_BATCH_PULL: pull when frontier out-edges x this > m
     tbc::BatchWorkspace bws;
     int bgrid = 0;
@@ -196,5 +196,6 @@ tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
                       cudaStream_t stream, int bfs_only);
 // batched engine (tbc_batch.cu)
 tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream);
+int batch_width(const tbc_graph *g);  // sources per sweep the next batched call uses
 void batch_free(tbc_graph *g);
 }  // namespace tbc

@@ -121,7 +121,7 @@ def test_sm_partitions(directed):
             G.set_partitions(9)
 
 
-@pytest.mark.parametrize("width", [32, 64])
+@pytest.mark.parametrize("width", [0, 32, 64])
 @pytest.mark.parametrize("directed", [False, True])
 @pytest.mark.parametrize("pull", [0.0, 8.0, 1e9])
 def test_batched_engine(directed, pull, width):

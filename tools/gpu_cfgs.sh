@@ -1,6 +1,12 @@
 #!/bin/bash
 mkdir -p gpurun_out
-( for c in 1 2; do timeout 600 python tools/tune.py --config $c --sources 1024 --reps 2 --settings "batch=1;batch=0" 2>&1 | grep -v TRACE | cut -c1-160; done
-  timeout 900 python tools/tune.py --config 4 --sources 64 --reps 1 --settings "batch=1;batch=0" 2>&1 | grep -v TRACE | cut -c1-160
-) > gpurun_out/cfgs.log 2>&1
-cat gpurun_out/cfgs.log
+timeout 900 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err; echo "ref rc=$?"
+timeout 1500 python bench.py --config 5 --steps 3 --warmup 3 > gpurun_out/bench_cfg5.json 2> gpurun_out/bench_cfg5.err; echo "cfg5 rc=$?"
+timeout 1500 python bench.py --config 4 --sources 64 --steps 3 --warmup 3 > gpurun_out/bench_cfg4.json 2> gpurun_out/bench_cfg4.err; echo "cfg4 rc=$?"
+timeout 900 python bench.py --config 2 --steps 5 --warmup 3 > gpurun_out/bench_cfg2.json 2> gpurun_out/bench_cfg2.err; echo "cfg2 rc=$?"
+for f in gpurun_out/bench_ref.json gpurun_out/bench_cfg5.json gpurun_out/bench_cfg4.json gpurun_out/bench_cfg2.json; do python -c "
+import json
+d=json.loads(open('$f').read())
+print('$f', round(d['value'],3), d['config'].get('engine_mode'), 'ms/step', round(d['ms_per_step'],1), 'e2e', round(d['e2e']['value'],3), 'frac', d.get('roofline',{}).get('frac'), 'cpu', d['cpu_baseline'] and round(d['cpu_baseline']['value'],3), 'dev_bytes', d.get('setup',{}).get('device_bytes'))
+" 2>&1 | tail -1; done
+tail -2 gpurun_out/*.err

@@ -537,6 +537,13 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->batch_width = (int)value;
         return TBC_OK;
     }
+    if (key == TBC_OPT_BATCH_PARTS) {
+        int v = (int)value;
+        if (v < 0 || v > kMaxPartitions || (double)v != value)
+            return set_error(TBC_ERR_INVALID, "batch partitions %g not in [0 (auto), %d]", value, kMaxPartitions);
+        g->batch_parts = v;
+        return TBC_OK;
+    }
     if (key == TBC_OPT_BATCH_PULL) {
         if (!(value >= 0)) return set_error(TBC_ERR_INVALID, "batch pull ratio %g", value);
         g->batch_pull = value;
@@ -639,8 +646,8 @@ tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
     TBC_CUDA(cudaSetDevice(g->device));
     TBC_CUDA(cudaDeviceSynchronize());
     *out = tbc_stats{};
-    for (int i = 0; i <= g->ws_count; ++i) {  // summed over the SM partitions' and the batch counters
-        Ctrs *src = i < g->ws_count ? g->ws[i].ctr : g->bws.ctr;
+    for (int i = 0; i < g->ws_count + kMaxPartitions; ++i) {  // per-source and batched partitions
+        Ctrs *src = i < g->ws_count ? g->ws[i].ctr : g->bws[i - g->ws_count].ctr;
         if (!src) continue;
         TBC_CUDA(cudaMemcpy(&c, src, sizeof c, cudaMemcpyDeviceToHost));
         out->sources += c.st_sources;
@@ -703,7 +710,8 @@ tbc_status tbc_stats_reset(tbc_graph *g) {
     TBC_CUDA(cudaDeviceSynchronize());
     for (int i = 0; i < g->ws_count; ++i)
         TBC_CUDA(cudaMemset(&g->ws[i].ctr->st_sources, 0, sizeof(long long) * 9));
-    if (g->bws.ctr) TBC_CUDA(cudaMemset(&g->bws.ctr->st_sources, 0, sizeof(long long) * 9));
+    for (int q = 0; q < kMaxPartitions; ++q)
+        if (g->bws[q].ctr) TBC_CUDA(cudaMemset(&g->bws[q].ctr->st_sources, 0, sizeof(long long) * 9));
     return TBC_OK;
 fail:
     return st;

@@ -97,8 +97,16 @@ struct BParams {
     int64_t k, n_scan, list_cap, tiles_cap, cand_tiles_cap;
     double bc_scale, pull_ratio;
     int ebits, dir_mode;
-    int64_t *trace;  // per-phase timeline of batch trace_b (TBC_OPT_TRACE: source index / 32)
+    int64_t *trace;  // per-phase timeline of batch trace_b (TBC_OPT_TRACE: source index / W)
     int64_t trace_cap, trace_b;
+};
+
+// one launch: a BParams per SM partition (its own workspace and counters/barrier); partition q
+// runs the batches q, q + nparts, ... on CTAs [q * cta_per_part, (q + 1) * cta_per_part)
+constexpr int kBParts = 8;
+struct BParamSet {
+    BParams p[kBParts];
+    int nparts, cta_per_part;
 };
 
 struct __align__(16) BWarpSmem {
@@ -123,7 +131,7 @@ __device__ __forceinline__ int64_t cdiv(int64_t a, int64_t b) { return (a + b - 
 // kinds as tbc_trace_get: 0 init, 1 level masks + candidates (B phase), 2 push, 3 pull, 4 backward
 __device__ __forceinline__ void btrace(const BParams &P, bool on, int kind, int64_t level, int64_t N, int64_t E,
                                        int64_t a, int64_t b) {
-    if (!on || blockIdx.x != 0 || threadIdx.x != 0) return;
+    if (!on || threadIdx.x != 0) return;  // on: the traced batch, CTA 0 of its partition
     const unsigned long long i = P.gctr->trace_n;
     if ((int64_t)i >= P.trace_cap) return;
     int64_t *t = P.trace + 8 * i;
@@ -567,19 +575,24 @@ __device__ __forceinline__ void bclear(const BParams &P, const Lv &l, void *fr_,
     }
 }
 
-template <int W>
-__global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams P) {
+// MULTI = false: one partition, every parameter at a static offset (S.p[0]); MULTI = true: the
+// partition's parameters are indexed by blockIdx (costs registers, so only used when P > 1)
+template <int W, bool MULTI>
+__global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSet S) {
     using MT = typename MaskT<W>::T;
     constexpr int NS = W / 32;
+    const int part = MULTI ? (int)blockIdx.x / S.cta_per_part : 0;
+    const BParams &P = S.p[part];
+    const int lcta = MULTI ? (int)blockIdx.x - part * S.cta_per_part : (int)blockIdx.x;  // CTA in the partition
     extern __shared__ __align__(16) unsigned char bsm[];
     BWarpSmem &ws = reinterpret_cast<BWarpSmem *>(bsm)[threadIdx.x >> 5];
     const int tid = threadIdx.x, lane = tid & 31;
-    const bool cta0 = blockIdx.x == 0;
-    const unsigned ncta = gridDim.x;
+    const bool cta0 = lcta == 0;
+    const unsigned ncta = MULTI ? (unsigned)S.cta_per_part : gridDim.x;
     const int64_t nwarps = (int64_t)ncta * kBWarps;
-    const int64_t gwarp = (int64_t)blockIdx.x * kBWarps + (tid >> 5);
+    const int64_t gwarp = (int64_t)lcta * kBWarps + (tid >> 5);
     const int64_t nthreads = (int64_t)ncta * kBB;
-    const int64_t gtid = (int64_t)blockIdx.x * kBB + tid;
+    const int64_t gtid = (int64_t)lcta * kBB + tid;
     Ctrs *C = P.ctr;
     unsigned gen = (tid == 0) ? ld_acquire(&C->bar_gen) : 0u;
     const unsigned long long emask = (1ull << P.ebits) - 1ull;
@@ -593,7 +606,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
     __syncthreads();
     const unsigned long long t_kernel0 = clock64();
 #endif
-    for (int64_t b = 0; b < nb; ++b) {
+    for (int64_t b = part; b < nb; b += MULTI ? S.nparts : 1) {
         // ---------------- level 0: the batch's sources (Alg.1 l.15-18): source b*W + 32k + l is
         // lane l's source k; a vertex repeated in the batch is appended once, by its lowest source
         if (cta0 && tid < 32) {
@@ -653,7 +666,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
                 C->st_sources += valid;
             }
         }
-        const bool tr = b == P.trace_b;
+        const bool tr = b == P.trace_b && cta0;
         if (tr && cta0 && tid == 0) P.gctr->trace_n = 0;
         bsync(C, gen, ncta);
         btrace(P, tr, 0, 0, 0, 0, 0, 0);
@@ -818,10 +831,10 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParams 
 
 // ------------------------------------------------------------------ host side
 
-static tbc_status batch_alloc(tbc_graph *g, int W) {
-    BatchWorkspace &w = g->bws;
+static tbc_status batch_alloc(tbc_graph *g, int q, int W) {
+    BatchWorkspace &w = g->bws[q];
     if (w.ready && w.width == W) return TBC_OK;
-    if (w.ready) batch_free(g);  // other width: reallocate
+    if (w.ready) batch_free_one(g, q);  // other width: reallocate
     const int64_t n = g->n, m = g->m;
     const int64_t nw = W / 32;  // 32-bit words per mask
     cudaStream_t s = g->stream;
@@ -855,25 +868,33 @@ static tbc_status batch_alloc(tbc_graph *g, int W) {
         (e = cudaMemsetAsync(w.fr[1], 0, sizeof(uint32_t) * n * nw, s)) ||
         (e = cudaMemsetAsync(w.ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s)))
         return cuda_error(e, "batch workspace init");
-    const void *fn = W == 64 ? (const void *)k_bcb<64> : (const void *)k_bcb<32>;
-    int per_sm = 0, sms = 0;
-    if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmem)) ||
-        (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kBB, kBSmem)) ||
-        (e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device)))
-        return cuda_error(e, "batch occupancy query");
-    if (per_sm < 1) return set_error(TBC_ERR_CUDA, "k_bcb cannot be resident (occupancy 0)");
-    g->bgrid = per_sm * sms;
+    if (!g->bgrid) {
+        int per_sm = 0, sms = 0;
+        for (const void *fn : {(const void *)k_bcb<32, false>, (const void *)k_bcb<64, false>,
+                               (const void *)k_bcb<32, true>, (const void *)k_bcb<64, true>})
+            if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmem)))
+                return cuda_error(e, "batch smem attribute");
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, (const void *)k_bcb<64, true>, kBB, kBSmem)) ||
+            (e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device)))
+            return cuda_error(e, "batch occupancy query");
+        if (per_sm < 1) return set_error(TBC_ERR_CUDA, "k_bcb cannot be resident (occupancy 0)");
+        g->bgrid = per_sm * sms;
+    }
     w.ready = true;
     return TBC_OK;
 }
 
-void batch_free(tbc_graph *g) {
-    BatchWorkspace &w = g->bws;
+void batch_free_one(tbc_graph *g, int q) {
+    BatchWorkspace &w = g->bws[q];
     void *ps[] = {w.sig, w.du, w.vis, w.fr[0], w.fr[1], w.list_v, w.list_pre, w.list_beg, w.list_m, w.tiles,
                   w.cand_v, w.cand_pre, w.cand_beg, w.cand_tiles, w.lvl, w.ctr};
     for (void *p : ps) cudaFree(p);
     g->device_bytes -= w.bytes;
     w = BatchWorkspace{};
+}
+
+void batch_free(tbc_graph *g) {
+    for (int q = 0; q < kMaxPartitions; ++q) batch_free_one(g, q);
 }
 
 // auto width: 64 sources per sweep while the (sigma, delta_u) rows stay within 1 GiB (measured:
@@ -884,55 +905,86 @@ int batch_width(const tbc_graph *g) {
     return g->n * 64 * 16 <= (1ll << 30) ? 64 : 32;
 }
 
+// auto partitions (measured): wide-level graphs -- sigma rows beyond 1 GiB with
+// average degree >= 8 (Kronecker 22/25), or average degree >= 64 (mycielski) -- keep the whole GPU
+// on one batch; the others (RMAT 18, high-diameter lattices) run up to 8 batches side by side, as
+// many as fit in 80 % of the free device memory
+static int batch_auto_parts(tbc_graph *g, int W) {
+    const int64_t n = g->n, m = g->m;
+    if ((n * (int64_t)W * 16 > (1ll << 30) && m >= 8 * n) || m >= 64 * n) return 1;
+    const double per = 16.0 * W * n + 16.0 * W * n + 4.0 * W * (n + m) / kBT + 64.0 * n;  // rows, lists, tiles, rest
+    size_t fr = 0, tot = 0;
+    if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) return 1;
+    double have = 0.8 * (double)fr;
+    for (int q = 0; q < kMaxPartitions; ++q) have += g->bws[q].ready ? (double)g->bws[q].bytes : 0.0;
+    int np = 1;
+    while (np < kMaxPartitions && (np * 2) * per <= have) np *= 2;
+    return np;
+}
+
 tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream) {
     const int W = batch_width(g);
-    tbc_status st = batch_alloc(g, W);
-    if (st != TBC_OK) return st;
-    const BatchWorkspace &w = g->bws;
-    BParams P{};
-    P.n = g->n;
-    P.m = g->m;
-    P.in_ptr = g->in_ptr;
-    P.in_idx = g->in_idx;
-    P.out_ptr = g->out_ptr;
-    P.out_idx = g->out_idx;
-    P.deg2 = g->deg2;
-    P.sig = w.sig;
-    P.du = w.du;
-    P.vis = w.vis;
-    P.fr0 = w.fr[0];
-    P.fr1 = w.fr[1];
-    P.list_v = w.list_v;
-    P.list_pre = w.list_pre;
-    P.list_beg = w.list_beg;
-    P.list_m = w.list_m;
-    P.tiles = w.tiles;
-    P.cand_v = w.cand_v;
-    P.cand_pre = w.cand_pre;
-    P.cand_beg = w.cand_beg;
-    P.cand_tiles = w.cand_tiles;
-    P.lvl = w.lvl;
-    P.ctr = w.ctr;
-    P.gctr = g->gctr;
-    P.bc = d_bc;
-    P.sources = d_sources;
-    P.perm = g->perm;
-    P.inv = g->inv;
-    P.k = k;
-    P.n_scan = g->n_scan;
-    P.list_cap = w.list_cap;
-    P.tiles_cap = w.tiles_cap;
-    P.cand_tiles_cap = w.cand_tiles_cap;
-    P.bc_scale = g->directed ? 1.0 : 0.5;
-    P.pull_ratio = g->batch_pull;
-    P.ebits = g->ebits;
-    P.dir_mode = g->dir_mode;
-    P.trace = g->trace;
-    P.trace_cap = g->trace ? kTraceCap : 0;
-    P.trace_b = g->trace_src >= 0 ? g->trace_src / W : -1;
-    void *args[] = {&P};
-    const void *fn = W == 64 ? (const void *)k_bcb<64> : (const void *)k_bcb<32>;
-    cudaError_t e = cudaLaunchCooperativeKernel(fn, dim3(g->bgrid), dim3(kBB), args, kBSmem, stream);
+    const int64_t nb = (k + W - 1) / W;
+    int np = g->batch_parts ? g->batch_parts : batch_auto_parts(g, W);
+    if (np > nb) np = (int)nb;
+    if (np < 1) np = 1;
+    for (int q = 0; q < np; ++q) {
+        tbc_status st = batch_alloc(g, q, W);
+        if (st != TBC_OK) return st;
+    }
+    if (np > g->bgrid) np = g->bgrid;
+    static_assert(sizeof(BParamSet) <= 32000, "kernel parameter space");
+    BParamSet S{};
+    S.nparts = np;
+    S.cta_per_part = g->bgrid / np;
+    for (int q = 0; q < np; ++q) {
+        const BatchWorkspace &w = g->bws[q];
+        BParams &P = S.p[q];
+        P.n = g->n;
+        P.m = g->m;
+        P.in_ptr = g->in_ptr;
+        P.in_idx = g->in_idx;
+        P.out_ptr = g->out_ptr;
+        P.out_idx = g->out_idx;
+        P.deg2 = g->deg2;
+        P.sig = w.sig;
+        P.du = w.du;
+        P.vis = w.vis;
+        P.fr0 = w.fr[0];
+        P.fr1 = w.fr[1];
+        P.list_v = w.list_v;
+        P.list_pre = w.list_pre;
+        P.list_beg = w.list_beg;
+        P.list_m = w.list_m;
+        P.tiles = w.tiles;
+        P.cand_v = w.cand_v;
+        P.cand_pre = w.cand_pre;
+        P.cand_beg = w.cand_beg;
+        P.cand_tiles = w.cand_tiles;
+        P.lvl = w.lvl;
+        P.ctr = w.ctr;
+        P.gctr = g->gctr;
+        P.bc = d_bc;  // shared by the partitions: every bc update is an fp64 atomic add
+        P.sources = d_sources;
+        P.perm = g->perm;
+        P.inv = g->inv;
+        P.k = k;
+        P.n_scan = g->n_scan;
+        P.list_cap = w.list_cap;
+        P.tiles_cap = w.tiles_cap;
+        P.cand_tiles_cap = w.cand_tiles_cap;
+        P.bc_scale = g->directed ? 1.0 : 0.5;
+        P.pull_ratio = g->batch_pull;
+        P.ebits = g->ebits;
+        P.dir_mode = g->dir_mode;
+        P.trace = g->trace;
+        P.trace_cap = g->trace ? kTraceCap : 0;
+        P.trace_b = g->trace_src >= 0 ? g->trace_src / W : -1;
+    }
+    void *args[] = {&S};
+    const void *fn = np > 1 ? (W == 64 ? (const void *)k_bcb<64, true> : (const void *)k_bcb<32, true>)
+                            : (W == 64 ? (const void *)k_bcb<64, false> : (const void *)k_bcb<32, false>);
+    cudaError_t e = cudaLaunchCooperativeKernel(fn, dim3(S.cta_per_part * np), dim3(kBB), args, kBSmem, stream);
     if (e != cudaSuccess) return cuda_error(e, "cudaLaunchCooperativeKernel(k_bcb)");
     return TBC_OK;
 }

@@ -176,7 +176,8 @@ struct tbc_graph {
     int batch = 1;                // TBC_OPT_BATCH: 1 batched engine, 0 per source
     int batch_width = 0;          // TBC_OPT_BATCH_WIDTH: sources per sweep (32 or 64; 0 auto)
     double batch_pull = 8.0;      // TBC_OPT_BATCH_PULL: pull when frontier out-edges x this > m
-    tbc::BatchWorkspace bws;
+    tbc::BatchWorkspace bws[tbc::kMaxPartitions];  // one per SM partition of the batched engine
+    int batch_parts = 0;          // TBC_OPT_BATCH_PARTS: SM partitions of the batched engine (0 auto)
     int bgrid = 0;
     int64_t *trace = nullptr;     // device, 8 * kTraceCap int64
     int64_t trace_src = -1;       // index in the next call's source list to trace (-1: off)
@@ -198,4 +199,5 @@ tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
 tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream);
 int batch_width(const tbc_graph *g);  // sources per sweep the next batched call uses
 void batch_free(tbc_graph *g);
+void batch_free_one(tbc_graph *g, int q);
 }  // namespace tbc

@@ -121,10 +121,11 @@ def test_sm_partitions(directed):
             G.set_partitions(9)
 
 
+@pytest.mark.parametrize("parts", [0, 1, 3])
 @pytest.mark.parametrize("width", [0, 32, 64])
 @pytest.mark.parametrize("directed", [False, True])
 @pytest.mark.parametrize("pull", [0.0, 8.0, 1e9])
-def test_batched_engine(directed, pull, width):
+def test_batched_engine(directed, pull, width, parts):
     """Batched engine: several sweeps (full and ragged last batch of 32), repeated sources inside a
     batch and across batches, push-only / auto / pull-from-level-2 forward levels; repeat runs agree
     to rounding (fp64 atomics of split owners)."""
@@ -135,6 +136,7 @@ def test_batched_engine(directed, pull, width):
     with gpu_graph(g) as G:
         G.set_batch(1)
         G.set_batch_width(width)
+        G.set_batch_parts(parts)
         G.set_batch_pull(pull)
         a = G.bc(src)
         assert_bc(a, want)

@@ -1,4 +1,8 @@
 #!/bin/bash
-timeout 600 python tools/tune.py --config 3 --sources 512 --reps 1 --settings "hot=0;hot=-1;hot=200000;hot=500000;hot=1000000;hot=4194304" 2>&1 | grep -v TRACE | cut -c1-90
-TBC_VARIANT="-DTBC_BHOT=0" timeout 600 python tools/tune.py --config 3 --sources 512 --reps 1 --settings "hot=0" 2>&1 | grep -v TRACE | cut -c1-90
-timeout 600 python tools/tune.py --config 2 --sources 1024 --reps 1 --settings "hot=0;hot=-1;width=64,hot=0;width=64,hot=-1" 2>&1 | grep -v TRACE | cut -c1-90
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests -m gpu -x -q -k "batched or small_graphs or random_small or hub or star or cfg1 or kronecker_reduced or errors or device" > gpurun_out/pytest_batch.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_batch.log
+tail -3 gpurun_out/pytest_batch.log; grep -m2 -A25 "^____" gpurun_out/pytest_batch.log | head -40
+timeout 600 python tools/tune.py --config 3 --sources 1024 --reps 1 --settings "bparts=0;bparts=1;bparts=2" 2>&1 | grep -v TRACE | cut -c1-90
+timeout 600 python tools/tune.py --config 2 --sources 1024 --reps 1 --settings "bparts=0;bparts=8,width=32" 2>&1 | grep -v TRACE | cut -c1-90
+timeout 900 python tools/tune.py --config 4 --sources 256 --reps 1 --settings "bparts=0" 2>&1 | grep -v TRACE | cut -c1-90
+timeout 900 python tools/tune.py --config 6 --sources 4096 --reps 1 --settings "bparts=1;bparts=0;bparts=8,width=32" 2>&1 | grep -v TRACE | cut -c1-90

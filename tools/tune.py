@@ -38,6 +38,7 @@ for setting in a.settings.split(";"):
     G.set_batch(int(kv.get("batch", 1)))
     G.set_batch_width(int(kv.get("width", 32)))
     G.set_batch_pull(float(kv.get("bpull", 8)))
+    G.set_batch_parts(int(kv.get("bparts", 0)))
     G.set_cost(**{k: float(v) for k, v in kv.items() if k in ("list", "stream", "atomic", "vertex", "scan", "bpush")})
     G.bc_device(s_d, bc, st)  # warm-up
     torch.cuda.synchronize()

@@ -262,9 +262,10 @@ def test_kronecker_reduced_scale_full_oracle(scale, directed):
 
 
 def test_cfg2_rmat18_sample():
-    """Config 2 at full size: 64 of its 1024 sources against the oracle (all cores)."""
+    """Config 2 at full size in the bench's launch configuration (auto: 64 sources per sweep, SM
+    partitions): 288 of its 1024 sources (5 batches, the last ragged) against the oracle."""
     g, src = gg.make_config(2, device="cuda")
-    src = src[:64]
+    src = src[:288]
     with gpu_graph(g) as G:
         assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, False, src))
         for s in src[:2]:
@@ -291,6 +292,19 @@ def test_cfg3_kron22_directed_sample_in_bench_launch_config():
         s = int(src[100])
         depth, _ = G.bfs(s)
         assert abs(G.bc([s]).sum() - float(np.sum(depth[depth > 0] - 1))) <= 1e-9 * max(1.0, depth.sum())
+
+
+def test_road_lattice_partitions():
+    """High-diameter lattice through the batched engine's SM partitions (auto: 64 sources per sweep,
+    several partitions), 160 sources = 3 batches (the last ragged)."""
+    g = gg.road_lattice(512, 0.10, seed=4)
+    src = gg.sources(g, 160, seed=14)
+    want = oracle.bc(g.col_ptr, g.row_idx, False, src)
+    with gpu_graph(g) as G:
+        assert_bc(G.bc(src), want)
+        G.set_batch_parts(3)
+        G.set_batch_width(32)
+        assert_bc(G.bc(src), want)
 
 
 @pytest.mark.parametrize("side", [256, 1024])

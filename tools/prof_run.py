@@ -1,4 +1,4 @@
-"""ncu target: one warm-up k_bc launch, then one profiled launch over --sources sources of a config."""
+"""ncu target: one warm-up k_bcb (or k_bc) launch, then one profiled launch over --sources sources of a config."""
 import argparse, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
@@ -10,7 +10,7 @@ ap.add_argument("--sources", type=int, default=16)
 ap.add_argument("--settings", default="")
 a = ap.parse_args()
 g, _ = gg.make_config(a.config, device="cuda")
-src = gg.sources(g, a.sources, seed=gg.CONFIGS[a.config]["src_seed"])
+src = gg.sources(g, a.sources, seed=gg.CONFIGS[a.config]["src_seed"] or 0)
 G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed)
 kv = dict(x.split("=") for x in a.settings.split(",") if x)
 G.set_format(int(kv.get("fmt", 0)))

@@ -25,7 +25,7 @@ __all__ = ["Graph", "TBCError", "lib", "ENGINE_CSC", "ENGINE_COOT", "DIR_AUTO", 
 ENGINE_CSC, ENGINE_COOT = 0, 1
 FLAG_ONE_FORMAT, FLAG_NO_VALIDATE, FLAG_NO_REORDER = 1, 2, 4
 OPT_DIRECTION, OPT_BWD_DIRECTION, OPT_TRACE, OPT_FORMAT, OPT_PARTITIONS = 1, 2, 3, 4, 11
-OPT_BATCH, OPT_BATCH_PULL, OPT_BATCH_WIDTH, OPT_BATCH_PARTS = 12, 13, 14, 16
+OPT_BATCH, OPT_BATCH_PULL, OPT_BATCH_WIDTH, OPT_BATCH_PARTS, OPT_BATCH_ORDER = 12, 13, 14, 16, 17
 OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8, "scan": 9, "bpush": 10}
 FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
 DIR_AUTO, DIR_PUSH, DIR_PULL = 0, 1, 2
@@ -175,6 +175,10 @@ class Graph:
     def set_batch_parts(self, parts: int):
         """Batched engine: SM partitions running batches concurrently (1..8; TBC_OPT_BATCH_PARTS)."""
         _check(lib().tbc_graph_set_option(self._h, OPT_BATCH_PARTS, float(parts)))
+
+    def set_batch_order(self, grouped: int):
+        """Batched engine: 1 group the sources by out-degree into batches (default), 0 as given."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_BATCH_ORDER, float(grouped)))
 
     def set_batch_pull(self, ratio: float):
         """Batched engine: pull a level when frontier out-edges x ratio > nnz (TBC_OPT_BATCH_PULL)."""

@@ -544,6 +544,12 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->batch_parts = v;
         return TBC_OK;
     }
+    if (key == TBC_OPT_BATCH_ORDER) {
+        int v = (int)value;
+        if (v < 0 || v > 1 || (double)v != value) return set_error(TBC_ERR_INVALID, "batch order %g", value);
+        g->batch_order = v;
+        return TBC_OK;
+    }
     if (key == TBC_OPT_BATCH_PULL) {
         if (!(value >= 0)) return set_error(TBC_ERR_INVALID, "batch pull ratio %g", value);
         g->batch_pull = value;

@@ -116,6 +116,14 @@ struct Workspace {
 };
 constexpr int kMaxPartitions = 8;
 
+// device buffers of the batched engine's source grouping (grow-only)
+struct BatchOrder {
+    void *keys = nullptr;   // 2 x cap uint32 keys + 2 x cap int32 values
+    void *temp = nullptr;   // cub temp storage
+    int64_t cap = 0;
+    size_t temp_bytes = 0;
+};
+
 // workspace of the batched engine (tbc_batch.cu): W = 32 or 64 sources per sweep, lane l of a
 // warp holding sources l (and l + 32); masks are W-bit words (W / 32 uint32 words)
 struct BatchWorkspace {
@@ -178,6 +186,8 @@ struct tbc_graph {
     double batch_pull = 8.0;      // TBC_OPT_BATCH_PULL: pull when frontier out-edges x this > m
     tbc::BatchWorkspace bws[tbc::kMaxPartitions];  // one per SM partition of the batched engine
     int batch_parts = 0;          // TBC_OPT_BATCH_PARTS: SM partitions of the batched engine (0 auto)
+    int batch_order = 1;          // TBC_OPT_BATCH_ORDER: group the sources by out-degree into batches
+    tbc::BatchOrder border;
     int bgrid = 0;
     int64_t *trace = nullptr;     // device, 8 * kTraceCap int64
     int64_t trace_src = -1;       // index in the next call's source list to trace (-1: off)

@@ -137,6 +137,7 @@ def test_batched_engine(directed, pull, width, parts):
         G.set_batch(1)
         G.set_batch_width(width)
         G.set_batch_parts(parts)
+        G.set_batch_order(int(pull != 8.0))  # grouped order, and the given order for the default pull
         G.set_batch_pull(pull)
         a = G.bc(src)
         assert_bc(a, want)
@@ -216,6 +217,24 @@ def test_errors_and_semantics():
     with pytest.raises(tbc.TBCError) as e:
         tbc.Graph.from_csc(asym.col_ptr, asym.row_idx, directed=False)
     assert e.value.status == 1
+
+
+def test_bc_device_skips_out_of_range_sources():
+    """tbc_bc_device: out-of-range entries are skipped (not validated on the host), in both the
+    given and the grouped source order, and with the per-source engine."""
+    import torch
+    g = gg.kronecker(10, 8, seed=3, directed=True)
+    src = gg.sources(g, 70, seed=2)
+    bad = np.concatenate([src[:30], [-1, g.n, 1 << 30], src[30:]]).astype(np.int32)
+    want = oracle.bc(g.col_ptr, g.row_idx, True, src)
+    with gpu_graph(g) as G:
+        for batch, order in ((1, 1), (1, 0), (0, 1)):
+            G.set_batch(batch)
+            G.set_batch_order(order)
+            acc = torch.zeros(g.n, dtype=torch.float64, device="cuda")
+            G.bc_device(torch.from_numpy(bad).cuda(), acc)
+            torch.cuda.synchronize()
+            assert_bc(acc.cpu().numpy(), want)
 
 
 def test_bc_device_accumulates():

@@ -10,6 +10,7 @@ import os
 import sys
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 import graphgen as gg  # noqa: E402
@@ -23,8 +24,13 @@ ap.add_argument("--trace", default="")
 ap.add_argument("--reps", type=int, default=2)
 a = ap.parse_args()
 
+ap2 = None
 g, _ = gg.make_config(a.config, device="cuda")
-src = gg.sources(g, a.sources, seed=gg.CONFIGS[a.config]["src_seed"])
+src = gg.sources(g, a.sources, seed=gg.CONFIGS[a.config]["src_seed"] or 0)
+if os.environ.get("TUNE_SORT") == "deg":      # group sources of similar out-degree into batches
+    src = src[np.argsort(-g.out_degree()[src], kind="stable")]
+elif os.environ.get("TUNE_SORT") == "indeg":
+    src = src[np.argsort(-g.in_degree()[src], kind="stable")]
 G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed)
 s_d = torch.from_numpy(src).cuda()
 bc = torch.zeros(g.n, dtype=torch.float64, device="cuda")
@@ -39,6 +45,7 @@ for setting in a.settings.split(";"):
     G.set_batch_width(int(kv.get("width", 32)))
     G.set_batch_pull(float(kv.get("bpull", 8)))
     G.set_batch_parts(int(kv.get("bparts", 0)))
+    G.set_batch_order(int(kv.get("order", 1)))
     G.set_cost(**{k: float(v) for k, v in kv.items() if k in ("list", "stream", "atomic", "vertex", "scan", "bpush")})
     G.bc_device(s_d, bc, st)  # warm-up
     torch.cuda.synchronize()

@@ -51,6 +51,7 @@ def parse():
     ap.add_argument("--engine", choices=["csc", "coot"], default="csc")
     ap.add_argument("--batch", type=int, default=1, help="1: batched engine, 0: per source")
     ap.add_argument("--width", type=int, default=0, help="batched engine: sources per sweep (32, 64; 0 auto)")
+    ap.add_argument("--order", type=int, default=1, help="batched engine: 1 group sources by out-degree, 0 as given")
     ap.add_argument("--cost", default="", help="cost model overrides, e.g. list=10,stream=2")
     ap.add_argument("--trace", type=int, default=-1, help="print the per-level timeline of this source to stderr")
     return ap.parse_args()
@@ -226,6 +227,7 @@ def main():
     G.set_format(args.format)
     G.set_batch(args.batch)
     G.set_batch_width(args.width)
+    G.set_batch_order(args.order)
     batched = bool(args.batch) and args.engine == "csc"
     kname = "k_bcb" if batched else "k_bc"
     if args.cost:
@@ -329,7 +331,9 @@ def main():
                        "l2": "inputs larger than L2 (CSC+CSR %.0f MB vs 126 MB L2); no flush" %
                              ((8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) / 1e6),
                        "direction": args.direction, "format": args.format, "engine_kind": args.engine,
-                       "engine_mode": f"batched, {wdt} sources per sweep" if batched
+                       "engine_mode": f"batched, {wdt} sources per sweep"
+                       + (", sources grouped by out-degree" if args.order else ", sources in the given order")
+                       if batched
                        else "per source, SM partitions",
                        "paper": PAPER_GTEPS[args.config][1] if args.config in PAPER_GTEPS else None,
                        "cost": args.cost},

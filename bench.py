@@ -51,7 +51,7 @@ def parse():
     ap.add_argument("--engine", choices=["csc", "coot"], default="csc")
     ap.add_argument("--batch", type=int, default=1, help="1: batched engine, 0: per source")
     ap.add_argument("--width", type=int, default=0, help="batched engine: sources per sweep (32, 64; 0 auto)")
-    ap.add_argument("--order", type=int, default=1, help="batched engine: 1 group sources by out-degree, 0 as given")
+    ap.add_argument("--order", type=int, default=1, help="batched engine: 1 group sources by 2-hop out-volume, 0 as given")
     ap.add_argument("--cost", default="", help="cost model overrides, e.g. list=10,stream=2")
     ap.add_argument("--trace", type=int, default=-1, help="print the per-level timeline of this source to stderr")
     return ap.parse_args()
@@ -332,7 +332,7 @@ def main():
                              ((8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) / 1e6),
                        "direction": args.direction, "format": args.format, "engine_kind": args.engine,
                        "engine_mode": f"batched, {wdt} sources per sweep"
-                       + (", sources grouped by out-degree" if args.order else ", sources in the given order")
+                       + (", sources grouped by 2-hop out-volume" if args.order else ", sources in the given order")
                        if batched
                        else "per source, SM partitions",
                        "paper": PAPER_GTEPS[args.config][1] if args.config in PAPER_GTEPS else None,

@@ -110,8 +110,9 @@ enum {
                                 batches q, q + P, ... on its own SMs, workspace and barrier (one
                                 workspace each); bc accumulates with fp64 atomics from all of them */
     TBC_OPT_BATCH_ORDER = 17 /* batched engine: 1 (default) cut the call's sources into batches after a
-                                stable sort by out-degree (bc is a sum over sources, so only the
-                                floating-point summation order changes), 0 in the given order */
+                                stable sort by 2-hop out-volume class, then out-degree (bc is a sum
+                                over sources, so only the floating-point summation order changes),
+                                0 in the given order */
 };
 
 /* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since

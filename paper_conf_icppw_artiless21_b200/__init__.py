@@ -177,7 +177,7 @@ class Graph:
         _check(lib().tbc_graph_set_option(self._h, OPT_BATCH_PARTS, float(parts)))
 
     def set_batch_order(self, grouped: int):
-        """Batched engine: 1 group the sources by out-degree into batches (default), 0 as given."""
+        """Batched engine: 1 group the sources by 2-hop out-volume into batches (default), 0 as given."""
         _check(lib().tbc_graph_set_option(self._h, OPT_BATCH_ORDER, float(grouped)))
 
     def set_batch_pull(self, ratio: float):

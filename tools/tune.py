@@ -31,6 +31,20 @@ if os.environ.get("TUNE_SORT") == "deg":      # group sources of similar out-deg
     src = src[np.argsort(-g.out_degree()[src], kind="stable")]
 elif os.environ.get("TUNE_SORT") == "indeg":
     src = src[np.argsort(-g.in_degree()[src], kind="stable")]
+elif os.environ.get("TUNE_SORT", "").startswith("hop2"):
+    od = g.out_degree().astype(np.float64)
+    col = np.repeat(np.arange(g.n), np.diff(g.col_ptr))        # edge row_idx[e] -> col[e]
+    hop2 = np.bincount(g.row_idx, weights=od[col], minlength=g.n)  # sum of out-degrees of out-neighbours
+    if os.environ["TUNE_SORT"] == "hop2":
+        src = src[np.argsort(-hop2[src], kind="stable")]
+    elif os.environ["TUNE_SORT"] == "hop3":
+        hop3 = np.bincount(g.row_idx, weights=hop2[col], minlength=g.n)
+        src = src[np.argsort(-hop3[src], kind="stable")]
+    elif os.environ["TUNE_SORT"] == "hop2log":  # coarse classes of log2 volume, degree within
+        cls = np.floor(np.log2(hop2[src] + 1) * 4)
+        src = src[np.lexsort((-od[src], -cls))]
+    else:  # hop2deg: out-degree, ties by 2-hop volume
+        src = src[np.lexsort((-hop2[src], -od[src]))]
 G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed)
 s_d = torch.from_numpy(src).cuda()
 bc = torch.zeros(g.n, dtype=torch.float64, device="cuda")

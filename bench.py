@@ -282,7 +282,7 @@ def main():
     alg_bytes_per_launch = (8.0 * st["reached_edges"] + 80.0 * st["reached"]) / args.steps
     # the batched engine's own compulsory traffic: the index stream once per stage per BATCH of W
     # sources (8 B per reached edge / W per source) + the per-(vertex, source) state (80 B)
-    wdt = (args.width or (64 if g.n * 64 * 16 <= (1 << 30) else 32)) if batched else 1
+    wdt = (args.width or (64 if g.n <= (8 << 20) else 32)) if batched else 1
     alg_bytes_batched = (8.0 * st["reached_edges"] / wdt + 80.0 * st["reached"]) / args.steps
     k_avg_s = statistics.mean(kern_ms) / 1e3
     peak, peak_kind = peaks()

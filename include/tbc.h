@@ -100,13 +100,13 @@ enum {
                                 when the frontier's out-edges x this value > nnz, else pushed
                                 (default 8; must be >= 0) */
     TBC_OPT_BATCH_WIDTH = 14, /* batched engine: sources per sweep, 32 (one per warp lane) or 64
-                                (two per lane), or 0 (default) = 64 when n x 1 KiB <= 1 GiB, else
-                                32 (measured crossover).  Workspace ~ 2 x 8 W B/vertex of (sigma,
+                                (two per lane), or 0 (default) = 64 up to 8 M vertices, else 32
+                                (measured).  Workspace ~ 2 x 8 W B/vertex of (sigma,
                                 delta_u) rows plus level lists of <= W entries per vertex. */
     TBC_OPT_BATCH_PARTS = 16, /* batched engine: SM partitions (1..8, or 0 = auto, the default: 1 for
                                 graphs whose sigma rows overflow 1 GiB with average degree >= 8 or
-                                with average degree >= 64, else up to 8 fitting 80 % of free
-                                memory); partition q runs
+                                with average degree >= 64, else up to 4 (average degree >= 8) or 8
+                                fitting 80 % of free memory); partition q runs
                                 batches q, q + P, ... on its own SMs, workspace and barrier (one
                                 workspace each); bc accumulates with fp64 atomics from all of them */
     TBC_OPT_BATCH_ORDER = 17 /* batched engine: 1 (default) cut the call's sources into batches after a

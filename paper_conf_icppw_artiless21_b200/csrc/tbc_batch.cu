@@ -903,12 +903,12 @@ void batch_free(tbc_graph *g) {
     g->border = BatchOrder{};
 }
 
-// auto width: 64 sources per sweep while the (sigma, delta_u) rows stay within 1 GiB (measured:
-// faster on RMAT scale 18 and the mycielski graphs), else 32 (faster on Kronecker scale 22, whose
-// rows miss in L2 either way and the wider rows cost more gather locality than they save)
+// auto width (measured with grouped sources): 64 sources per sweep up to 8 M
+// vertices (faster on RMAT 18, Kronecker 22 and the mycielski graphs), else 32 (faster on
+// Kronecker 25, and half the workspace of the 16 M-vertex lattice)
 int batch_width(const tbc_graph *g) {
     if (g->batch_width) return g->batch_width;
-    return g->n * 64 * 16 <= (1ll << 30) ? 64 : 32;
+    return g->n <= (8ll << 20) ? 64 : 32;
 }
 
 // source grouping key of each source (one warp per source): its 2-hop out-volume V = sum of the
@@ -989,14 +989,15 @@ static tbc_status batch_group_sources(tbc_graph *g, const int32_t *d_sources, in
 // many as fit in 80 % of the free device memory
 static int batch_auto_parts(tbc_graph *g, int W) {
     const int64_t n = g->n, m = g->m;
-    if ((n * (int64_t)W * 16 > (1ll << 30) && m >= 8 * n) || m >= 64 * n) return 1;
+    if ((n * 32ll * 16 > (1ll << 30) && m >= 8 * n) || m >= 64 * n) return 1;
+    const int cap = m >= 8 * n ? 4 : kMaxPartitions;  // RMAT 18: 4 beats 8; lattices: 8
     const double per = 16.0 * W * n + 16.0 * W * n + 4.0 * W * (n + m) / kBT + 64.0 * n;  // rows, lists, tiles, rest
     size_t fr = 0, tot = 0;
     if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) return 1;
     double have = 0.8 * (double)fr;
     for (int q = 0; q < kMaxPartitions; ++q) have += g->bws[q].ready ? (double)g->bws[q].bytes : 0.0;
     int np = 1;
-    while (np < kMaxPartitions && (np * 2) * per <= have) np *= 2;
+    while (np < cap && (np * 2) * per <= have) np *= 2;
     return np;
 }
 

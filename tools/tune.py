@@ -40,9 +40,14 @@ elif os.environ.get("TUNE_SORT", "").startswith("hop2"):
     elif os.environ["TUNE_SORT"] == "hop3":
         hop3 = np.bincount(g.row_idx, weights=hop2[col], minlength=g.n)
         src = src[np.argsort(-hop3[src], kind="stable")]
-    elif os.environ["TUNE_SORT"] == "hop2log":  # coarse classes of log2 volume, degree within
-        cls = np.floor(np.log2(hop2[src] + 1) * 4)
+    elif os.environ["TUNE_SORT"].startswith("hop2log"):  # classes of log2 volume, degree within
+        gran = float(os.environ["TUNE_SORT"][7:] or 4)
+        cls = np.floor(np.log2(hop2[src] + 1) * gran)
         src = src[np.lexsort((-od[src], -cls))]
+    elif os.environ["TUNE_SORT"].startswith("degloghop"):  # classes of log2 degree, volume within
+        gran = float(os.environ["TUNE_SORT"][9:] or 4)
+        cls = np.floor(np.log2(od[src] + 1) * gran)
+        src = src[np.lexsort((-hop2[src], -cls))]
     else:  # hop2deg: out-degree, ties by 2-hop volume
         src = src[np.lexsort((-hop2[src], -od[src]))]
 G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed)

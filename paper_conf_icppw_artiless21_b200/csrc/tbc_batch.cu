@@ -1015,6 +1015,12 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
     if (np < 1) np = 1;
     for (int q = 0; q < np; ++q) {
         tbc_status st = batch_alloc(g, q, W);
+        if (st == TBC_ERR_OOM && q > 0) {  // run on the partitions that fit
+            batch_free_one(g, q);
+            (void)cudaGetLastError();
+            np = q;
+            break;
+        }
         if (st != TBC_OK) return st;
     }
     if (np > g->bgrid) np = g->bgrid;

@@ -61,7 +61,7 @@ for setting in a.settings.split(";"):
     G.set_bwd_direction(int(kv.get("bwd", 0)))
     G.set_partitions(int(kv.get("parts", 8)))
     G.set_batch(int(kv.get("batch", 1)))
-    G.set_batch_width(int(kv.get("width", 32)))
+    G.set_batch_width(int(kv.get("width", 0)))
     G.set_batch_pull(float(kv.get("bpull", 8)))
     G.set_batch_parts(int(kv.get("bparts", 0)))
     G.set_batch_order(int(kv.get("order", 1)))

@@ -296,6 +296,10 @@ def test_cfg3_kron22_directed_sample_in_bench_launch_config():
     g, src = gg.make_config(3, device="cuda")
     sample = src[:8]
     want = oracle.bc(g.col_ptr, g.row_idx, True, sample)
+    # the bench's launch configuration (auto width 64, grouped sources): 96 sources = 2 batches
+    many = src[:96]
+    with gpu_graph(g) as G:
+        assert_bc(G.bc(many), oracle.bc(g.col_ptr, g.row_idx, True, many))
     with gpu_graph(g, engine=tbc.ENGINE_COOT) as G:
         assert_bc(G.bc(sample[:3]), oracle.bc(g.col_ptr, g.row_idx, True, sample[:3]))
     with gpu_graph(g) as G:
@@ -358,6 +362,10 @@ def test_cfg5_kron25_full_size():
     with gpu_graph(g) as G:
         assert G.nnz == g.nnz
         assert_bfs(g, G, src[0])
+        # a source subset against the oracle, 40 = two batches (32 + a ragged 8) in
+        # the bench's launch configuration
+        sub = src[:40]
+        assert_bc(G.bc(sub), oracle.bc(g.col_ptr, g.row_idx, False, sub))
         for s in src[1:3]:
             depth, _ = G.bfs(int(s))
             got = G.bc([int(s)]).sum()

@@ -45,7 +45,14 @@ constexpr int kPad = 8;
 #ifndef TBC_BUNROLL
 #define TBC_BUNROLL 6
 #endif
-constexpr int kBU = TBC_BUNROLL;  // gathers in flight per lane in the slot loop
+#ifndef TBC_BUNROLL64
+#define TBC_BUNROLL64 8
+#endif
+// gathers in flight per lane in the slot loop, by batch width (A/B on B200: W = 32 best at 6 --
+// Kronecker 25: 394 vs 389 at 4, 373 at 8; W = 64 best at 8, i.e. 4 per source -- Kronecker 22:
+// 332 vs 318 at 6, RMAT 18: 359 vs 350)
+constexpr int kBU = TBC_BUNROLL;
+constexpr int kBU64 = TBC_BUNROLL64;
 
 enum { B_PUSH = 0, B_PULL = 1, B_BWD = 2 };
 
@@ -269,7 +276,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                                       const BOut &out) {
     using MT = typename MaskT<W>::T;
     constexpr int NS = W / 32;                 // sources per lane
-    constexpr int U2 = kBU / NS > 0 ? kBU / NS : 1;  // gathers in flight per lane and source
+    constexpr int U2 = (NS == 1 ? kBU : kBU64) / NS > 0 ? (NS == 1 ? kBU : kBU64) / NS : 1;  // gathers in flight per lane and source
     const MT *omsk = static_cast<const MT *>(omsk_);
     const MT *emsk = static_cast<const MT *>(emsk_);
     MT *fr_out = static_cast<MT *>(fr_out_);

@@ -282,7 +282,10 @@ def main():
     alg_bytes_per_launch = (8.0 * st["reached_edges"] + 80.0 * st["reached"]) / args.steps
     # the batched engine's own compulsory traffic: the index stream once per stage per BATCH of W
     # sources (8 B per reached edge / W per source) + the per-(vertex, source) state (80 B)
-    wdt = (args.width or (64 if g.n <= (8 << 20) else 32)) if batched else 1
+    # mirrors csrc/tbc_batch.cu batch_width (64 up to 8 M vertices, or average degree >= 8 when the
+    # W = 64 workspace fits the device; the library's exact rule uses the free memory at the call)
+    auto_w = 64 if (g.n <= (8 << 20) or (g.nnz >= 8 * g.n and 40.0 * 64 * g.n <= 0.85 * torch.cuda.get_device_properties(0).total_memory)) else 32
+    wdt = (args.width or auto_w) if batched else 1
     alg_bytes_batched = (8.0 * st["reached_edges"] / wdt + 80.0 * st["reached"]) / args.steps
     k_avg_s = statistics.mean(kern_ms) / 1e3
     peak, peak_kind = peaks()

@@ -911,11 +911,20 @@ void batch_free(tbc_graph *g) {
 }
 
 // auto width (measured with grouped sources): 64 sources per sweep up to 8 M
-// vertices (faster on RMAT 18, Kronecker 22 and the mycielski graphs), else 32 (faster on
-// Kronecker 25, and half the workspace of the 16 M-vertex lattice)
+// vertices (faster on RMAT 18, Kronecker 22 and the mycielski graphs) and above it for average
+// degree >= 8 while the W = 64 workspace fits 85 % of the free memory (Kronecker 25: 400 vs 389
+// GTEPS), else 32 (the 16 M-vertex lattice: 2.03 vs 1.91, at half the workspace)
 int batch_width(const tbc_graph *g) {
     if (g->batch_width) return g->batch_width;
-    return g->n <= (8ll << 20) ? 64 : 32;
+    const int64_t n = g->n, m = g->m;
+    if (n <= (8ll << 20)) return 64;
+    if (m < 8 * n) return 32;
+    const double need = 16.0 * 64 * n + 20.0 * 64 * n + 4.0 * 64 * (n + m) / kBT + 64.0 * n;  // rows, lists, tiles, rest
+    size_t fr = 0, tot = 0;
+    if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) return 32;
+    double have = 0.85 * (double)fr;
+    for (int q = 0; q < kMaxPartitions; ++q) have += g->bws[q].ready ? (double)g->bws[q].bytes : 0.0;
+    return need <= have ? 64 : 32;
 }
 
 // source grouping key of each source (one warp per source): its 2-hop out-volume V = sum of the

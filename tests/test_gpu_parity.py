@@ -362,9 +362,9 @@ def test_cfg5_kron25_full_size():
     with gpu_graph(g) as G:
         assert G.nnz == g.nnz
         assert_bfs(g, G, src[0])
-        # a source subset against the oracle, 40 = two batches (32 + a ragged 8) in
-        # the bench's launch configuration
-        sub = src[:40]
+        # a source subset against the oracle, 72 = two batches (64 + a ragged 8) in
+        # the bench's launch configuration (auto width 64 for Kronecker 25)
+        sub = src[:72]
         assert_bc(G.bc(sub), oracle.bc(g.col_ptr, g.row_idx, False, sub))
         for s in src[1:3]:
             depth, _ = G.bfs(int(s))

@@ -16,8 +16,9 @@ Kronecker: A,B,C,D = 0.57,0.19,0.19,0.05 (Graph500), seeded label permutation,
 self-loops and duplicates removed, undirected = symmetrised.
 Sources: the first k of a seeded permutation of the vertices with out-degree >= 1.
 
-Kronecker/ER generation runs in torch on whatever device is given (CUDA for the big
-configs; the RNG stream then differs from CPU, so m is recorded per generated graph).
+Kronecker generation runs in torch on whatever device is given (CUDA for the big configs)
+with a counter-based generator, so the host and the GPU produce the same graph bit for bit
+(the oracle caches of tests/golden/ are computed from host-generated graphs).
 """
 from __future__ import annotations
 
@@ -116,35 +117,90 @@ def erdos_renyi(n: int, m_edges: int, seed: int, directed: bool = False) -> Grap
     return Graph(f"er_n{n}_M{m_edges}_s{seed}", n, cp, ri, directed)
 
 
+def _s64(c: int) -> int:
+    """An unsigned 64-bit constant as the signed int64 torch stores."""
+    return c - (1 << 64) if c >= (1 << 63) else c
+
+
+_GOLDEN = _s64(0x9E3779B97F4A7C15)
+_MIX1 = _s64(0xBF58476D1CE4E5B9)
+_MIX2 = _s64(0x94D049BB133111EB)
+
+
+def _lsr(x, k: int):
+    """Logical right shift of an int64 tensor (torch's >> is arithmetic)."""
+    return (x >> k) & ((1 << (64 - k)) - 1)
+
+
+def mix64(x):
+    """splitmix64 finaliser of an int64 tensor, arithmetic mod 2^64 (two's complement wrap),
+    computed in place (x is consumed).  A counter-based generator: the same counters give the
+    same bits on CPU and CUDA, so a graph generated on the GPU is bit-identical to the one
+    generated on the host."""
+    y = x >> 30
+    y &= (1 << 34) - 1
+    x ^= y
+    x *= _MIX1
+    y = x >> 27
+    y &= (1 << 37) - 1
+    x ^= y
+    x *= _MIX2
+    y = x >> 31
+    y &= (1 << 33) - 1
+    x ^= y
+    return x
+
+
+def _stream_key(seed: int, stream: int) -> int:
+    """Key of an independent counter stream (a pure-Python splitmix64 of (seed, stream))."""
+    z = (seed * 0x9E3779B97F4A7C15 + stream * 0xD1B54A32D192ED03 + 0x632BE59BD9B4E019) % (1 << 64)
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) % (1 << 64)
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) % (1 << 64)
+    return _s64(z ^ (z >> 31))
+
+
 def kronecker(scale: int, edgefactor: int, seed: int, directed: bool, device: str = "cpu",
               abc=(0.57, 0.19, 0.19)) -> Graph:
     """Graph500 Kronecker/RMAT generator: edgefactor * 2^scale tuples, each bit of (src,dst)
-    drawn from the 2x2 initiator (A,B;C,D), then a seeded vertex-label permutation."""
+    drawn from the 2x2 initiator (A,B;C,D), then a seeded vertex-label permutation.
+
+    Randomness is counter-based (mix64 of (stream key + counter)): tuple t, bit b draws one
+    64-bit word whose high / low 32 bits are the two uniforms of that bit, and the label
+    permutation sorts the vertices by mix64 of (key + v).  Every step is integer or exact
+    fp64 arithmetic, so device="cpu" and device="cuda" give the same graph bit for bit."""
     if torch is None:
         raise RuntimeError("torch required for kronecker()")
     n = 1 << scale
     m_t = edgefactor * n
     a, b, c = abc
-    g = torch.Generator(device=device)
-    g.manual_seed(seed)
     src = torch.zeros(m_t, dtype=torch.int64, device=device)
     dst = torch.zeros(m_t, dtype=torch.int64, device=device)
     ab = a + b
     c_norm = c / (1.0 - ab)
     a_norm = a / ab
-    chunk = 1 << 26
+    key_bits = _stream_key(seed, 1)
+    key_perm = _stream_key(seed, 2)
+    # integer thresholds: bit i of the source is 1 iff the high 32-bit draw exceeds
+    # floor((A+B) 2^32), i.e. with probability C+D; bit j of the destination is 1 iff the low
+    # draw exceeds floor(C/(C+D) 2^32) when i = 1, floor(A/(A+B) 2^32) when i = 0
+    t_ab = int(ab * 4294967296.0)
+    t_c = int(c_norm * 4294967296.0)
+    t_a = int(a_norm * 4294967296.0)
+    chunk = 1 << 24
     for lo in range(0, m_t, chunk):
         hi = min(m_t, lo + chunk)
         s = src[lo:hi]
         d = dst[lo:hi]
+        ctr = torch.arange(lo, hi, dtype=torch.int64, device=device) * scale + key_bits
         for bit in range(scale):
-            r1 = torch.rand(hi - lo, generator=g, device=device)
-            r2 = torch.rand(hi - lo, generator=g, device=device)
-            ii = r1 > ab
-            jj = r2 > torch.where(ii, torch.full_like(r2, c_norm), torch.full_like(r2, a_norm))
+            h = mix64(ctr + bit)
+            ii = _lsr(h, 32) > t_ab
+            h &= 0xFFFFFFFF
+            jj = h > torch.where(ii, t_c, t_a)
             s |= ii.to(torch.int64) << bit
             d |= jj.to(torch.int64) << bit
-    perm = torch.randperm(n, generator=g, device=device)
+        del ctr
+    perm = torch.sort(mix64(torch.arange(n, dtype=torch.int64, device=device) + key_perm), stable=True).indices
     src = perm[src]
     dst = perm[dst]
     if device == "cpu":

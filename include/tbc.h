@@ -128,6 +128,12 @@ typedef struct {
     int64_t pull_levels; /* forward levels run as pull */
     int64_t scans;       /* candidate scans (first pull level of a source) */
     int64_t max_depth;   /* deepest BFS height seen */
+    int64_t list_peak;   /* batched engine: most level-list entries one batch used (sizing) */
+    int64_t bad_sources; /* tbc_bc_device: out-of-range entries of d_sources that were skipped */
+    int64_t batch_width; /* batched engine: sources per sweep of the latest call (0: none yet) */
+    int64_t batch_parts; /* batched engine: SM partitions of the latest call */
+    int64_t workspace_bytes; /* device bytes of the engine workspaces now allocated (included in
+                                tbc_graph_info's device_bytes); not reset by tbc_stats_reset */
 } tbc_stats;
 
 /* Create a graph from the CSC of A (CP_A = col_ptr, row_A = row_idx, here 0-based).
@@ -170,12 +176,25 @@ tbc_status tbc_bc(tbc_graph *g, const int32_t *sources, int64_t k, double *bc_ou
 tbc_status tbc_bc_device(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc,
                          void *cuda_stream);
 
-/* Forward stage only (Alg.1 l.11-28) from one source.
+/* Forward stage only (Alg.1 l.11-28) from one source, by the per-source engine.
  *   depth_out: host int32[n] or NULL; sigma_out: host double[n] or NULL.  Synchronous. */
 tbc_status tbc_bfs(tbc_graph *g, int32_t source, int32_t *depth_out, double *sigma_out);
 
+/* Forward stage of the batched engine -- the engine tbc_bc runs -- for a list of sources
+ * (Alg.1 l.11-28 for W sources per sweep, W as TBC_OPT_BATCH_WIDTH; sources are cut into sweeps
+ * in the given order, not grouped).
+ *   sources  : host int32[k], each in [0, n) (validated)
+ *   depth_out: host int32[k * n]; depth_out[i * n + v] = depth of v from sources[i] (0 at the
+ *              source, -1 unreachable)
+ *   sigma_out: host double[k * n]; sigma_out[i * n + v] = number of shortest paths (0 unreachable)
+ * Synchronous.  Device scratch of 12 k n bytes is kept for reuse until tbc_destroy.
+ * TBC_ERR_UNSUPPORTED for TBC_ENGINE_COOT graphs. */
+tbc_status tbc_bfs_batch(tbc_graph *g, const int32_t *sources, int64_t k, int32_t *depth_out,
+                         double *sigma_out);
+
 /* Graph properties after canonicalisation; any output pointer may be NULL.
- *   nnz = stored entries of A after deduplication; device_bytes = device memory owned. */
+ *   nnz = stored entries of A after deduplication; device_bytes = device memory owned now: the
+ *   graph arrays plus every engine workspace allocated so far (they are sized at the first call). */
 tbc_status tbc_graph_info(const tbc_graph *g, int64_t *n, int64_t *nnz, int *directed,
                           size_t *device_bytes);
 

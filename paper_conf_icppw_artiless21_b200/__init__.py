@@ -33,7 +33,7 @@ STATUS = {0: "TBC_OK", 1: "TBC_ERR_INVALID", 2: "TBC_ERR_OOM", 3: "TBC_ERR_CUDA"
 
 # every symbol include/tbc.h declares (checked by tests/test_abi.py)
 SYMBOLS = ["tbc_graph_create_csc", "tbc_graph_create_coo", "tbc_bc", "tbc_bc_device", "tbc_bfs",
-           "tbc_graph_info", "tbc_graph_set_option", "tbc_stats_get", "tbc_stats_reset", "tbc_trace_get",
+           "tbc_bfs_batch", "tbc_graph_info", "tbc_graph_set_option", "tbc_stats_get", "tbc_stats_reset", "tbc_trace_get",
            "tbc_profile_get", "tbc_destroy", "tbc_status_string", "tbc_last_error"]
 
 
@@ -45,7 +45,8 @@ class TBCError(RuntimeError):
 
 class Stats(ctypes.Structure):
     _fields_ = [(f, ctypes.c_int64) for f in
-                ("sources", "reached", "reached_edges", "fwd_edges", "bwd_edges", "levels", "pull_levels", "scans", "max_depth")]
+                ("sources", "reached", "reached_edges", "fwd_edges", "bwd_edges", "levels", "pull_levels", "scans",
+                 "max_depth", "list_peak", "bad_sources", "batch_width", "batch_parts", "workspace_bytes")]
 
     def as_dict(self):
         return {f: int(getattr(self, f)) for f, _ in self._fields_}
@@ -70,6 +71,7 @@ def lib():
         L.tbc_bc.argtypes = [vp, P(i32), i64, P(ctypes.c_double)]
         L.tbc_bc_device.argtypes = [vp, vp, i64, vp, vp]
         L.tbc_bfs.argtypes = [vp, i32, P(i32), P(ctypes.c_double)]
+        L.tbc_bfs_batch.argtypes = [vp, P(i32), i64, P(i32), P(ctypes.c_double)]
         L.tbc_graph_info.argtypes = [vp, P(i64), P(i64), P(ctypes.c_int), P(ctypes.c_size_t)]
         L.tbc_graph_set_option.argtypes = [vp, ctypes.c_int, ctypes.c_double]
         L.tbc_stats_get.argtypes = [vp, P(Stats)]
@@ -80,7 +82,7 @@ def lib():
         L.tbc_status_string.argtypes = [ctypes.c_int]
         L.tbc_status_string.restype = ctypes.c_char_p
         L.tbc_last_error.restype = ctypes.c_char_p
-        for name in SYMBOLS[:12]:
+        for name in SYMBOLS[:13]:
             getattr(L, name).restype = ctypes.c_int
         _LIB = L
     return _LIB
@@ -157,6 +159,22 @@ class Graph:
         _check(lib().tbc_bfs(self._h, int(source), _p(depth, ctypes.c_int32), _p(sigma, ctypes.c_double)))
         return depth, sigma
 
+    def bfs_batch(self, sources):
+        """tbc_bfs_batch: forward stage of the batched engine (the one tbc_bc runs) for a source list;
+        returns (depth int32[k, n], sigma float64[k, n]), row i for sources[i]."""
+        src = np.ascontiguousarray(sources, dtype=np.int32)
+        depth = np.empty((src.size, self.n), dtype=np.int32)
+        sigma = np.empty((src.size, self.n), dtype=np.float64)
+        _check(lib().tbc_bfs_batch(self._h, _p(src, ctypes.c_int32) if src.size else None, src.size,
+                                   _p(depth, ctypes.c_int32), _p(sigma, ctypes.c_double)))
+        return depth, sigma
+
+    def info(self) -> dict:
+        """tbc_graph_info now (device_bytes includes the engine workspaces allocated so far)."""
+        n, m, d, b = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int(), ctypes.c_size_t()
+        _check(lib().tbc_graph_info(self._h, ctypes.byref(n), ctypes.byref(m), ctypes.byref(d), ctypes.byref(b)))
+        return {"n": n.value, "nnz": m.value, "directed": bool(d.value), "device_bytes": b.value}
+
     def set_direction(self, mode: int):
         _check(lib().tbc_graph_set_option(self._h, OPT_DIRECTION, float(mode)))
 
@@ -165,11 +183,11 @@ class Graph:
         _check(lib().tbc_graph_set_option(self._h, OPT_BWD_DIRECTION, float(mode)))
 
     def set_batch(self, on: int):
-        """bc engine: 1 batched (32 sources per sweep, default), 0 per source (TBC_OPT_BATCH)."""
+        """bc engine: 1 batched (W = 32 or 64 sources per sweep, default), 0 per source (TBC_OPT_BATCH)."""
         _check(lib().tbc_graph_set_option(self._h, OPT_BATCH, float(on)))
 
     def set_batch_width(self, width: int):
-        """Batched engine: sources per sweep, 32 or 64 (TBC_OPT_BATCH_WIDTH)."""
+        """Batched engine: sources per sweep, 32 or 64, or 0 = auto (TBC_OPT_BATCH_WIDTH; tbc.h states the rule)."""
         _check(lib().tbc_graph_set_option(self._h, OPT_BATCH_WIDTH, float(width)))
 
     def set_batch_parts(self, parts: int):

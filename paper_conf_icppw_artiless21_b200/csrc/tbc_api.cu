@@ -3,6 +3,7 @@
 // options, statistics and error reporting.  Declarations and contracts: include/tbc.h.
 #include <cstdarg>
 #include <cstdio>
+#include <cstddef>
 #include <cstring>
 #include <vector>
 
@@ -188,6 +189,8 @@ void free_graph(tbc_graph *g) {
     cudaFree(g->in_col);
     if (g->out_row != g->in_col) cudaFree(g->out_row);
     engine_free(g);
+    cudaFree(g->bfs_depth);
+    cudaFree(g->bfs_sigma);
     cudaFree(g->bc_tmp);
     cudaFree(g->src_tmp);
     if (g->stream) cudaStreamDestroy(g->stream);
@@ -645,6 +648,50 @@ fail:
     return st;
 }
 
+tbc_status tbc_bfs_batch(tbc_graph *g, const int32_t *sources, int64_t k, int32_t *depth_out, double *sigma_out) {
+    g_err[0] = 0;
+    if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
+    if (k < 0) return set_error(TBC_ERR_INVALID, "k < 0");
+    if (k > 0 && (!sources || !depth_out || !sigma_out)) return set_error(TBC_ERR_INVALID, "NULL pointer");
+    if (g->engine != TBC_ENGINE_CSC) return set_error(TBC_ERR_UNSUPPORTED, "tbc_bfs_batch: CSC engine only");
+    for (int64_t i = 0; i < k; ++i)
+        if (sources[i] < 0 || sources[i] >= g->n)
+            return set_error(TBC_ERR_INVALID, "sources[%lld] = %d out of range", (long long)i, sources[i]);
+    if (k == 0) return TBC_OK;
+    if (k > (int64_t)((1ull << 62) / (uint64_t)g->n)) return set_error(TBC_ERR_INVALID, "k * n overflows");
+    tbc_status st = TBC_OK;
+    const int64_t kn = k * g->n;
+    TBC_CUDA(cudaSetDevice(g->device));
+    if (kn > g->bfs_cap) {
+        cudaFree(g->bfs_depth);
+        cudaFree(g->bfs_sigma);
+        g->bfs_depth = nullptr;
+        g->bfs_sigma = nullptr;
+        g->bfs_cap = 0;
+        TBC_CUDA(cudaMalloc(&g->bfs_depth, sizeof(int32_t) * kn));
+        TBC_CUDA(cudaMalloc(&g->bfs_sigma, sizeof(double) * kn));
+        g->bfs_cap = kn;
+    }
+    if (k > g->src_cap) {
+        cudaFree(g->src_tmp);
+        g->src_tmp = nullptr;
+        g->src_cap = 0;
+        TBC_CUDA(cudaMalloc(&g->src_tmp, sizeof(int32_t) * k));
+        g->src_cap = k;
+    }
+    TBC_CUDA(cudaMemsetAsync(g->bfs_depth, 0xff, sizeof(int32_t) * kn, g->stream));
+    TBC_CUDA(cudaMemsetAsync(g->bfs_sigma, 0, sizeof(double) * kn, g->stream));
+    TBC_CUDA(cudaMemcpyAsync(g->src_tmp, sources, sizeof(int32_t) * k, cudaMemcpyHostToDevice, g->stream));
+    st = batch_run(g, g->src_tmp, k, nullptr, g->stream, g->bfs_depth, g->bfs_sigma);
+    if (st != TBC_OK) return st;
+    TBC_CUDA(cudaMemcpyAsync(depth_out, g->bfs_depth, sizeof(int32_t) * kn, cudaMemcpyDeviceToHost, g->stream));
+    TBC_CUDA(cudaMemcpyAsync(sigma_out, g->bfs_sigma, sizeof(double) * kn, cudaMemcpyDeviceToHost, g->stream));
+    TBC_CUDA(cudaStreamSynchronize(g->stream));
+    return TBC_OK;
+fail:
+    return st;
+}
+
 tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
     if (!g || !out) return set_error(TBC_ERR_INVALID, "NULL pointer");
     tbc_status st = TBC_OK;
@@ -652,10 +699,16 @@ tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
     TBC_CUDA(cudaSetDevice(g->device));
     TBC_CUDA(cudaDeviceSynchronize());
     *out = tbc_stats{};
+    out->batch_width = g->last_width;
+    out->batch_parts = g->last_parts;
+    for (int q = 0; q < kMaxPartitions; ++q) out->workspace_bytes += (int64_t)g->bws[q].bytes;
+    out->workspace_bytes += (int64_t)g->ws_bytes;
     for (int i = 0; i < g->ws_count + kMaxPartitions; ++i) {  // per-source and batched partitions
         Ctrs *src = i < g->ws_count ? g->ws[i].ctr : g->bws[i - g->ws_count].ctr;
         if (!src) continue;
         TBC_CUDA(cudaMemcpy(&c, src, sizeof c, cudaMemcpyDeviceToHost));
+        out->bad_sources += (int64_t)c.bad_sources;
+        if (c.st_list_peak > out->list_peak) out->list_peak = c.st_list_peak;
         out->sources += c.st_sources;
         out->reached += c.st_reached;
         out->reached_edges += c.st_reached_edges;
@@ -709,15 +762,19 @@ fail:
 #endif
 }
 
+static constexpr size_t kStatBytes = offsetof(Ctrs, st_list_peak) + sizeof(long long) - offsetof(Ctrs, st_sources);
+
 tbc_status tbc_stats_reset(tbc_graph *g) {
     if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
     tbc_status st = TBC_OK;
     TBC_CUDA(cudaSetDevice(g->device));
     TBC_CUDA(cudaDeviceSynchronize());
-    for (int i = 0; i < g->ws_count; ++i)
-        TBC_CUDA(cudaMemset(&g->ws[i].ctr->st_sources, 0, sizeof(long long) * 9));
-    for (int q = 0; q < kMaxPartitions; ++q)
-        if (g->bws[q].ctr) TBC_CUDA(cudaMemset(&g->bws[q].ctr->st_sources, 0, sizeof(long long) * 9));
+    for (int i = 0; i < g->ws_count + kMaxPartitions; ++i) {
+        Ctrs *c = i < g->ws_count ? g->ws[i].ctr : g->bws[i - g->ws_count].ctr;
+        if (!c) continue;
+        TBC_CUDA(cudaMemset(&c->st_sources, 0, kStatBytes));  // st_sources .. st_list_peak
+        TBC_CUDA(cudaMemset(&c->bad_sources, 0, sizeof(unsigned long long)));
+    }
     return TBC_OK;
 fail:
     return st;

@@ -109,6 +109,10 @@ struct BParams {
     int ebits, dir_mode;
     int64_t *trace;  // per-phase timeline of batch trace_b (TBC_OPT_TRACE: source index / W)
     int64_t trace_cap, trace_b;
+    // tbc_bfs_batch: forward stage only; depth / sigma of source i (list order, caller labels)
+    // exported to bfs_depth[i n + v], bfs_sigma[i n + v] (pre-set to -1 / 0 by the host)
+    int32_t *bfs_depth;
+    double *bfs_sigma;
 };
 
 // one launch: a BParams per SM partition (its own workspace and counters/barrier); partition q
@@ -134,6 +138,12 @@ constexpr size_t kBSmem = sizeof(BWarpSmem) * kBWarps;
 struct Lv {
     int64_t p0, N, E, tb;
 };
+
+// list entries used by a batch whose deepest level is D (levels 0..D are concatenated)
+__device__ __forceinline__ int64_t nxt_p0_end(const BParams &P, int D) {
+    const int64_t *l = P.lvl + 4 * (int64_t)D;
+    return l[0] + l[1];
+}
 
 __device__ __forceinline__ int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
@@ -551,9 +561,12 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
 }
 
 // zero the (vertex, source) state of a level list's entries: sigma, delta_u, visited lanes and
-// the dense mask of its parity (atomicAnd: a concurrent scatter of another level may share the word)
-template <int W>
-__device__ __forceinline__ void bclear(const BParams &P, const Lv &l, void *fr_, int64_t gwarp, int64_t nwarps) {
+// the dense mask of its parity (atomicAnd: a concurrent scatter of another level may share the word).
+// EXPORT (tbc_bfs_batch): first write depth = level and sigma of every (vertex, lane) of the list to
+// the caller's [source][vertex] arrays (source index b W + lane word)
+template <int W, bool EXPORT = false>
+__device__ __forceinline__ void bclear(const BParams &P, const Lv &l, void *fr_, int64_t gwarp, int64_t nwarps,
+                                       int level = 0, int64_t b = 0) {
     using MT = typename MaskT<W>::T;
     constexpr int NS = W / 32;
     MT *fr = static_cast<MT *>(fr_);
@@ -577,8 +590,14 @@ __device__ __forceinline__ void bclear(const BParams &P, const Lv &l, void *fr_,
 #pragma unroll
             for (int k = 0; k < NS; ++k) {
                 if ((mq >> (32 * k + lane)) & 1u) {
-                    P.sig[(int64_t)vq * W + 32 * k + lane] = 0.0;
-                    P.du[(int64_t)vq * W + 32 * k + lane] = 0.0;
+                    const int64_t row = (int64_t)vq * W + 32 * k + lane;
+                    if (EXPORT) {
+                        const int64_t o = (b * W + 32 * k + lane) * P.n + (P.inv ? P.inv[vq] : vq);
+                        P.bfs_depth[o] = level;
+                        P.bfs_sigma[o] = P.sig[row];
+                    }
+                    P.sig[row] = 0.0;
+                    P.du[row] = 0.0;
                 }
             }
         }
@@ -795,6 +814,17 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             C->st_pull_levels += pulls;
             C->st_fwd_edges += fwd_edges;
             if (D > C->st_max_depth) C->st_max_depth = D;
+            const int64_t used = nxt_p0_end(P, D);
+            if (used > C->st_list_peak) C->st_list_peak = used;
+        }
+        if (P.bfs_depth) {  // tbc_bfs_batch: export depth / sigma level by level, retire, next batch
+            for (int L = 0; L <= D; ++L) {
+                const int64_t *l = P.lvl + 4 * (int64_t)L;
+                bclear<W, true>(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps, L, b);
+            }
+            if (cta0 && tid == 0) C->st_scans += pulls;
+            bsync(C, gen, ncta);
+            continue;
         }
         // ---------------- backward, L = D..1 (Alg.1 l.29-47); level L+2 retired on the way
         int64_t bwd_edges = 0;
@@ -868,6 +898,7 @@ static tbc_status batch_alloc(tbc_graph *g, int q, int W) {
         (e = alloc(&w.cand_v, n + kPad)) || (e = alloc(&w.cand_pre, n + kPad)) || (e = alloc(&w.cand_beg, n + kPad)) ||
         (e = alloc(&w.cand_tiles, w.cand_tiles_cap)) || (e = alloc(&w.lvl, 4 * (n + 2))) || (e = alloc(&w.ctr, 1))) {
         g->device_bytes += w.bytes;
+        batch_free_one(g, q);  // release the arrays that were allocated (no leak, device_bytes exact)
         return cuda_error(e, "batch workspace cudaMalloc");
     }
     g->device_bytes += w.bytes;
@@ -876,8 +907,10 @@ static tbc_status batch_alloc(tbc_graph *g, int q, int W) {
         (e = cudaMemsetAsync(w.vis, 0, sizeof(uint32_t) * n * nw, s)) ||
         (e = cudaMemsetAsync(w.fr[0], 0, sizeof(uint32_t) * n * nw, s)) ||
         (e = cudaMemsetAsync(w.fr[1], 0, sizeof(uint32_t) * n * nw, s)) ||
-        (e = cudaMemsetAsync(w.ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s)))
+        (e = cudaMemsetAsync(w.ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s))) {
+        batch_free_one(g, q);
         return cuda_error(e, "batch workspace init");
+    }
     if (!g->bgrid) {
         int per_sm = 0, sms = 0;
         for (const void *fn : {(const void *)k_bcb<32, false>, (const void *)k_bcb<64, false>,
@@ -913,18 +946,28 @@ void batch_free(tbc_graph *g) {
 // auto width (measured with grouped sources): 64 sources per sweep up to 8 M
 // vertices (faster on RMAT 18, Kronecker 22 and the mycielski graphs) and above it for average
 // degree >= 8 while the W = 64 workspace fits 85 % of the free memory (Kronecker 25: 400 vs 389
-// GTEPS), else 32 (the 16 M-vertex lattice: 2.03 vs 1.91, at half the workspace)
+// GTEPS), else 32 (the 16 M-vertex lattice: 2.03 vs 1.91, at half the workspace).  The choice is
+// made once per graph (a later change in free memory cannot flip it and reallocate), and falls
+// back to 32 if the W = 64 workspace then fails to allocate (batch_run).
+static int64_t batch_ws_bytes(const tbc_graph *g, int W) {  // batch_alloc's sizes, one partition
+    const int64_t n = g->n, m = g->m, nw = W / 32;
+    const int64_t list_cap = (int64_t)W * n + kPad;
+    const int64_t tiles_cap = ((int64_t)W * (n + m)) / kBT + n + 2 + kPad;
+    return 16 * W * n + 12 * n * nw + list_cap * (12 + 4 * nw) + 4 * tiles_cap + 16 * (n + kPad) +
+           4 * ((n + m) / kBT + 2 + kPad) + 32 * (n + 2) + (int64_t)sizeof(Ctrs);
+}
+
 int batch_width(const tbc_graph *g) {
     if (g->batch_width) return g->batch_width;
+    if (g->auto_width) return g->auto_width;
     const int64_t n = g->n, m = g->m;
     if (n <= (8ll << 20)) return 64;
     if (m < 8 * n) return 32;
-    const double need = 16.0 * 64 * n + 20.0 * 64 * n + 4.0 * 64 * (n + m) / kBT + 64.0 * n;  // rows, lists, tiles, rest
     size_t fr = 0, tot = 0;
     if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) return 32;
     double have = 0.85 * (double)fr;
     for (int q = 0; q < kMaxPartitions; ++q) have += g->bws[q].ready ? (double)g->bws[q].bytes : 0.0;
-    return need <= have ? 64 : 32;
+    return (double)batch_ws_bytes(g, 64) <= have ? 64 : 32;
 }
 
 // source grouping key of each source (one warp per source): its 2-hop out-volume V = sum of the
@@ -1007,7 +1050,7 @@ static int batch_auto_parts(tbc_graph *g, int W) {
     const int64_t n = g->n, m = g->m;
     if ((n * 32ll * 16 > (1ll << 30) && m >= 8 * n) || m >= 64 * n) return 1;
     const int cap = m >= 8 * n ? 4 : kMaxPartitions;  // RMAT 18: 4 beats 8; lattices: 8
-    const double per = 16.0 * W * n + 16.0 * W * n + 4.0 * W * (n + m) / kBT + 64.0 * n;  // rows, lists, tiles, rest
+    const double per = (double)batch_ws_bytes(g, W);
     size_t fr = 0, tot = 0;
     if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) return 1;
     double have = 0.8 * (double)fr;
@@ -1017,13 +1060,25 @@ static int batch_auto_parts(tbc_graph *g, int W) {
     return np;
 }
 
-tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream) {
-    const int W = batch_width(g);
+tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
+                     int32_t *bfs_depth, double *bfs_sigma) {
+    int W = batch_width(g);
     const int32_t *src = d_sources;
-    const bool grouped = g->batch_order && k > 1 && k < (1ll << 31);
+    // tbc_bfs_batch exports per list index: batches are cut from the list as given
+    const bool grouped = g->batch_order && k > 1 && k < (1ll << 31) && !bfs_depth;
     if (grouped) {
         tbc_status st = batch_group_sources(g, d_sources, k, stream, &src);
         if (st != TBC_OK) return st;
+    }
+    if (!g->batch_width && !g->auto_width) {  // settle the auto width once, with an OOM fallback
+        tbc_status st = batch_alloc(g, 0, W);
+        if (st == TBC_ERR_OOM && W == 64) {
+            (void)cudaGetLastError();
+            W = 32;
+            st = batch_alloc(g, 0, W);
+        }
+        if (st != TBC_OK) return st;
+        g->auto_width = W;
     }
     const int64_t nb = (k + W - 1) / W;
     int np = g->batch_parts ? g->batch_parts : batch_auto_parts(g, W);
@@ -1032,7 +1087,6 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
     for (int q = 0; q < np; ++q) {
         tbc_status st = batch_alloc(g, q, W);
         if (st == TBC_ERR_OOM && q > 0) {  // run on the partitions that fit
-            batch_free_one(g, q);
             (void)cudaGetLastError();
             np = q;
             break;
@@ -1088,7 +1142,11 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
         P.trace = g->trace;
         P.trace_cap = g->trace ? kTraceCap : 0;
         P.trace_b = g->trace_src >= 0 ? g->trace_src / W : -1;
+        P.bfs_depth = bfs_depth;
+        P.bfs_sigma = bfs_sigma;
     }
+    g->last_width = W;
+    g->last_parts = np;
     void *args[] = {&S};
     const void *fn = np > 1 ? (W == 64 ? (const void *)k_bcb<64, true> : (const void *)k_bcb<32, true>)
                             : (W == 64 ? (const void *)k_bcb<64, false> : (const void *)k_bcb<32, false>);

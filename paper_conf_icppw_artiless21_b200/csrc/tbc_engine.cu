@@ -1191,7 +1191,10 @@ tbc_status engine_workspaces(tbc_graph *g, int count) {
     auto alloc = [&](auto **p, size_t cnt) -> cudaError_t {
         size_t bytes = sizeof(**p) * (cnt > 0 ? cnt : 1);
         cudaError_t r = cudaMalloc((void **)p, bytes);
-        if (r == cudaSuccess) g->device_bytes += bytes;
+        if (r == cudaSuccess) {
+            g->device_bytes += bytes;
+            g->ws_bytes += bytes;
+        }
         return r;
     };
     const int64_t list_tiles = (n + m) / kWT + n + 2 + kListPad;
@@ -1252,6 +1255,8 @@ void engine_free(tbc_graph *g) {
         w = Workspace{};
     }
     g->ws_count = 0;
+    g->device_bytes -= g->ws_bytes;
+    g->ws_bytes = 0;
     batch_free(g);
     cudaFree(g->gctr);
     cudaFree(g->trace);

@@ -32,7 +32,7 @@ struct Ctrs {
     unsigned long long trace_n;   // entries written to the trace buffer
     // accumulated statistics (tbc_stats)
     long long st_sources, st_reached, st_reached_edges, st_fwd_edges, st_bwd_edges, st_levels, st_pull_levels,
-        st_scans, st_max_depth;
+        st_scans, st_max_depth, st_list_peak;
     unsigned long long prof[32];  // TBC_PROF builds: warp-cycles per code region (gctr only)
 };
 
@@ -168,6 +168,7 @@ struct tbc_graph {
     // workspaces (device), one per SM partition; ws_count allocated so far
     tbc::Workspace ws[tbc::kMaxPartitions];
     int ws_count = 0;
+    size_t ws_bytes = 0;          // device bytes of the per-source engine's workspaces
     int nparts = 8;               // TBC_OPT_PARTITIONS
     tbc::Ctrs *gctr = nullptr;    // shared counters: full-grid barrier, trace
     int64_t n_scan = 0, n_in = 0;
@@ -189,6 +190,11 @@ struct tbc_graph {
     int batch_order = 1;          // TBC_OPT_BATCH_ORDER: group the sources by out-degree into batches
     tbc::BatchOrder border;
     int bgrid = 0;
+    int auto_width = 0;           // batch width the auto rule settled on for this graph (0: not yet)
+    int last_width = 0, last_parts = 0;  // of the latest batched call (tbc_stats)
+    int32_t *bfs_depth = nullptr; // tbc_bfs_batch device outputs (grow-only)
+    double *bfs_sigma = nullptr;
+    int64_t bfs_cap = 0;          // elements of bfs_depth / bfs_sigma
     int64_t *trace = nullptr;     // device, 8 * kTraceCap int64
     int64_t trace_src = -1;       // index in the next call's source list to trace (-1: off)
     cudaStream_t stream = nullptr;  // internal stream for the synchronous host API
@@ -206,7 +212,8 @@ void engine_free(tbc_graph *g);                          // workspaces + shared 
 tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc,
                       cudaStream_t stream, int bfs_only);
 // batched engine (tbc_batch.cu)
-tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream);
+tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
+                     int32_t *bfs_depth = nullptr, double *bfs_sigma = nullptr);
 int batch_width(const tbc_graph *g);  // sources per sweep the next batched call uses
 void batch_free(tbc_graph *g);
 void batch_free_one(tbc_graph *g, int q);

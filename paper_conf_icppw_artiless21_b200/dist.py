@@ -33,7 +33,7 @@ def shard_sum(sources, compute_partial, group=None):
     world, rank = _world(group)
     lo, hi = partition(len(sources), world, rank)
     part = compute_partial(sources[lo:hi])
-    if world > 1:
+    if dist.is_available() and dist.is_initialized():  # also at world 1: the same collective path
         dist.all_reduce(part, op=dist.ReduceOp.SUM, group=group)
     return part
 

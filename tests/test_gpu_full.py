@@ -1,0 +1,214 @@
+"""Full-size parity of the engine the bench times, per-source depth/sigma of the batched engine,
+and the multi-GPU entry points with the real kernel.  Needs a B200.
+
+* Full source lists (configs 2-4, and the cached config-5 slice): the GPU runs tbc_bc over the
+  config's WHOLE list in the bench's launch configuration (default options: auto width, auto
+  partitions, sources grouped into batches); the result is compared with a fixture written by
+  tools/make_oracle_cache.py, which calls only graphgen and oracle/ on a HOST-generated graph.
+  The device regenerates the graph and must match the fixture's fingerprint first (graphgen's
+  counter-based generator).  Compared: bc at 2^16 seeded vertices + the 1024 largest (or every
+  vertex for n <= 2^20) to 1e-9 relative, the exact-zero mask (sha256), the zero count and fsum(bc).
+  PAPER.md P:332 (Sec. 4): only results verified against the sequential code are accepted.
+* tbc_bfs_batch: depth bit-exact, sigma bit-exact below 2^53 (relative 1e-12 above) for every
+  source of a sweep of the batched engine k_bcb (sigma is an output, Alg.1 l.2; depth S is
+  set at l.24).
+* dist.bc / dist.bc_device (north star (d)): world-1 NCCL group, and gloo world 2 with both ranks
+  on cuda:0, against the oracle.
+"""
+import hashlib
+import json
+import math
+import os
+import socket
+
+import numpy as np
+import pytest
+
+import graphgen as gg
+import oracle
+import paper_conf_icppw_artiless21_b200 as tbc
+from tbc_testutil import ROOT, assert_bc, assert_bfs_rows
+
+pytestmark = pytest.mark.gpu
+
+
+def _sha(a):
+    return hashlib.sha256(np.ascontiguousarray(a).tobytes()).hexdigest()
+
+
+def _fixture(name):
+    path = os.path.join(ROOT, "tests", "golden", name + ".npz")
+    if not os.path.exists(path):
+        pytest.skip(f"{name}.npz not generated (tools/make_oracle_cache.py)")
+    z = np.load(path)
+    return json.loads(str(z["meta"])), z
+
+
+# ------------------------------------------------------------------ generator determinism
+
+@pytest.mark.parametrize("directed", [False, True])
+def test_kronecker_generator_identical_on_host_and_device(directed):
+    a = gg.kronecker(14, 16, seed=7, directed=directed, device="cpu")
+    b = gg.kronecker(14, 16, seed=7, directed=directed, device="cuda")
+    np.testing.assert_array_equal(a.col_ptr, b.col_ptr)
+    np.testing.assert_array_equal(a.row_idx, b.row_idx)
+
+
+# ------------------------------------------------------------------ full source lists vs cached oracle
+
+def _check_full_list(cfg, name=None, k=None):
+    meta, z = _fixture(name or f"oracle_cfg{cfg}")
+    g, src = gg.make_config(cfg, device="cpu" if gg.CONFIGS[cfg]["kind"] != "kron" else "cuda")
+    src = src[: meta["k"]]
+    assert (g.n, g.nnz) == (meta["n"], meta["nnz"])
+    assert _sha(g.col_ptr.astype(np.int64)) == meta["col_ptr_sha"]
+    assert _sha(g.row_idx.astype(np.int32)) == meta["row_idx_sha"]
+    assert _sha(np.ascontiguousarray(src, dtype=np.int32)) == meta["src_sha"]
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:  # bench launch configuration
+        got = G.bc(src)
+        st = G.stats()
+    assert st["sources"] == meta["k"] and st["bad_sources"] == 0
+    zero = got == 0.0
+    assert _sha(np.packbits(zero)) == meta["zero_sha"], (int(zero.sum()), meta["nzero"])
+    assert abs(math.fsum(got.tolist()) - meta["fsum"]) <= 1e-9 * abs(meta["fsum"])
+    if "full" in z.files:
+        assert_bc(got, z["full"])
+    else:
+        assert_bc(got[z["sample_idx"]], z["sample_val"])
+        assert_bc(got[z["top_idx"]], z["top_val"])
+    return st
+
+
+def test_cfg2_full_source_list_cached_oracle():
+    _check_full_list(2)
+
+
+def test_cfg3_full_source_list_cached_oracle():
+    """The bench workload exactly: Kronecker 22 directed, all 4096 sources, 64 grouped sources per sweep."""
+    st = _check_full_list(3)
+    assert st["batch_width"] == 64
+
+
+def test_cfg4_full_source_list_cached_oracle():
+    _check_full_list(4)
+
+
+def test_cfg5_rank0_slice_cached_oracle():
+    """Config 5 (Kronecker 25, 1.05e9 entries): the first 1024 sources of its list -- the slice rank 0
+    runs when 8 GPUs share 8192 sources -- against the cached oracle."""
+    _check_full_list(5, name="oracle_cfg5_k1024")
+
+
+# ------------------------------------------------------------------ per-source depth / sigma of k_bcb
+
+SMALL = [gg.star(7), gg.path(7, directed=True), gg.cycle(9), gg.complete_bipartite(3, 5), gg.grid(6, 7),
+         gg.random_tree(50, 1), gg.mycielski(6), gg.from_edges("iso", 4, [(1, 2), (2, 3)], False)]
+
+
+@pytest.mark.parametrize("direction", [tbc.DIR_AUTO, tbc.DIR_PUSH, tbc.DIR_PULL])
+@pytest.mark.parametrize("width", [32, 64])
+@pytest.mark.parametrize("g", SMALL, ids=lambda g: g.name)
+def test_bfs_batch_small_all_sources(g, width, direction):
+    src = np.arange(g.n, dtype=np.int32)
+    src = np.concatenate([src, src[:3]]).astype(np.int32)  # repeats inside a sweep
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+        G.set_batch_width(width)
+        G.set_direction(direction)
+        depth, sigma = G.bfs_batch(src)
+    assert_bfs_rows(g, src, depth, sigma)
+
+
+@pytest.mark.parametrize("width", [0, 32, 64])
+@pytest.mark.parametrize("scale,directed", [(14, False), (15, True)])
+def test_bfs_batch_kronecker(scale, directed, width):
+    g = gg.kronecker(scale, 16, seed=2, directed=directed, device="cuda")
+    src = gg.sources(g, 70, seed=12)  # a full sweep of 64 and a ragged one (or 3 of 32)
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+        G.set_batch_width(width)
+        G.set_batch_parts(2)
+        depth, sigma = G.bfs_batch(src)
+        assert G.stats()["batch_parts"] == 2
+    assert_bfs_rows(g, src, depth, sigma)
+
+
+def test_bfs_batch_grid_sigma_crosses_2_53():
+    g = gg.grid(40, 40)
+    src = np.array([0, 820, 39, 1599], dtype=np.int32)
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+        for direction in (tbc.DIR_AUTO, tbc.DIR_PUSH, tbc.DIR_PULL):
+            G.set_direction(direction)
+            depth, sigma = G.bfs_batch(src)
+            assert sigma[0].max() > 2.0 ** 53
+            assert_bfs_rows(g, src, depth, sigma)
+
+
+@pytest.mark.parametrize("cfg", [2, 3])
+def test_bfs_batch_full_size_kronecker_sweep(cfg):
+    """One full sweep (64 sources, the auto width) of configs 2 and 3 at full size."""
+    g, src = gg.make_config(cfg, device="cuda")
+    src = src[:64]
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+        depth, sigma = G.bfs_batch(src)
+        assert G.stats()["batch_width"] == 64
+    assert_bfs_rows(g, src, depth, sigma)
+
+
+def test_bfs_batch_full_size_road_lattice():
+    g, src = gg.make_config(4)
+    src = src[:6]
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+        depth, sigma = G.bfs_batch(src)
+    assert depth.max() > 1000
+    assert_bfs_rows(g, src, depth, sigma)
+
+
+# ------------------------------------------------------------------ multi-GPU entry points, real kernel
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _dist_graph():
+    g = gg.kronecker(12, 16, seed=21, directed=True)
+    return g, gg.sources(g, 101, seed=3)
+
+
+def _dist_worker(rank, world, backend, port, out_dir):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_icppw_artiless21_b200 import dist as tdist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group(backend, rank=rank, world_size=world)
+    g, src = _dist_graph()
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, device=0) as G:
+        host = tdist.bc(G, src)                                          # host API
+        dev = tdist.bc_device(G, torch.from_numpy(src).cuda())          # device API
+        torch.cuda.synchronize()
+        st = G.stats()
+    np.save(os.path.join(out_dir, f"host_{rank}.npy"), host)
+    np.save(os.path.join(out_dir, f"dev_{rank}.npy"), dev.cpu().numpy())
+    np.save(os.path.join(out_dir, f"srcs_{rank}.npy"), np.array([st["sources"]]))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("backend,world", [("nccl", 1), ("gloo", 2)])
+def test_dist_bc_real_kernel(tmp_path, backend, world):
+    import torch.multiprocessing as mp
+    mp.spawn(_dist_worker, args=(world, backend, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    g, src = _dist_graph()
+    want = oracle.bc(g.col_ptr, g.row_idx, True, src)
+    per_rank = []
+    for r in range(world):
+        assert_bc(np.load(tmp_path / f"host_{r}.npy"), want)
+        assert_bc(np.load(tmp_path / f"dev_{r}.npy"), want)
+        per_rank.append(int(np.load(tmp_path / f"srcs_{r}.npy")[0]))
+    # each rank ran only its contiguous slice, twice (host and device API)
+    from paper_conf_icppw_artiless21_b200 import dist as tdist
+    assert per_rank == [2 * (hi - lo) for lo, hi in (tdist.partition(len(src), world, r) for r in range(world))]

@@ -10,6 +10,7 @@ import pytest
 import graphgen as gg
 import oracle
 import paper_conf_icppw_artiless21_b200 as tbc
+from tbc_testutil import assert_bc, assert_sigma
 
 pytestmark = pytest.mark.gpu
 
@@ -33,23 +34,11 @@ def set_mode(G, mode):
     G.set_batch_width(mode[4] if len(mode) > 4 else 32)
 
 
-def assert_bc(got, want, rel=1e-9):
-    got = np.asarray(got)
-    want = np.asarray(want)
-    zero = want == 0
-    assert np.all(got[zero] == 0.0), np.nonzero(got[zero])[0][:10]
-    err = np.abs(got[~zero] - want[~zero]) / np.abs(want[~zero])
-    assert err.size == 0 or err.max() <= rel, (err.max(), np.argmax(err))
-
-
 def assert_bfs(g, G, s):
     d_gpu, s_gpu = G.bfs(int(s))
     d_ora, s_ora = oracle.bfs(g.col_ptr, g.row_idx, int(s))
     np.testing.assert_array_equal(d_gpu, d_ora)
-    exact = s_ora < 2.0 ** 53
-    np.testing.assert_array_equal(s_gpu[exact], s_ora[exact])
-    if (~exact).any():
-        np.testing.assert_allclose(s_gpu[~exact], s_ora[~exact], rtol=1e-12)
+    assert_sigma(s_gpu, s_ora)
 
 
 def gpu_graph(g, **kw):

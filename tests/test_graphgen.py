@@ -29,8 +29,8 @@ def test_kronecker_deterministic_and_shaped():
     c = gg.kronecker(10, 16, seed=4, directed=True)
     assert np.array_equal(a.row_idx, b.row_idx) and np.array_equal(a.col_ptr, b.col_ptr)
     assert not np.array_equal(a.row_idx, c.row_idx)
-    # Graph500 shape: ~0.9-0.97 of the 16 * 2^10 tuples survive dedup, a skewed degree distribution
-    assert 0.85 * 16 * 1024 < a.nnz < 16 * 1024
+    # Graph500 shape: most of the 16 * 2^10 tuples survive dedup (0.73 at scale 10, 0.97 at 22), skewed degrees
+    assert 0.6 * 16 * 1024 < a.nnz < 16 * 1024
     deg = a.out_degree()
     assert deg.max() > 20 * deg.mean()
     u = gg.kronecker(10, 16, seed=3, directed=False)

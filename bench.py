@@ -49,7 +49,8 @@ def parse():
     ap.add_argument("--direction", type=int, default=0)
     ap.add_argument("--format", type=int, default=0, help="0 auto, 1 list passes, 2 edge streams")
     ap.add_argument("--engine", choices=["csc", "coot"], default="csc")
-    ap.add_argument("--batch", type=int, default=1, help="1: batched engine, 0: per source")
+    ap.add_argument("--batch", type=int, default=-1,
+                    help="engine: -1 auto (level-width probe), 0 per source, 1 batched, 2 narrow-level")
     ap.add_argument("--width", type=int, default=0, help="batched engine: sources per sweep (32, 64; 0 auto)")
     ap.add_argument("--order", type=int, default=1, help="batched engine: 1 group sources by 2-hop out-volume, 0 as given")
     ap.add_argument("--cost", default="", help="cost model overrides, e.g. list=10,stream=2")
@@ -228,8 +229,6 @@ def main():
     G.set_batch(args.batch)
     G.set_batch_width(args.width)
     G.set_batch_order(args.order)
-    batched = bool(args.batch) and args.engine == "csc"
-    kname = "k_bcb" if batched else "k_bc"
     if args.cost:
         G.set_cost(**{k: float(v) for k, v in (kv.split("=") for kv in args.cost.split(","))})
     src_d = torch.from_numpy(my_src).to(dev)
@@ -272,6 +271,9 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
     st = G.stats()
+    eng = st["engine"] if args.engine == "csc" else 0
+    batched = eng == 1
+    kname = {0: "k_bc", 1: "k_bcb", 2: "k_bcs"}[eng]
     sources_total = n_sources * args.steps
     gteps = sources_total * g.nnz / (total_ms / 1e3) / 1e9
     ms_per_step = total_ms / args.steps
@@ -284,8 +286,7 @@ def main():
     # sources (8 B per reached edge / W per source) + the per-(vertex, source) state (80 B)
     # mirrors csrc/tbc_batch.cu batch_width (64 up to 8 M vertices, or average degree >= 8 when the
     # W = 64 workspace fits the device; the library's exact rule uses the free memory at the call)
-    auto_w = 64 if (g.n <= (8 << 20) or (g.nnz >= 8 * g.n and 40.0 * 64 * g.n <= 0.85 * torch.cuda.get_device_properties(0).total_memory)) else 32
-    wdt = (args.width or auto_w) if batched else 1
+    wdt = st["batch_width"] if batched else 1
     alg_bytes_batched = (8.0 * st["reached_edges"] / wdt + 80.0 * st["reached"]) / args.steps
     k_avg_s = statistics.mean(kern_ms) / 1e3
     peak, peak_kind = peaks()
@@ -334,10 +335,13 @@ def main():
                        "l2": "inputs larger than L2 (CSC+CSR %.0f MB vs 126 MB L2); no flush" %
                              ((8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) / 1e6),
                        "direction": args.direction, "format": args.format, "engine_kind": args.engine,
-                       "engine_mode": f"batched, {wdt} sources per sweep"
-                       + (", sources grouped by 2-hop out-volume" if args.order else ", sources in the given order")
-                       if batched
+                       "engine_mode": (f"batched, {wdt} sources per sweep, {st['batch_parts']} SM partition(s)"
+                                       + (", sources grouped by 2-hop out-volume" if args.order
+                                          else ", sources in the given order")) if eng == 1
+                       else "narrow-level: one source per CTA, CTA barriers between levels" if eng == 2
                        else "per source, SM partitions",
+                       "engine_choice": "auto (level-width probe: %d vertices per level)" % st["probe_width"]
+                       if args.batch == -1 else f"forced {args.batch}",
                        "paper": PAPER_GTEPS[args.config][1] if args.config in PAPER_GTEPS else None,
                        "cost": args.cost},
             "clocks": clocks,
@@ -361,7 +365,8 @@ def main():
                           "pull_levels_per_source": st["pull_levels"] / max(st["sources"], 1),
                           "traversed_gteps": (st["reached_edges"] / args.steps) * world * args.steps
                           / (total_ms / 1e3) / 1e9},
-            "setup": {"generate_s": gen_s, "create_s": create_s, "device_bytes": G.device_bytes},
+            "setup": {"generate_s": gen_s, "create_s": create_s, "graph_bytes": G.device_bytes,
+                      "device_bytes": G.info()["device_bytes"], "workspace_bytes": st["workspace_bytes"]},
         }
         print(json.dumps(line), flush=True)
     if args.trace >= 0 and rank == 0:

@@ -91,11 +91,17 @@ enum {
                                 are summed in partition order at the end of the call (deterministic
                                 for a given value).  Costs one workspace (~50 B/vertex + 8 B/edge/64)
                                 per partition.  Per-source engine only. */
-    TBC_OPT_BATCH = 12,      /* bc engine: 1 (default) batched -- W sources per sweep (W = 32 or 64,
-                                TBC_OPT_BATCH_WIDTH), A^T times an n x W frontier block; 0 the
-                                per-source engine.  tbc_bfs and TBC_ENGINE_COOT always use the
-                                per-source engine.  The batched workspace holds 2 x 256 B/vertex of
-                                (sigma, delta_u) rows plus level lists of <= 32 entries per vertex. */
+    TBC_OPT_BATCH = 12,      /* bc engine (TBC_ENGINE_CSC graphs):
+                                -1 (default) auto: the first call with sources runs a level-width probe (a
+                                   forward BFS from its first source by one CTA, stopped after 65536
+                                   vertices; synchronises the stream once per graph) and picks 2 when
+                                   the probe's vertices per level < TBC_OPT_NARROW_WIDTH, else 1;
+                                 0 the per-source grid engine (k_bc);
+                                 1 batched -- W sources per sweep (W = 32 or 64, TBC_OPT_BATCH_WIDTH), A^T
+                                   times an n x W frontier block;
+                                 2 narrow-level -- one source per CTA, CTA barriers between levels, as
+                                   many sources at once as CTAs fit (20 B/vertex of workspace each).
+                                tbc_bfs and TBC_ENGINE_COOT always use the per-source engine. */
     TBC_OPT_BATCH_PULL = 13, /* batched engine: a forward level is pulled (candidates' in-edges)
                                 when the frontier's out-edges x this value > nnz, else pushed
                                 (default 8; must be >= 0) */
@@ -109,10 +115,12 @@ enum {
                                 fitting 80 % of free memory); partition q runs
                                 batches q, q + P, ... on its own SMs, workspace and barrier (one
                                 workspace each); bc accumulates with fp64 atomics from all of them */
-    TBC_OPT_BATCH_ORDER = 17 /* batched engine: 1 (default) cut the call's sources into batches after a
+    TBC_OPT_BATCH_ORDER = 17, /* batched engine: 1 (default) cut the call's sources into batches after a
                                 stable sort by 2-hop out-volume class, then out-degree (bc is a sum
                                 over sources, so only the floating-point summation order changes),
                                 0 in the given order */
+    TBC_OPT_NARROW_WIDTH = 18 /* auto engine: probe vertices per level below which the narrow-level
+                                engine runs (default 4096; setting it re-runs the probe next call) */
 };
 
 /* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since
@@ -134,6 +142,8 @@ typedef struct {
     int64_t batch_parts; /* batched engine: SM partitions of the latest call */
     int64_t workspace_bytes; /* device bytes of the engine workspaces now allocated (included in
                                 tbc_graph_info's device_bytes); not reset by tbc_stats_reset */
+    int64_t engine;      /* engine of the latest bc call: 0 per source, 1 batched, 2 narrow-level, -1 none */
+    int64_t probe_width; /* auto engine: the probe's vertices per level (0 before the probe) */
 } tbc_stats;
 
 /* Create a graph from the CSC of A (CP_A = col_ptr, row_A = row_idx, here 0-based).
@@ -180,15 +190,15 @@ tbc_status tbc_bc_device(tbc_graph *g, const int32_t *d_sources, int64_t k, doub
  *   depth_out: host int32[n] or NULL; sigma_out: host double[n] or NULL.  Synchronous. */
 tbc_status tbc_bfs(tbc_graph *g, int32_t source, int32_t *depth_out, double *sigma_out);
 
-/* Forward stage of the batched engine -- the engine tbc_bc runs -- for a list of sources
- * (Alg.1 l.11-28 for W sources per sweep, W as TBC_OPT_BATCH_WIDTH; sources are cut into sweeps
- * in the given order, not grouped).
+/* Forward stage (Alg.1 l.11-28) of the engine tbc_bc runs on this graph -- batched (W sources per
+ * sweep, W as TBC_OPT_BATCH_WIDTH; sources cut into sweeps in the given order, not grouped) or
+ * narrow-level (TBC_OPT_BATCH) -- for a list of sources.
  *   sources  : host int32[k], each in [0, n) (validated)
  *   depth_out: host int32[k * n]; depth_out[i * n + v] = depth of v from sources[i] (0 at the
  *              source, -1 unreachable)
  *   sigma_out: host double[k * n]; sigma_out[i * n + v] = number of shortest paths (0 unreachable)
  * Synchronous.  Device scratch of 12 k n bytes is kept for reuse until tbc_destroy.
- * TBC_ERR_UNSUPPORTED for TBC_ENGINE_COOT graphs. */
+ * TBC_ERR_UNSUPPORTED for TBC_ENGINE_COOT graphs and for TBC_OPT_BATCH = 0 (use tbc_bfs). */
 tbc_status tbc_bfs_batch(tbc_graph *g, const int32_t *sources, int64_t k, int32_t *depth_out,
                          double *sigma_out);
 

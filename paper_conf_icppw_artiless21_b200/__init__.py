@@ -26,6 +26,8 @@ ENGINE_CSC, ENGINE_COOT = 0, 1
 FLAG_ONE_FORMAT, FLAG_NO_VALIDATE, FLAG_NO_REORDER = 1, 2, 4
 OPT_DIRECTION, OPT_BWD_DIRECTION, OPT_TRACE, OPT_FORMAT, OPT_PARTITIONS = 1, 2, 3, 4, 11
 OPT_BATCH, OPT_BATCH_PULL, OPT_BATCH_WIDTH, OPT_BATCH_PARTS, OPT_BATCH_ORDER = 12, 13, 14, 16, 17
+OPT_NARROW_WIDTH = 18
+ENGINE_AUTO, ENGINE_PER_SOURCE, ENGINE_BATCHED, ENGINE_NARROW = -1, 0, 1, 2
 OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8, "scan": 9, "bpush": 10}
 FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
 DIR_AUTO, DIR_PUSH, DIR_PULL = 0, 1, 2
@@ -46,7 +48,8 @@ class TBCError(RuntimeError):
 class Stats(ctypes.Structure):
     _fields_ = [(f, ctypes.c_int64) for f in
                 ("sources", "reached", "reached_edges", "fwd_edges", "bwd_edges", "levels", "pull_levels", "scans",
-                 "max_depth", "list_peak", "bad_sources", "batch_width", "batch_parts", "workspace_bytes")]
+                 "max_depth", "list_peak", "bad_sources", "batch_width", "batch_parts", "workspace_bytes",
+                 "engine", "probe_width")]
 
     def as_dict(self):
         return {f: int(getattr(self, f)) for f, _ in self._fields_}
@@ -183,8 +186,13 @@ class Graph:
         _check(lib().tbc_graph_set_option(self._h, OPT_BWD_DIRECTION, float(mode)))
 
     def set_batch(self, on: int):
-        """bc engine: 1 batched (W = 32 or 64 sources per sweep, default), 0 per source (TBC_OPT_BATCH)."""
+        """bc engine (TBC_OPT_BATCH): -1 auto (default: level-width probe), 0 per source (grid),
+        1 batched (W = 32 or 64 sources per sweep), 2 narrow-level (one source per CTA)."""
         _check(lib().tbc_graph_set_option(self._h, OPT_BATCH, float(on)))
+
+    def set_narrow_width(self, width: float):
+        """Auto engine: probe vertices per level below which the narrow-level engine runs (TBC_OPT_NARROW_WIDTH)."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_NARROW_WIDTH, float(width)))
 
     def set_batch_width(self, width: int):
         """Batched engine: sources per sweep, 32 or 64, or 0 = auto (TBC_OPT_BATCH_WIDTH; tbc.h states the rule)."""

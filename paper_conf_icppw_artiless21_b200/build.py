@@ -11,7 +11,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libturbobc.so")
 LIB_DEBUG = os.path.join(PKG, "libturbobc_debug.so")  # -DTBC_DEBUG: device bounds checks
-SOURCES = ["tbc_api.cu", "tbc_engine.cu", "tbc_batch.cu"]
+SOURCES = ["tbc_api.cu", "tbc_engine.cu", "tbc_batch.cu", "tbc_single.cu"]
 HEADERS = ["tbc_internal.cuh", "tbc_device.cuh"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

@@ -530,8 +530,14 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
     }
     if (key == TBC_OPT_BATCH) {
         int v = (int)value;
-        if (v < 0 || v > 1 || (double)v != value) return set_error(TBC_ERR_INVALID, "batch %g", value);
+        if (v < -1 || v > 2 || (double)v != value) return set_error(TBC_ERR_INVALID, "engine %g not in [-1, 2]", value);
         g->batch = v;
+        return TBC_OK;
+    }
+    if (key == TBC_OPT_NARROW_WIDTH) {
+        if (!(value >= 0)) return set_error(TBC_ERR_INVALID, "narrow width %g", value);
+        g->narrow_width = value;
+        g->narrow = -1;  // decide again at the next call
         return TBC_OK;
     }
     if (key == TBC_OPT_BATCH_WIDTH) {
@@ -654,6 +660,7 @@ tbc_status tbc_bfs_batch(tbc_graph *g, const int32_t *sources, int64_t k, int32_
     if (k < 0) return set_error(TBC_ERR_INVALID, "k < 0");
     if (k > 0 && (!sources || !depth_out || !sigma_out)) return set_error(TBC_ERR_INVALID, "NULL pointer");
     if (g->engine != TBC_ENGINE_CSC) return set_error(TBC_ERR_UNSUPPORTED, "tbc_bfs_batch: CSC engine only");
+    if (g->batch == 0) return set_error(TBC_ERR_UNSUPPORTED, "tbc_bfs_batch: per-source engine selected (use tbc_bfs)");
     for (int64_t i = 0; i < k; ++i)
         if (sources[i] < 0 || sources[i] >= g->n)
             return set_error(TBC_ERR_INVALID, "sources[%lld] = %d out of range", (long long)i, sources[i]);
@@ -682,8 +689,14 @@ tbc_status tbc_bfs_batch(tbc_graph *g, const int32_t *sources, int64_t k, int32_
     TBC_CUDA(cudaMemsetAsync(g->bfs_depth, 0xff, sizeof(int32_t) * kn, g->stream));
     TBC_CUDA(cudaMemsetAsync(g->bfs_sigma, 0, sizeof(double) * kn, g->stream));
     TBC_CUDA(cudaMemcpyAsync(g->src_tmp, sources, sizeof(int32_t) * k, cudaMemcpyHostToDevice, g->stream));
-    st = batch_run(g, g->src_tmp, k, nullptr, g->stream, g->bfs_depth, g->bfs_sigma);
-    if (st != TBC_OK) return st;
+    {
+        int mode = 1;
+        st = engine_choose(g, g->src_tmp, k, g->stream, &mode);
+        if (st != TBC_OK) return st;
+        st = mode == 2 ? single_run(g, g->src_tmp, k, nullptr, g->stream, g->bfs_depth, g->bfs_sigma)
+                       : batch_run(g, g->src_tmp, k, nullptr, g->stream, g->bfs_depth, g->bfs_sigma);
+        if (st != TBC_OK) return st;
+    }
     TBC_CUDA(cudaMemcpyAsync(depth_out, g->bfs_depth, sizeof(int32_t) * kn, cudaMemcpyDeviceToHost, g->stream));
     TBC_CUDA(cudaMemcpyAsync(sigma_out, g->bfs_sigma, sizeof(double) * kn, cudaMemcpyDeviceToHost, g->stream));
     TBC_CUDA(cudaStreamSynchronize(g->stream));
@@ -701,10 +714,13 @@ tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
     *out = tbc_stats{};
     out->batch_width = g->last_width;
     out->batch_parts = g->last_parts;
+    out->engine = g->last_mode;
+    out->probe_width = (int64_t)g->probe_width;
     for (int q = 0; q < kMaxPartitions; ++q) out->workspace_bytes += (int64_t)g->bws[q].bytes;
-    out->workspace_bytes += (int64_t)g->ws_bytes;
-    for (int i = 0; i < g->ws_count + kMaxPartitions; ++i) {  // per-source and batched partitions
-        Ctrs *src = i < g->ws_count ? g->ws[i].ctr : g->bws[i - g->ws_count].ctr;
+    out->workspace_bytes += (int64_t)g->ws_bytes + (int64_t)g->sws.bytes;
+    for (int i = 0; i < g->ws_count + kMaxPartitions + 1; ++i) {  // per-source, batched, narrow-level
+        Ctrs *src = i < g->ws_count ? g->ws[i].ctr
+                    : i < g->ws_count + kMaxPartitions ? g->bws[i - g->ws_count].ctr : g->sws.ctr;
         if (!src) continue;
         TBC_CUDA(cudaMemcpy(&c, src, sizeof c, cudaMemcpyDeviceToHost));
         out->bad_sources += (int64_t)c.bad_sources;
@@ -769,8 +785,9 @@ tbc_status tbc_stats_reset(tbc_graph *g) {
     tbc_status st = TBC_OK;
     TBC_CUDA(cudaSetDevice(g->device));
     TBC_CUDA(cudaDeviceSynchronize());
-    for (int i = 0; i < g->ws_count + kMaxPartitions; ++i) {
-        Ctrs *c = i < g->ws_count ? g->ws[i].ctr : g->bws[i - g->ws_count].ctr;
+    for (int i = 0; i < g->ws_count + kMaxPartitions + 1; ++i) {
+        Ctrs *c = i < g->ws_count ? g->ws[i].ctr
+                  : i < g->ws_count + kMaxPartitions ? g->bws[i - g->ws_count].ctr : g->sws.ctr;
         if (!c) continue;
         TBC_CUDA(cudaMemset(&c->st_sources, 0, kStatBytes));  // st_sources .. st_list_peak
         TBC_CUDA(cudaMemset(&c->bad_sources, 0, sizeof(unsigned long long)));

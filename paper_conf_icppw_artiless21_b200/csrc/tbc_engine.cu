@@ -1258,6 +1258,7 @@ void engine_free(tbc_graph *g) {
     g->device_bytes -= g->ws_bytes;
     g->ws_bytes = 0;
     batch_free(g);
+    single_free(g);
     cudaFree(g->gctr);
     cudaFree(g->trace);
     g->gctr = nullptr;
@@ -1306,10 +1307,40 @@ tbc_status engine_setup(tbc_graph *g) {
     return TBC_OK;
 }
 
+// auto (TBC_OPT_BATCH = -1): the first call with sources probes the graph's level width once
+// (single_probe); graphs whose levels average fewer than TBC_OPT_NARROW_WIDTH vertices (road
+// networks, lattices, small graphs) run the narrow-level engine, the others the batched engine
+tbc_status engine_choose(tbc_graph *g, const int32_t *d_sources, int64_t k, cudaStream_t stream, int *mode) {
+    if (g->engine != TBC_ENGINE_CSC) {
+        *mode = g->last_mode = 0;
+        return TBC_OK;
+    }
+    if (g->batch >= 0) {
+        *mode = g->last_mode = g->batch;
+        return TBC_OK;
+    }
+    if (g->narrow < 0 && k > 0) {
+        double width = 0.0;
+        tbc_status st = single_probe(g, d_sources, stream, &width);
+        if (st != TBC_OK) return st;
+        g->narrow = width < g->narrow_width ? 1 : 0;
+        g->probe_width = width;
+    }
+    *mode = g->last_mode = g->narrow == 1 ? 2 : 1;
+    return TBC_OK;
+}
+
 tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
                       int bfs_only) {
-    // the batched engine (tbc_batch.cu) runs every bc call of the CSC engine unless TBC_OPT_BATCH = 0
-    if (!bfs_only && g->batch && g->engine == TBC_ENGINE_CSC) return batch_run(g, d_sources, k, d_bc, stream);
+    // bc calls of the CSC engine: batched (tbc_batch.cu) or narrow-level (tbc_single.cu) engine, or
+    // this file's per-source engine (TBC_OPT_BATCH, auto by default: engine_choose)
+    if (!bfs_only && g->engine == TBC_ENGINE_CSC) {
+        int mode = 0;
+        tbc_status st = engine_choose(g, d_sources, k, stream, &mode);
+        if (st != TBC_OK) return st;
+        if (mode == 1) return batch_run(g, d_sources, k, d_bc, stream);
+        if (mode == 2) return single_run(g, d_sources, k, d_bc, stream);
+    }
     // SM partitions: never more than the sources (a partition without sources only waits)
     int np = g->nparts;
     if (bfs_only || k < 1) np = 1;

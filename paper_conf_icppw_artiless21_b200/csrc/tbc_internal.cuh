@@ -147,6 +147,18 @@ struct BatchWorkspace {
     int64_t list_cap = 0, tiles_cap = 0, cand_tiles_cap = 0;
     bool ready = false;
 };
+// workspace of the narrow-level engine (tbc_single.cu): one slot of per-vertex arrays per
+// concurrently running source (one per resident CTA)
+struct SingleWorkspace {
+    int slots = 0;
+    size_t bytes = 0;
+    int32_t *depth = nullptr;    // [slots][n]
+    double *sd = nullptr;        // [slots][n] sigma, then delta_u
+    int32_t *order = nullptr;    // [slots][n]
+    int32_t *lvl = nullptr;      // [slots][n + 2]
+    Ctrs *ctr = nullptr;
+    int64_t *probe_out = nullptr;
+};
 }  // namespace tbc
 
 struct tbc_graph {
@@ -182,7 +194,12 @@ struct tbc_graph {
     int bwd_mode = 0;
     int fmt_mode = 0;
     double c_list = 12.0, c_stream = 4.0, c_atom = 18.0, c_vert = 10.0, c_scan = 3.0, c_bpush = 6.0;
-    int batch = 1;                // TBC_OPT_BATCH: 1 batched engine, 0 per source
+    int batch = -1;               // TBC_OPT_BATCH: -1 auto, 0 per source, 1 batched, 2 narrow-level
+    int narrow = -1;              // auto choice, settled by the first call's probe: 1 narrow-level engine
+    double narrow_width = 4096.0; // TBC_OPT_NARROW_WIDTH: probe's vertices per level below which auto is narrow
+    double probe_width = 0.0;     // the probe's measured vertices per level (tbc_stats)
+    int last_mode = -1;           // engine of the latest bc call (0 per source, 1 batched, 2 narrow-level)
+    tbc::SingleWorkspace sws;
     int batch_width = 0;          // TBC_OPT_BATCH_WIDTH: sources per sweep (32 or 64; 0 auto)
     double batch_pull = 8.0;      // TBC_OPT_BATCH_PULL: pull when frontier out-edges x this > m
     tbc::BatchWorkspace bws[tbc::kMaxPartitions];  // one per SM partition of the batched engine
@@ -215,6 +232,14 @@ tbc_status engine_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
 tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
                      int32_t *bfs_depth = nullptr, double *bfs_sigma = nullptr);
 int batch_width(const tbc_graph *g);  // sources per sweep the next batched call uses
+// narrow-level engine (tbc_single.cu)
+tbc_status single_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
+                      int32_t *bfs_depth = nullptr, double *bfs_sigma = nullptr);
+tbc_status single_probe(tbc_graph *g, const int32_t *d_sources, cudaStream_t stream, double *width);
+void single_free(tbc_graph *g);
+// engine the next bc call on these sources runs (auto: probes once per graph): 0 per source,
+// 1 batched, 2 narrow-level
+tbc_status engine_choose(tbc_graph *g, const int32_t *d_sources, int64_t k, cudaStream_t stream, int *mode);
 void batch_free(tbc_graph *g);
 void batch_free_one(tbc_graph *g, int q);
 }  // namespace tbc

@@ -1,0 +1,376 @@
+// tbc_single.cu -- the narrow-level engine: Algorithm 1 of PAPER.md for ONE source per
+// CTA, many sources side by side (one per resident CTA), every level separated by a CTA barrier
+// (__syncthreads) instead of a grid barrier.
+//
+// Why: on high-diameter graphs (road networks, lattices: thousands of levels of a
+// few thousand vertices) the grid-wide engines pay a grid barrier and several dependent memory round
+// trips per level for a level that only a handful of SMs' worth of threads can use; the paper's own
+// runs on such graphs are its slowest (luxembourg-osm, d = 1035: 5 MTEPs).  Here a level of
+// w vertices costs ceil(w / 512) rounds of a few dependent loads inside one SM, and 148+ sources
+// progress concurrently, so the whole GPU streams memory while each source walks its levels.
+//
+// Per source (Alg.1 with R1-R5 of DESIGN.md):
+//   forward level d -> d+1 (l.19-27): every frontier vertex u (BFS order list, level offsets lvl)
+//     pushes sigma(u) along its out-edges: depth(w) is claimed with atomicCAS(-1 -> d+1) (the
+//     claimer appends w to the order list) and sigma(w) += sigma(u) (fp64 atomic) iff depth(w) = d+1
+//     -- the masked SpMV f_t = A^T f restricted to the unvisited vertices (l.19-25).
+//   backward level L = D..1 (l.29-47): every v on level L pulls acc = sum of delta_u(w) over its
+//     out-edges with depth(w) = L+1 (A delta_u, R1), adds scale * sigma(v) * acc to bc (l.39, l.45,
+//     1/2 if undirected P:180) and overwrites sigma(v) with delta_u(v) = 1/sigma(v) + acc (l.35):
+//     in place, because a vertex has one level and its sigma is read only by its own update.
+//   level L+2 is reset (depth -1, sigma 0) during level L, levels 0..2 at the end: a CTA's arrays
+//   are all-unvisited between sources, with no O(n) clear.
+// Out-degrees above kHeavy are deferred to a per-level shared-memory queue and run by a whole warp.
+#include <cstdio>
+
+#include "tbc_internal.cuh"
+#include "tbc_device.cuh"
+
+namespace tbc {
+namespace {
+
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int kSB = 512;            // threads per CTA
+constexpr int kSWarps = kSB / 32;
+constexpr int kHeavy = 32;          // out-degree above which a whole warp handles the vertex
+constexpr int kHeavyCap = 2048;     // heavy vertices queued per level (overflow: handled by one thread)
+
+struct SParams {
+    int64_t n;
+    const int64_t *__restrict__ out_ptr;  // CSR of A (== the CSC when undirected)
+    const int32_t *__restrict__ out_idx;
+    int32_t *depth;   // [slots][n], -1 between sources
+    double *sd;       // [slots][n], sigma (forward) then delta_u (backward); 0 between sources
+    int32_t *order;   // [slots][n], BFS order, levels concatenated
+    int32_t *lvl;     // [slots][n + 2], level offsets into order
+    Ctrs *ctr;
+    double *bc;       // caller labels, accumulated (fp64 atomics: the CTAs share it)
+    const int32_t *sources;  // caller labels
+    const int32_t *__restrict__ perm;  // caller -> internal label (nullptr: identity)
+    const int32_t *__restrict__ inv;   // internal -> caller label
+    int64_t k;
+    double bc_scale;
+    int32_t *bfs_depth;  // tbc_bfs_batch: forward only, export [source index][caller label]
+    double *bfs_sigma;
+    int64_t probe_cap;   // > 0: probe run (one source, forward only, stop after ~probe_cap vertices)
+    int64_t *probe_out;  // {levels completed, vertices discovered}
+};
+
+// relax the out-edge u -> w of frontier level d: claim w for level d+1, add sigma(u)
+__device__ __forceinline__ void relax(const SParams &P, int32_t *depth, double *sd, int32_t *order, int32_t w,
+                                      int d, double su, int *cnt, int end) {
+    int dw = __ldcg(depth + w);
+    if (dw == -1) {
+        dw = atomicCAS(depth + w, -1, d + 1);
+        if (dw == -1) {
+            order[end + atomicAdd(cnt, 1)] = w;
+            dw = d + 1;
+        }
+    }
+    if (dw == d + 1) atomicAdd(sd + w, su);
+}
+
+// Alg.1 l.35-45 for v with acc = sum of delta_u over its level-(L+1) out-neighbours
+__device__ __forceinline__ void finish(const SParams &P, double *sd, int32_t v, double acc) {
+    const double sv = __ldcg(sd + v);
+    const double delta = sv * acc;
+    if (delta != 0.0) atomicAdd(P.bc + (P.inv ? P.inv[v] : v), delta * P.bc_scale);
+    sd[v] = 1.0 / sv + acc;
+}
+
+__device__ __forceinline__ void reset_level(int32_t *depth, double *sd, const int32_t *order, int b0, int b1) {
+    for (int i = b0 + (int)threadIdx.x; i < b1; i += kSB) {
+        const int32_t x = order[i];
+        depth[x] = -1;
+        sd[x] = 0.0;
+    }
+}
+
+__global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int64_t n = P.n;
+    const int64_t slot = blockIdx.x;
+    int32_t *depth = P.depth + slot * n;
+    double *sd = P.sd + slot * n;
+    int32_t *order = P.order + slot * n;
+    int32_t *lvl = P.lvl + slot * (n + 2);
+    __shared__ int s_cnt[2], s_hcnt[2];
+    __shared__ int32_t s_heavy[kHeavyCap];
+    __shared__ unsigned long long s_edges[2];
+    for (int64_t si = blockIdx.x; si < P.k; si += gridDim.x) {
+        int32_t s = P.sources[si];
+        if (s < 0 || s >= n) {  // skipped and counted (tbc_bc_device does not validate on the host)
+            if (tid == 0) atomicAdd(&P.ctr->bad_sources, 1ull);
+            continue;
+        }
+        if (P.perm) s = P.perm[s];
+        if (tid == 0) {  // level 0 (Alg.1 l.15-18)
+            depth[s] = 0;
+            sd[s] = 1.0;
+            order[0] = s;
+            lvl[0] = 0;
+            lvl[1] = 1;
+            s_cnt[0] = s_cnt[1] = 0;
+            s_hcnt[0] = s_hcnt[1] = 0;
+            s_edges[0] = s_edges[1] = 0;
+        }
+        __syncthreads();
+        // ---------------- forward (Alg.1 l.11-28)
+        int d = 0, beg = 0, end = 1;
+        unsigned long long my_edges = 0;
+        bool probe_stop = false;
+        for (;;) {
+            const int par = d & 1;
+            for (int i = beg + tid; i < end; i += kSB) {
+                if (P.probe_cap > 0 && end + *(volatile int *)&s_cnt[par] > P.probe_cap) break;
+                const int32_t u = order[i];
+                const int64_t e0 = P.out_ptr[u], e1 = P.out_ptr[u + 1];
+                my_edges += (unsigned long long)(e1 - e0);
+                if (e1 - e0 > kHeavy) {
+                    const int h = atomicAdd(&s_hcnt[par], 1);
+                    if (h < kHeavyCap) {
+                        s_heavy[h] = u;
+                        continue;
+                    }
+                }
+                const double su = __ldcg(sd + u);
+                for (int64_t e = e0; e < e1; ++e) relax(P, depth, sd, order, P.out_idx[e], d, su, &s_cnt[par], end);
+            }
+            __syncthreads();
+            if (tid == 0) {  // counters of level d+2 (their level-d readers are past the barrier)
+                s_cnt[par ^ 1] = 0;
+                s_hcnt[par ^ 1] = 0;
+            }
+            const int nh = min(s_hcnt[par], kHeavyCap);
+            for (int h = warp; h < nh; h += kSWarps) {
+                const int32_t u = s_heavy[h];
+                const double su = __ldcg(sd + u);
+                const int64_t e1 = P.out_ptr[u + 1];
+                for (int64_t e = P.out_ptr[u] + lane; e < e1; e += 32)
+                    relax(P, depth, sd, order, P.out_idx[e], d, su, &s_cnt[par], end);
+            }
+            __syncthreads();
+            const int nn = s_cnt[par];
+            if (P.probe_cap > 0 && end + nn > P.probe_cap) {
+                probe_stop = true;
+                end += nn;  // every claimed vertex is in the list (reset below)
+                break;
+            }
+            if (nn == 0) break;
+            beg = end;
+            end += nn;
+            ++d;
+            if (tid == 0) lvl[d + 1] = end;
+        }
+        const int D = d;  // deepest non-empty level
+        atomicAdd(&s_edges[0], my_edges);
+        if (tid == 0) s_hcnt[0] = s_hcnt[1] = 0;  // their forward readers are past the last barrier
+        __syncthreads();
+        if (P.probe_cap > 0) {  // probe: report, reset every listed vertex, done
+            if (tid == 0) {
+                P.probe_out[0] = D + 1;  // levels whose expansion ran
+                P.probe_out[1] = end;    // vertices discovered
+                P.probe_out[2] = probe_stop ? 0 : 1;
+            }
+            reset_level(depth, sd, order, 0, end);
+            __syncthreads();
+            return;
+        }
+        if (tid == 0) {
+            atomicAdd((unsigned long long *)&P.ctr->st_sources, 1ull);
+            atomicAdd((unsigned long long *)&P.ctr->st_reached, (unsigned long long)end);
+            atomicAdd((unsigned long long *)&P.ctr->st_reached_edges, s_edges[0]);
+            atomicAdd((unsigned long long *)&P.ctr->st_fwd_edges, s_edges[0]);
+            atomicAdd((unsigned long long *)&P.ctr->st_levels, (unsigned long long)(D + 2));
+            atomicMax((unsigned long long *)&P.ctr->st_max_depth, (unsigned long long)D);
+        }
+        if (P.bfs_depth) {  // tbc_bfs_batch: export depth / sigma, reset, next source
+            for (int L = 0; L <= D; ++L) {
+                const int b0 = lvl[L], b1 = lvl[L + 1];
+                for (int i = b0 + tid; i < b1; i += kSB) {
+                    const int32_t x = order[i];
+                    const int64_t o = si * n + (P.inv ? P.inv[x] : x);
+                    P.bfs_depth[o] = L;
+                    P.bfs_sigma[o] = __ldcg(sd + x);
+                }
+            }
+            __syncthreads();
+            reset_level(depth, sd, order, 0, end);
+            if (tid == 0) s_edges[0] = 0;
+            __syncthreads();
+            continue;
+        }
+        // ---------------- backward, L = D..1 (Alg.1 l.29-47)
+        unsigned long long my_bwd = 0;
+        for (int L = D; L >= 1; --L) {
+            const int par = L & 1;
+            const int b0 = lvl[L], b1 = lvl[L + 1];
+            for (int i = b0 + tid; i < b1; i += kSB) {
+                const int32_t v = order[i];
+                const int64_t e0 = P.out_ptr[v], e1 = P.out_ptr[v + 1];
+                my_bwd += (unsigned long long)(e1 - e0);
+                if (e1 - e0 > kHeavy) {
+                    const int h = atomicAdd(&s_hcnt[par], 1);
+                    if (h < kHeavyCap) {
+                        s_heavy[h] = v;
+                        continue;
+                    }
+                }
+                double acc = 0.0;
+                for (int64_t e = e0; e < e1; ++e) {
+                    const int32_t w = P.out_idx[e];
+                    if (__ldcg(depth + w) == L + 1) acc += __ldcg(sd + w);
+                }
+                finish(P, sd, v, acc);
+            }
+            if (L + 2 <= D) reset_level(depth, sd, order, lvl[L + 2], lvl[L + 3]);
+            __syncthreads();
+            if (tid == 0) s_hcnt[par ^ 1] = 0;
+            const int nh = min(s_hcnt[par], kHeavyCap);
+            for (int h = warp; h < nh; h += kSWarps) {
+                const int32_t v = s_heavy[h];
+                const int64_t e1 = P.out_ptr[v + 1];
+                double acc = 0.0;
+                for (int64_t e = P.out_ptr[v] + lane; e < e1; e += 32) {
+                    const int32_t w = P.out_idx[e];
+                    if (__ldcg(depth + w) == L + 1) acc += __ldcg(sd + w);
+                }
+#pragma unroll
+                for (int o = 16; o >= 1; o >>= 1) acc += __shfl_xor_sync(FULL, acc, o);
+                if (lane == 0) finish(P, sd, v, acc);
+            }
+            __syncthreads();
+        }
+        reset_level(depth, sd, order, 0, lvl[min(D, 2) + 1]);
+        atomicAdd(&s_edges[1], my_bwd);
+        __syncthreads();
+        if (tid == 0) {
+            atomicAdd((unsigned long long *)&P.ctr->st_bwd_edges, s_edges[1]);
+            s_edges[0] = s_edges[1] = 0;
+            s_hcnt[0] = s_hcnt[1] = 0;
+        }
+        __syncthreads();
+    }
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ host side
+
+static int64_t single_slot_bytes(const tbc_graph *g) { return 20 * g->n + 8; }
+
+void single_free(tbc_graph *g) {
+    SingleWorkspace &w = g->sws;
+    cudaFree(w.depth);
+    cudaFree(w.sd);
+    cudaFree(w.order);
+    cudaFree(w.lvl);
+    cudaFree(w.ctr);
+    cudaFree(w.probe_out);
+    g->device_bytes -= w.bytes;
+    w = SingleWorkspace{};
+}
+
+// one slot (a CTA's arrays) per concurrently running source: as many as the GPU keeps resident,
+// within 80 % of the free memory (at least one); sized once per graph
+static tbc_status single_alloc(tbc_graph *g) {
+    SingleWorkspace &w = g->sws;
+    if (w.slots > 0) return TBC_OK;
+    cudaError_t e = cudaSuccess;
+    int per_sm = 0, sms = 0;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_bcs, kSB, 0)) ||
+        (e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device)))
+        return cuda_error(e, "k_bcs occupancy query");
+    if (per_sm < 1) return set_error(TBC_ERR_CUDA, "k_bcs cannot be resident");
+    size_t fr = 0, tot = 0;
+    if ((e = cudaMemGetInfo(&fr, &tot))) return cuda_error(e, "cudaMemGetInfo");
+    int64_t slots = (int64_t)per_sm * sms;
+    const int64_t fit = (int64_t)(0.8 * (double)fr / (double)single_slot_bytes(g));
+    if (slots > fit) slots = fit;
+    if (slots < 1) slots = 1;
+    const int64_t n = g->n;
+    auto alloc = [&](auto **p, size_t cnt) -> cudaError_t {
+        const size_t bytes = sizeof(**p) * (cnt > 0 ? cnt : 1);
+        cudaError_t r = cudaMalloc((void **)p, bytes);
+        if (r == cudaSuccess) {
+            w.bytes += bytes;
+            g->device_bytes += bytes;
+        }
+        return r;
+    };
+    if ((e = alloc(&w.depth, slots * n)) || (e = alloc(&w.sd, slots * n)) || (e = alloc(&w.order, slots * n)) ||
+        (e = alloc(&w.lvl, slots * (n + 2))) || (e = alloc(&w.ctr, 1)) || (e = alloc(&w.probe_out, 4))) {
+        single_free(g);
+        return cuda_error(e, "narrow-level engine workspace cudaMalloc");
+    }
+    cudaStream_t s = g->stream;
+    if ((e = cudaMemsetAsync(w.depth, 0xff, sizeof(int32_t) * slots * n, s)) ||
+        (e = cudaMemsetAsync(w.sd, 0, sizeof(double) * slots * n, s)) ||
+        (e = cudaMemsetAsync(w.ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s))) {
+        single_free(g);
+        return cuda_error(e, "narrow-level engine workspace init");
+    }
+    w.slots = (int)slots;
+    return TBC_OK;
+}
+
+static SParams single_params(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc) {
+    const SingleWorkspace &w = g->sws;
+    SParams P{};
+    P.n = g->n;
+    P.out_ptr = g->out_ptr;
+    P.out_idx = g->out_idx;
+    P.depth = w.depth;
+    P.sd = w.sd;
+    P.order = w.order;
+    P.lvl = w.lvl;
+    P.ctr = w.ctr;
+    P.bc = d_bc;
+    P.sources = d_sources;
+    P.perm = g->perm;
+    P.inv = g->inv;
+    P.k = k;
+    P.bc_scale = g->directed ? 1.0 : 0.5;
+    P.probe_out = w.probe_out;
+    return P;
+}
+
+tbc_status single_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
+                      int32_t *bfs_depth, double *bfs_sigma) {
+    if (!g->out_ptr) return set_error(TBC_ERR_UNSUPPORTED, "narrow-level engine needs the out-edge format");
+    tbc_status st = single_alloc(g);
+    if (st != TBC_OK) return st;
+    SParams P = single_params(g, d_sources, k, d_bc);
+    P.bfs_depth = bfs_depth;
+    P.bfs_sigma = bfs_sigma;
+    const int grid = (int)(k < g->sws.slots ? k : g->sws.slots);
+    if (grid < 1) return TBC_OK;
+    k_bcs<<<grid, kSB, 0, stream>>>(P);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_error(e, "k_bcs launch");
+    return TBC_OK;
+}
+
+// Level-width probe (auto engine choice): a forward BFS from the call's first source
+// by one CTA, stopped once it has discovered kProbeCap vertices; returns the average number of
+// vertices per level seen so far (a narrow, deep graph stays far below the threshold long before
+// the cap; a scale-free graph crosses the cap within 2-3 levels).  Synchronises the stream.
+tbc_status single_probe(tbc_graph *g, const int32_t *d_sources, cudaStream_t stream, double *width) {
+    constexpr int64_t kProbeCap = 1 << 16;
+    tbc_status st = single_alloc(g);
+    if (st != TBC_OK) return st;
+    SParams P = single_params(g, d_sources, 1, nullptr);
+    P.probe_cap = kProbeCap;
+    cudaError_t e = cudaMemsetAsync(g->sws.probe_out, 0, 4 * sizeof(int64_t), stream);
+    if (e) return cuda_error(e, "level-width probe");
+    k_bcs<<<1, kSB, 0, stream>>>(P);
+    int64_t h[4] = {0, 0, 0, 0};
+    e = cudaGetLastError();
+    if (!e) e = cudaMemcpyAsync(h, g->sws.probe_out, sizeof h, cudaMemcpyDeviceToHost, stream);
+    if (!e) e = cudaStreamSynchronize(stream);
+    if (e) return cuda_error(e, "level-width probe");
+    *width = (double)h[1] / (double)(h[0] > 0 ? h[0] : 1);
+    return TBC_OK;
+}
+
+}  // namespace tbc

@@ -106,28 +106,39 @@ SMALL = [gg.star(7), gg.path(7, directed=True), gg.cycle(9), gg.complete_biparti
 
 
 @pytest.mark.parametrize("direction", [tbc.DIR_AUTO, tbc.DIR_PUSH, tbc.DIR_PULL])
-@pytest.mark.parametrize("width", [32, 64])
+@pytest.mark.parametrize("width", [32, 64, "narrow"])
 @pytest.mark.parametrize("g", SMALL, ids=lambda g: g.name)
 def test_bfs_batch_small_all_sources(g, width, direction):
     src = np.arange(g.n, dtype=np.int32)
     src = np.concatenate([src, src[:3]]).astype(np.int32)  # repeats inside a sweep
     with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
-        G.set_batch_width(width)
+        if width == "narrow":
+            G.set_batch(tbc.ENGINE_NARROW)
+        else:
+            G.set_batch(tbc.ENGINE_BATCHED)
+            G.set_batch_width(width)
         G.set_direction(direction)
         depth, sigma = G.bfs_batch(src)
     assert_bfs_rows(g, src, depth, sigma)
 
 
-@pytest.mark.parametrize("width", [0, 32, 64])
+@pytest.mark.parametrize("width", [0, 32, 64, "narrow"])
 @pytest.mark.parametrize("scale,directed", [(14, False), (15, True)])
 def test_bfs_batch_kronecker(scale, directed, width):
     g = gg.kronecker(scale, 16, seed=2, directed=directed, device="cuda")
     src = gg.sources(g, 70, seed=12)  # a full sweep of 64 and a ragged one (or 3 of 32)
     with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
-        G.set_batch_width(width)
-        G.set_batch_parts(2)
+        if width == "narrow":
+            G.set_batch(tbc.ENGINE_NARROW)
+        else:
+            G.set_batch(tbc.ENGINE_BATCHED)
+            G.set_batch_width(width)
+            G.set_batch_parts(2)
         depth, sigma = G.bfs_batch(src)
-        assert G.stats()["batch_parts"] == 2
+        st = G.stats()
+        assert st["engine"] == (2 if width == "narrow" else 1)
+        if width != "narrow":
+            assert st["batch_parts"] == 2
     assert_bfs_rows(g, src, depth, sigma)
 
 
@@ -153,13 +164,50 @@ def test_bfs_batch_full_size_kronecker_sweep(cfg):
     assert_bfs_rows(g, src, depth, sigma)
 
 
-def test_bfs_batch_full_size_road_lattice():
+@pytest.mark.parametrize("engine", [tbc.ENGINE_AUTO, tbc.ENGINE_BATCHED])
+def test_bfs_batch_full_size_road_lattice(engine):
     g, src = gg.make_config(4)
     src = src[:6]
     with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+        G.set_batch(engine)
         depth, sigma = G.bfs_batch(src)
+        assert G.stats()["engine"] == (2 if engine == tbc.ENGINE_AUTO else 1)
     assert depth.max() > 1000
     assert_bfs_rows(g, src, depth, sigma)
+
+
+def test_auto_engine_choice():
+    """The level-width probe sends deep narrow graphs (lattice, ER 1024) to the narrow-level engine
+    and scale-free graphs to the batched engine."""
+    cases = [(gg.road_lattice(512, 0.10, seed=4), 2), (gg.make_config(1)[0], 2),
+             (gg.kronecker(16, 16, seed=2, directed=False, device="cuda"), 1)]
+    for g, want in cases:
+        src = gg.sources(g, 40, seed=5)
+        with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+            assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, g.directed, src))
+            st = G.stats()
+            assert st["engine"] == want, (g.name, st["probe_width"])
+
+
+@pytest.mark.parametrize("directed", [False, True])
+def test_narrow_engine_kronecker_and_hubs(directed):
+    """The narrow-level engine on a scale-free graph (hubs: the warp-per-vertex queue of both stages,
+    queue overflow to single threads) and with out-of-range device sources."""
+    import torch
+    g = gg.kronecker(15, 16, seed=9, directed=directed, device="cuda")
+    src = gg.sources(g, 300, seed=4)
+    want = oracle.bc(g.col_ptr, g.row_idx, directed, src)
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+        G.set_batch(tbc.ENGINE_NARROW)
+        assert_bc(G.bc(src), want)
+        bad = np.concatenate([src[:7], [-3, g.n], src[7:]]).astype(np.int32)
+        acc = torch.zeros(g.n, dtype=torch.float64, device="cuda")
+        G.reset_stats()
+        G.bc_device(torch.from_numpy(bad).cuda(), acc)
+        torch.cuda.synchronize()
+        assert_bc(acc.cpu().numpy(), want)
+        st = G.stats()
+        assert st["bad_sources"] == 2 and st["sources"] == len(src)
 
 
 # ------------------------------------------------------------------ multi-GPU entry points, real kernel

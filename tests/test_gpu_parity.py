@@ -17,13 +17,13 @@ pytestmark = pytest.mark.gpu
 # (forward direction, format, backward direction) triples: every forward/backward pass kind
 # gets exercised -- (PULL, LIST) forces the candidate scan + list pull after the first push
 # level; backward 1 = pull over level L's out-edges only, 2 = push from level L+1 (in-edges)
-# the 4th element selects the engine: 1 batched (the default), 0 per source; the 5th the batch
-# width (sources per sweep, 32 default, or 64)
+# the 4th element selects the engine: 1 batched, 0 per source, 2 narrow-level (one source per CTA);
+# the 5th the batch width (sources per sweep, 32 default, or 64)
 MODES = [(tbc.DIR_AUTO, tbc.FMT_AUTO, 0, 1), (tbc.DIR_PUSH, tbc.FMT_AUTO, 0, 1), (tbc.DIR_PULL, tbc.FMT_AUTO, 0, 1),
          (tbc.DIR_AUTO, tbc.FMT_AUTO, 0, 1, 64), (tbc.DIR_PULL, tbc.FMT_AUTO, 0, 1, 64),
          (tbc.DIR_AUTO, tbc.FMT_AUTO, 0, 0), (tbc.DIR_PUSH, tbc.FMT_LIST, 1, 0), (tbc.DIR_PUSH, tbc.FMT_STREAM, 0, 0),
          (tbc.DIR_PULL, tbc.FMT_AUTO, 0, 0), (tbc.DIR_PULL, tbc.FMT_STREAM, 0, 0), (tbc.DIR_PULL, tbc.FMT_LIST, 2, 0),
-         (tbc.DIR_AUTO, tbc.FMT_LIST, 2, 0)]
+         (tbc.DIR_AUTO, tbc.FMT_LIST, 2, 0), (tbc.DIR_AUTO, tbc.FMT_AUTO, 0, 2)]
 
 
 def set_mode(G, mode):

@@ -60,8 +60,10 @@ enum {
     TBC_FLAG_ONE_FORMAT = 1u << 0,  /* reserved (strict single-format directed mode, not yet built) */
     TBC_FLAG_NO_VALIDATE = 1u << 1, /* skip host-side input validation (caller guarantees it) */
     TBC_FLAG_NO_REORDER = 1u << 2   /* keep the caller's vertex labels internally (default: relabel by
-                                       decreasing degree for cache locality; all inputs and outputs
-                                       stay in the caller's labels either way) */
+                                       decreasing degree when the degree distribution is skewed --
+                                       max degree > 16 x mean -- so hubs share cache lines; flat
+                                       graphs keep their labels; all inputs and outputs stay in the
+                                       caller's labels either way) */
 };
 
 /* options for tbc_graph_set_option.  Every forward level is run as one of five passes, chosen

@@ -234,10 +234,23 @@ tbc_status build_from_keys(tbc_graph *g, unsigned long long *d_keys, int64_t nnz
         }
         if (!e1) e1 = cudaMalloc(&rtemp, rbytes);
         if (!e1) e1 = cub::DeviceRadixSort::SortPairsDescending(rtemp, rbytes, deg, deg_s, ids, g->inv, g->n, 0, 32, s);
-        if (!e1) {
+        // only degree-skewed graphs are relabelled (max endpoint count > 16 x the mean): on flat
+        // degree distributions (lattices, road networks, ER) the caller's labels keep whatever
+        // locality they have, which the sort by degree would scatter
+        int32_t dmax = 0;
+        if (!e1) e1 = cudaMemcpyAsync(&dmax, deg_s, sizeof dmax, cudaMemcpyDeviceToHost, s);
+        if (!e1) e1 = cudaStreamSynchronize(s);
+        const bool skewed = (double)dmax > 16.0 * 2.0 * (double)nnz / (double)g->n;
+        if (!e1 && skewed) {
             k_invert<<<grid_for(g->n), 256, 0, s>>>(g->n, g->inv, g->perm);
             k_relabel<<<grid_for(nnz), 256, 0, s>>>(nnz, d_keys, g->perm);
             e1 = cudaStreamSynchronize(s);
+        }
+        if (!e1 && !skewed) {
+            cudaFree(g->inv);
+            cudaFree(g->perm);
+            g->inv = g->perm = nullptr;
+            g->device_bytes -= 2 * sizeof(int32_t) * g->n;
         }
         cudaFree(deg);
         cudaFree(deg_s);

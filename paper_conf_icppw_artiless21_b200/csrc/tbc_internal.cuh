@@ -149,11 +149,19 @@ struct BatchWorkspace {
 };
 // workspace of the narrow-level engine (tbc_single.cu): one slot of per-vertex arrays per
 // concurrently running source (one per resident CTA)
+// per (slot, vertex) state of the narrow-level engine: one 32-byte DRAM sector
+struct __align__(32) VRec {
+    double sd;     // sigma (forward), then delta_u (backward); 0 between sources
+    int32_t depth; // -1 between sources
+    int32_t pad;
+    double bc;     // the slot's partial bc, summed into the caller's bc after each call
+    double pad2;
+};
+static_assert(sizeof(VRec) == 32, "one sector per vertex record");
 struct SingleWorkspace {
     int slots = 0;
     size_t bytes = 0;
-    int32_t *depth = nullptr;    // [slots][n]
-    double *sd = nullptr;        // [slots][n] sigma, then delta_u
+    VRec *rec = nullptr;         // [slots][n]
     int32_t *order = nullptr;    // [slots][n]
     int32_t *lvl = nullptr;      // [slots][n + 2]
     Ctrs *ctr = nullptr;

@@ -20,6 +20,10 @@
 //     in place, because a vertex has one level and its sigma is read only by its own update.
 //   level L+2 is reset (depth -1, sigma 0) during level L, levels 0..2 at the end: a CTA's arrays
 //   are all-unvisited between sources, with no O(n) clear.
+// A vertex's whole per-source state is one 32-byte record (one DRAM sector): {sigma / delta_u,
+// depth, the slot's partial bc}; every step touches one sector per vertex.  The partial bc of a
+// slot accumulates over its sources with plain read-modify-writes (a slot belongs to one CTA) and
+// k_bcs_reduce adds the slots into the caller's bc after the kernel.
 // Out-degrees above kHeavy are deferred to a per-level shared-memory queue and run by a whole warp.
 #include <cstdio>
 
@@ -39,8 +43,7 @@ struct SParams {
     int64_t n;
     const int64_t *__restrict__ out_ptr;  // CSR of A (== the CSC when undirected)
     const int32_t *__restrict__ out_idx;
-    int32_t *depth;   // [slots][n], -1 between sources
-    double *sd;       // [slots][n], sigma (forward) then delta_u (backward); 0 between sources
+    VRec *rec;        // [slots][n]: sigma / delta_u (0 between sources), depth (-1 between sources), bc
     int32_t *order;   // [slots][n], BFS order, levels concatenated
     int32_t *lvl;     // [slots][n + 2], level offsets into order
     Ctrs *ctr;
@@ -57,32 +60,36 @@ struct SParams {
 };
 
 // relax the out-edge u -> w of frontier level d: claim w for level d+1, add sigma(u)
-__device__ __forceinline__ void relax(const SParams &P, int32_t *depth, double *sd, int32_t *order, int32_t w,
-                                      int d, double su, int *cnt, int end) {
-    int dw = __ldcg(depth + w);
+__device__ __forceinline__ void relax(VRec *rec, int32_t *order, int32_t w, int d, double su, int *cnt, int end) {
+    int dw = __ldcg(&rec[w].depth);
     if (dw == -1) {
-        dw = atomicCAS(depth + w, -1, d + 1);
+        dw = atomicCAS(&rec[w].depth, -1, d + 1);
         if (dw == -1) {
             order[end + atomicAdd(cnt, 1)] = w;
             dw = d + 1;
         }
     }
-    if (dw == d + 1) atomicAdd(sd + w, su);
+    if (dw == d + 1) atomicAdd(&rec[w].sd, su);
+}
+
+// delta_u(w) if w is on level L+1, else 0 (one 16-byte load: sd and depth share it)
+__device__ __forceinline__ double child(const VRec *rec, int32_t w, int L) {
+    const double2 r = __ldcg(reinterpret_cast<const double2 *>(rec + w));
+    return __double2loint(r.y) == L + 1 ? r.x : 0.0;
 }
 
 // Alg.1 l.35-45 for v with acc = sum of delta_u over its level-(L+1) out-neighbours
-__device__ __forceinline__ void finish(const SParams &P, double *sd, int32_t v, double acc) {
-    const double sv = __ldcg(sd + v);
+__device__ __forceinline__ void finish(const SParams &P, VRec *rec, int32_t v, double acc) {
+    const double sv = __ldcg(&rec[v].sd);
     const double delta = sv * acc;
-    if (delta != 0.0) atomicAdd(P.bc + (P.inv ? P.inv[v] : v), delta * P.bc_scale);
-    sd[v] = 1.0 / sv + acc;
+    if (delta != 0.0) rec[v].bc += delta * P.bc_scale;
+    rec[v].sd = 1.0 / sv + acc;
 }
 
-__device__ __forceinline__ void reset_level(int32_t *depth, double *sd, const int32_t *order, int b0, int b1) {
+__device__ __forceinline__ void reset_level(VRec *rec, const int32_t *order, int b0, int b1) {
     for (int i = b0 + (int)threadIdx.x; i < b1; i += kSB) {
         const int32_t x = order[i];
-        depth[x] = -1;
-        sd[x] = 0.0;
+        *reinterpret_cast<int4 *>(rec + x) = make_int4(0, 0, -1, 0);  // sd = 0, depth = -1, pad = 0
     }
 }
 
@@ -90,8 +97,7 @@ __global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int64_t n = P.n;
     const int64_t slot = blockIdx.x;
-    int32_t *depth = P.depth + slot * n;
-    double *sd = P.sd + slot * n;
+    VRec *rec = P.rec + slot * n;
     int32_t *order = P.order + slot * n;
     int32_t *lvl = P.lvl + slot * (n + 2);
     __shared__ int s_cnt[2], s_hcnt[2];
@@ -105,8 +111,8 @@ __global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) 
         }
         if (P.perm) s = P.perm[s];
         if (tid == 0) {  // level 0 (Alg.1 l.15-18)
-            depth[s] = 0;
-            sd[s] = 1.0;
+            rec[s].depth = 0;
+            rec[s].sd = 1.0;
             order[0] = s;
             lvl[0] = 0;
             lvl[1] = 1;
@@ -133,8 +139,8 @@ __global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) 
                         continue;
                     }
                 }
-                const double su = __ldcg(sd + u);
-                for (int64_t e = e0; e < e1; ++e) relax(P, depth, sd, order, P.out_idx[e], d, su, &s_cnt[par], end);
+                const double su = __ldcg(&rec[u].sd);
+                for (int64_t e = e0; e < e1; ++e) relax(rec, order, P.out_idx[e], d, su, &s_cnt[par], end);
             }
             __syncthreads();
             if (tid == 0) {  // counters of level d+2 (their level-d readers are past the barrier)
@@ -144,10 +150,10 @@ __global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) 
             const int nh = min(s_hcnt[par], kHeavyCap);
             for (int h = warp; h < nh; h += kSWarps) {
                 const int32_t u = s_heavy[h];
-                const double su = __ldcg(sd + u);
+                const double su = __ldcg(&rec[u].sd);
                 const int64_t e1 = P.out_ptr[u + 1];
                 for (int64_t e = P.out_ptr[u] + lane; e < e1; e += 32)
-                    relax(P, depth, sd, order, P.out_idx[e], d, su, &s_cnt[par], end);
+                    relax(rec, order, P.out_idx[e], d, su, &s_cnt[par], end);
             }
             __syncthreads();
             const int nn = s_cnt[par];
@@ -172,7 +178,7 @@ __global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) 
                 P.probe_out[1] = end;    // vertices discovered
                 P.probe_out[2] = probe_stop ? 0 : 1;
             }
-            reset_level(depth, sd, order, 0, end);
+            reset_level(rec, order, 0, end);
             __syncthreads();
             return;
         }
@@ -191,11 +197,11 @@ __global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) 
                     const int32_t x = order[i];
                     const int64_t o = si * n + (P.inv ? P.inv[x] : x);
                     P.bfs_depth[o] = L;
-                    P.bfs_sigma[o] = __ldcg(sd + x);
+                    P.bfs_sigma[o] = __ldcg(&rec[x].sd);
                 }
             }
             __syncthreads();
-            reset_level(depth, sd, order, 0, end);
+            reset_level(rec, order, 0, end);
             if (tid == 0) s_edges[0] = 0;
             __syncthreads();
             continue;
@@ -217,13 +223,10 @@ __global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) 
                     }
                 }
                 double acc = 0.0;
-                for (int64_t e = e0; e < e1; ++e) {
-                    const int32_t w = P.out_idx[e];
-                    if (__ldcg(depth + w) == L + 1) acc += __ldcg(sd + w);
-                }
-                finish(P, sd, v, acc);
+                for (int64_t e = e0; e < e1; ++e) acc += child(rec, P.out_idx[e], L);
+                finish(P, rec, v, acc);
             }
-            if (L + 2 <= D) reset_level(depth, sd, order, lvl[L + 2], lvl[L + 3]);
+            if (L + 2 <= D) reset_level(rec, order, lvl[L + 2], lvl[L + 3]);
             __syncthreads();
             if (tid == 0) s_hcnt[par ^ 1] = 0;
             const int nh = min(s_hcnt[par], kHeavyCap);
@@ -231,17 +234,14 @@ __global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) 
                 const int32_t v = s_heavy[h];
                 const int64_t e1 = P.out_ptr[v + 1];
                 double acc = 0.0;
-                for (int64_t e = P.out_ptr[v] + lane; e < e1; e += 32) {
-                    const int32_t w = P.out_idx[e];
-                    if (__ldcg(depth + w) == L + 1) acc += __ldcg(sd + w);
-                }
+                for (int64_t e = P.out_ptr[v] + lane; e < e1; e += 32) acc += child(rec, P.out_idx[e], L);
 #pragma unroll
                 for (int o = 16; o >= 1; o >>= 1) acc += __shfl_xor_sync(FULL, acc, o);
-                if (lane == 0) finish(P, sd, v, acc);
+                if (lane == 0) finish(P, rec, v, acc);
             }
             __syncthreads();
         }
-        reset_level(depth, sd, order, 0, lvl[min(D, 2) + 1]);
+        reset_level(rec, order, 0, lvl[min(D, 2) + 1]);
         atomicAdd(&s_edges[1], my_bwd);
         __syncthreads();
         if (tid == 0) {
@@ -253,16 +253,33 @@ __global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) 
     }
 }
 
+// bc(v) += sum over the used slots of their partial bc(v); the partials return to 0
+__global__ void k_bcs_reduce(int64_t n, int64_t slots, VRec *rec, double *bc, const int32_t *__restrict__ inv) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
+        double sum = 0.0;
+        for (int64_t q = 0; q < slots; ++q) {
+            double *p = &rec[q * n + v].bc;
+            sum += *p;
+            *p = 0.0;
+        }
+        if (sum != 0.0) bc[inv ? inv[v] : v] += sum;
+    }
+}
+
+__global__ void k_rec_init(int64_t count, VRec *rec) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x)
+        rec[i] = VRec{0.0, -1, 0, 0.0, 0.0};
+}
+
 }  // namespace
 
 // ------------------------------------------------------------------ host side
 
-static int64_t single_slot_bytes(const tbc_graph *g) { return 20 * g->n + 8; }
+static int64_t single_slot_bytes(const tbc_graph *g) { return (int64_t)sizeof(VRec) * g->n + 8 * g->n + 8; }
 
 void single_free(tbc_graph *g) {
     SingleWorkspace &w = g->sws;
-    cudaFree(w.depth);
-    cudaFree(w.sd);
+    cudaFree(w.rec);
     cudaFree(w.order);
     cudaFree(w.lvl);
     cudaFree(w.ctr);
@@ -298,15 +315,14 @@ static tbc_status single_alloc(tbc_graph *g) {
         }
         return r;
     };
-    if ((e = alloc(&w.depth, slots * n)) || (e = alloc(&w.sd, slots * n)) || (e = alloc(&w.order, slots * n)) ||
+    if ((e = alloc(&w.rec, slots * n)) || (e = alloc(&w.order, slots * n)) ||
         (e = alloc(&w.lvl, slots * (n + 2))) || (e = alloc(&w.ctr, 1)) || (e = alloc(&w.probe_out, 4))) {
         single_free(g);
         return cuda_error(e, "narrow-level engine workspace cudaMalloc");
     }
     cudaStream_t s = g->stream;
-    if ((e = cudaMemsetAsync(w.depth, 0xff, sizeof(int32_t) * slots * n, s)) ||
-        (e = cudaMemsetAsync(w.sd, 0, sizeof(double) * slots * n, s)) ||
-        (e = cudaMemsetAsync(w.ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s))) {
+    k_rec_init<<<148 * 8, 256, 0, s>>>(slots * n, w.rec);
+    if ((e = cudaGetLastError()) || (e = cudaMemsetAsync(w.ctr, 0, sizeof(Ctrs), s)) || (e = cudaStreamSynchronize(s))) {
         single_free(g);
         return cuda_error(e, "narrow-level engine workspace init");
     }
@@ -320,8 +336,7 @@ static SParams single_params(tbc_graph *g, const int32_t *d_sources, int64_t k, 
     P.n = g->n;
     P.out_ptr = g->out_ptr;
     P.out_idx = g->out_idx;
-    P.depth = w.depth;
-    P.sd = w.sd;
+    P.rec = w.rec;
     P.order = w.order;
     P.lvl = w.lvl;
     P.ctr = w.ctr;
@@ -348,6 +363,10 @@ tbc_status single_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
     k_bcs<<<grid, kSB, 0, stream>>>(P);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_bcs launch");
+    if (!bfs_depth) {
+        k_bcs_reduce<<<148 * 8, 256, 0, stream>>>(g->n, grid, g->sws.rec, d_bc, g->inv);
+        if ((e = cudaGetLastError()) != cudaSuccess) return cuda_error(e, "k_bcs_reduce launch");
+    }
     return TBC_OK;
 }
 

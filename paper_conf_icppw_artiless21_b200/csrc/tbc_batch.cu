@@ -48,6 +48,9 @@ constexpr int kPad = 8;
 #ifndef TBC_BUNROLL64
 #define TBC_BUNROLL64 8
 #endif
+#ifndef TBC_STATIC_PCT
+#define TBC_STATIC_PCT 60  // share of a pass's tiles dealt statically (the rest: dynamic, one per atomic)
+#endif
 // gathers in flight per lane in the slot loop, by batch width (A/B on B200: W = 32 best at 6 --
 // Kronecker 25: 394 vs 389 at 4, 373 at 8; W = 64 best at 8, i.e. 4 per source -- Kronecker 22:
 // 332 vs 318 at 6, RMAT 18: 359 vs 350)
@@ -283,7 +286,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                                       const uint32_t *obeg, const void *omsk_, const int32_t *otiles, int64_t N,
                                       int64_t E, const int32_t *__restrict__ adj_idx, const void *emsk_,
                                       void *fr_out_, unsigned long long active_, int64_t gwarp, int64_t nwarps,
-                                      const BOut &out) {
+                                      const BOut &out, unsigned long long *dyn) {
     using MT = typename MaskT<W>::T;
     constexpr int NS = W / 32;                 // sources per lane
     constexpr int U2 = (NS == 1 ? kBU : kBU64) / NS > 0 ? (NS == 1 ? kBU : kBU64) / NS : 1;  // gathers in flight per lane and source
@@ -297,7 +300,17 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
     const int64_t ntiles = cdiv(K, kBT);
     const uint64_t pol = policy_evict_first();
     double *const sig = P.sig;
-    for (int64_t tile = gwarp; tile < ntiles; tile += nwarps) {
+    // tiles [0, nstat) are dealt round-robin; the rest are taken one at a time from the pass's
+    // counter by warps that ran out, so the costly tiles (many active lanes) do not leave most
+    // warps waiting at the next grid barrier
+    const int64_t nstat = (ntiles * TBC_STATIC_PCT) / 100;
+    for (int64_t tile = gwarp < nstat ? gwarp : ntiles; ; ) {
+        if (tile >= nstat) {
+            unsigned long long t = 0;
+            if (lane == 0) t = atomicAdd(dyn, 1ull);
+            tile = nstat + (int64_t)__shfl_sync(FULL, t, 0);
+            if (tile >= ntiles) break;
+        }
         BPROF_START();
         const int64_t ks = tile * kBT;
         const int64_t ke = min(ks + (int64_t)kBT, K);
@@ -557,6 +570,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
         }
         __syncwarp();
         BPROF(BR_OWN);
+        tile += nwarps;
     }
 }
 
@@ -692,9 +706,11 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
                 C->list = ((unsigned long long)pos0 << P.ebits) | e0;
                 C->ilist = 0;
                 C->cand[0] = 0;
+                C->dyn[0] = C->dyn[1] = 0;
                 C->st_sources += valid;
             }
         }
+        unsigned ph = 0;  // edge passes of this batch so far (selects the dynamic-tile counter)
         const bool tr = b == P.trace_b && cta0;
         if (tr && cta0 && tid == 0) P.gctr->trace_n = 0;
         bsync(C, gen, ncta);
@@ -779,17 +795,20 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             const BOut lo{&C->list, P.list_v + nxt.p0, P.list_pre + nxt.p0, P.list_beg + nxt.p0, P.tiles + nxt.tb,
                           P.list_cap - nxt.p0, P.tiles_cap - nxt.tb};
             MT *fro = fr[(d + 1) & 1];
+            if (cta0 && tid == 0) C->dyn[(ph + 1) & 1] = 0;  // the next pass's counter (its last user is done)
             if (pull) {
                 const int64_t cN = (int64_t)(cs >> P.ebits), cE = (int64_t)(cs & emask);
                 bpass<B_PULL, W>(P, ws, P.cand_v, P.cand_pre, P.cand_beg, nullptr, P.cand_tiles, cN, cE, P.in_idx,
-                              fr[d & 1], fro, (unsigned long long)active, gwarp, nwarps, lo);
+                              fr[d & 1], fro, (unsigned long long)active, gwarp, nwarps, lo, &C->dyn[ph & 1]);
                 fwd_edges += cE;
                 ++pulls;
             } else {
                 bpass<B_PUSH, W>(P, ws, P.list_v + cur.p0, P.list_pre + cur.p0, P.list_beg + cur.p0, list_m + cur.p0,
-                              P.tiles + cur.tb, cur.N, cur.E, P.out_idx, nullptr, fro, 0u, gwarp, nwarps, lo);
+                              P.tiles + cur.tb, cur.N, cur.E, P.out_idx, nullptr, fro, 0u, gwarp, nwarps, lo,
+                              &C->dyn[ph & 1]);
                 fwd_edges += cur.E;
             }
+            ++ph;
             bsync(C, gen, ncta);
             {
                 const unsigned long long lv = ld_volatile_u64(&C->snap[0]);
@@ -832,8 +851,11 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             const int64_t *l = P.lvl + 4 * (int64_t)L;
             const Lv lv{l[0], l[1], l[2], l[3]};
             const BOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0};
+            if (cta0 && tid == 0) C->dyn[(ph + 1) & 1] = 0;  // the next pass's counter (its last user is done)
             bpass<B_BWD, W>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.list_beg + lv.p0, list_m + lv.p0,
-                         P.tiles + lv.tb, lv.N, lv.E, P.out_idx, fr[(L + 1) & 1], fr[L & 1], 0u, gwarp, nwarps, none);
+                         P.tiles + lv.tb, lv.N, lv.E, P.out_idx, fr[(L + 1) & 1], fr[L & 1], 0u, gwarp, nwarps, none,
+                         &C->dyn[ph & 1]);
+            ++ph;
             bwd_edges += lv.E;
             if (L + 2 <= D) {
                 BPROF_START();

@@ -29,6 +29,7 @@ struct Ctrs {
     // already be appending to (next push level) or zeroing (candidate reset)
     unsigned long long snap[4];
     unsigned long long bad_sources;
+    unsigned long long dyn[2];    // batched engine: dynamic tile counters of consecutive edge passes
     unsigned long long trace_n;   // entries written to the trace buffer
     // accumulated statistics (tbc_stats)
     long long st_sources, st_reached, st_reached_edges, st_fwd_edges, st_bwd_edges, st_levels, st_pull_levels,

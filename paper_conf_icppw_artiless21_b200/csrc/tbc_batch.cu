@@ -37,7 +37,10 @@ namespace tbc {
 namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
-constexpr int kBB = 1024;        // threads per CTA (one CTA per SM)
+#ifndef TBC_BBLOCK
+#define TBC_BBLOCK 1024
+#endif
+constexpr int kBB = TBC_BBLOCK;  // threads per CTA (one CTA per SM)
 constexpr int kBWarps = kBB / 32;
 constexpr int kBI = 2;           // tile items per lane (window / index phases)
 constexpr int kBT = 32 * kBI;    // diagonal items (owner end items + edges) per warp tile
@@ -49,7 +52,10 @@ constexpr int kPad = 8;
 #define TBC_BUNROLL64 8
 #endif
 #ifndef TBC_STATIC_PCT
-#define TBC_STATIC_PCT 60  // share of a pass's tiles dealt statically (the rest: dynamic, one per atomic)
+#define TBC_STATIC_PCT 60  // share of a pass's tiles dealt statically (the rest: dynamic)
+#endif
+#ifndef TBC_DYN_CHUNK
+#define TBC_DYN_CHUNK 1    // tiles taken per atomic in the dynamic share
 #endif
 // gathers in flight per lane in the slot loop, by batch width (A/B on B200: W = 32 best at 6 --
 // Kronecker 25: 394 vs 389 at 4, 373 at 8; W = 64 best at 8, i.e. 4 per source -- Kronecker 22:
@@ -304,13 +310,15 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
     // counter by warps that ran out, so the costly tiles (many active lanes) do not leave most
     // warps waiting at the next grid barrier
     const int64_t nstat = (ntiles * TBC_STATIC_PCT) / 100;
-    for (int64_t tile = gwarp < nstat ? gwarp : ntiles; ; ) {
-        if (tile >= nstat) {
+    int64_t dend = -1;  // end of the warp's current dynamic chunk of TBC_DYN_CHUNK tiles
+    for (int64_t tile = gwarp;;) {
+        if (tile >= nstat && tile >= dend) {
             unsigned long long t = 0;
             if (lane == 0) t = atomicAdd(dyn, 1ull);
-            tile = nstat + (int64_t)__shfl_sync(FULL, t, 0);
-            if (tile >= ntiles) break;
+            tile = nstat + (int64_t)__shfl_sync(FULL, t, 0) * TBC_DYN_CHUNK;
+            dend = tile + TBC_DYN_CHUNK;
         }
+        if (tile >= ntiles) break;
         BPROF_START();
         const int64_t ks = tile * kBT;
         const int64_t ke = min(ks + (int64_t)kBT, K);
@@ -570,7 +578,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
         }
         __syncwarp();
         BPROF(BR_OWN);
-        tile += nwarps;
+        tile += tile < nstat ? nwarps : 1;
     }
 }
 

@@ -1325,6 +1325,7 @@ tbc_status engine_choose(tbc_graph *g, const int32_t *d_sources, int64_t k, cuda
         if (st != TBC_OK) return st;
         g->narrow = width < g->narrow_width ? 1 : 0;
         g->probe_width = width;
+        if (!g->narrow) single_free(g);  // the probe's slot
     }
     *mode = g->last_mode = g->narrow == 1 ? 2 : 1;
     return TBC_OK;

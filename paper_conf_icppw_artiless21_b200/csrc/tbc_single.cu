@@ -289,10 +289,12 @@ void single_free(tbc_graph *g) {
 }
 
 // one slot (a CTA's arrays) per concurrently running source: as many as the GPU keeps resident,
-// within 80 % of the free memory (at least one); sized once per graph
-static tbc_status single_alloc(tbc_graph *g) {
+// within 60 % of the free memory (at least one); sized once per graph.  probe_only: one slot (the
+// level-width probe must not take the memory the batched engine may need)
+static tbc_status single_alloc(tbc_graph *g, bool probe_only = false) {
     SingleWorkspace &w = g->sws;
-    if (w.slots > 0) return TBC_OK;
+    if (w.slots > 1 || (w.slots == 1 && probe_only)) return TBC_OK;
+    if (w.slots) single_free(g);  // the probe's single slot: grow to the full set
     cudaError_t e = cudaSuccess;
     int per_sm = 0, sms = 0;
     if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_bcs, kSB, 0)) ||
@@ -301,8 +303,8 @@ static tbc_status single_alloc(tbc_graph *g) {
     if (per_sm < 1) return set_error(TBC_ERR_CUDA, "k_bcs cannot be resident");
     size_t fr = 0, tot = 0;
     if ((e = cudaMemGetInfo(&fr, &tot))) return cuda_error(e, "cudaMemGetInfo");
-    int64_t slots = (int64_t)per_sm * sms;
-    const int64_t fit = (int64_t)(0.8 * (double)fr / (double)single_slot_bytes(g));
+    int64_t slots = probe_only ? 1 : (int64_t)per_sm * sms;
+    const int64_t fit = (int64_t)(0.6 * (double)fr / (double)single_slot_bytes(g));
     if (slots > fit) slots = fit;
     if (slots < 1) slots = 1;
     const int64_t n = g->n;
@@ -376,7 +378,7 @@ tbc_status single_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
 // the cap; a scale-free graph crosses the cap within 2-3 levels).  Synchronises the stream.
 tbc_status single_probe(tbc_graph *g, const int32_t *d_sources, cudaStream_t stream, double *width) {
     constexpr int64_t kProbeCap = 1 << 16;
-    tbc_status st = single_alloc(g);
+    tbc_status st = single_alloc(g, true);
     if (st != TBC_OK) return st;
     SParams P = single_params(g, d_sources, 1, nullptr);
     P.probe_cap = kProbeCap;

@@ -4,8 +4,8 @@
 IFS='|' read -ra VARS <<< "${AB_VARIANTS:-}"
 IFS='|' read -ra CFGS <<< "${AB_CONFIGS:-3}"
 run() {  # "cfg extra" variant
-  TBC_VARIANT="$2" timeout 400 python bench.py --config $1 --steps ${AB_STEPS:-3} --warmup 2 --no-cpu-baseline 2>/dev/null | tail -1 |
-    python -c "import json,sys; d=json.loads(sys.stdin.read()); print(round(d['value'],2), round(d['roofline']['frac'],3), d['clocks']['sm_mhz'], d['config']['engine_mode'][:30])" 2>&1
+  TBC_VARIANT="$2" timeout 400 python bench.py --config $1 --steps ${AB_STEPS:-3} --warmup 2 --no-cpu-baseline > /tmp/ab_out.txt 2>&1
+  grep '^{' /tmp/ab_out.txt | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(round(d['value'],2), round(d['roofline']['frac'],3), d['clocks']['sm_mhz'], d['config']['engine_mode'][:30])" 2>/dev/null || tail -3 /tmp/ab_out.txt
 }
 for c in "${CFGS[@]}"; do
   for rep in $(seq ${AB_REPS:-2}); do

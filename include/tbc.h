@@ -108,9 +108,12 @@ enum {
                                 when the frontier's out-edges x this value > nnz, else pushed
                                 (default 8; must be >= 0) */
     TBC_OPT_BATCH_WIDTH = 14, /* batched engine: sources per sweep, 32 (one per warp lane) or 64
-                                (two per lane), or 0 (default) = 64 up to 8 M vertices, else 32
-                                (measured).  Workspace ~ 2 x 8 W B/vertex of (sigma,
-                                delta_u) rows plus level lists of <= W entries per vertex. */
+                                (two per lane), or 0 (default, settled once per graph) = 64 up to 8 M
+                                vertices, and above that for average degree >= 8 when the W = 64
+                                workspace fits 85 % of the free memory, else 32 (measured, DESIGN.md
+                                4.5); a W = 64 workspace that then fails to allocate falls back to 32.
+                                Workspace per SM partition ~ 16 W B/vertex of (sigma, delta_u) rows +
+                                TBC_OPT_BATCH_LIST x (12 + W/8) B/vertex of level lists + tile starts. */
     TBC_OPT_BATCH_PARTS = 16, /* batched engine: SM partitions (1..8, or 0 = auto, the default: 1 for
                                 graphs whose sigma rows overflow 1 GiB with average degree >= 8 or
                                 with average degree >= 64, else up to 4 (average degree >= 8) or 8
@@ -121,8 +124,11 @@ enum {
                                 stable sort by 2-hop out-volume class, then out-degree (bc is a sum
                                 over sources, so only the floating-point summation order changes),
                                 0 in the given order */
-    TBC_OPT_NARROW_WIDTH = 18 /* auto engine: probe vertices per level below which the narrow-level
+    TBC_OPT_NARROW_WIDTH = 18, /* auto engine: probe vertices per level below which the narrow-level
                                 engine runs (default 4096; setting it re-runs the probe next call) */
+    TBC_OPT_BATCH_LIST = 19  /* batched engine: level-list entries allocated per vertex (1..64, default 2;
+                                capped at W).  A sweep whose lists outgrow them is re-run as two half
+                                sweeps (tbc_stats.list_overflows) and the next call doubles them. */
 };
 
 /* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since
@@ -145,6 +151,8 @@ typedef struct {
     int64_t workspace_bytes; /* device bytes of the engine workspaces now allocated (included in
                                 tbc_graph_info's device_bytes); not reset by tbc_stats_reset */
     int64_t engine;      /* engine of the latest bc call: 0 per source, 1 batched, 2 narrow-level, -1 none */
+    int64_t list_overflows; /* batched engine: sweeps whose level lists outgrew the workspace and were
+                               re-run as two half sweeps (the next call grows the lists) */
     int64_t probe_width; /* auto engine: the probe's vertices per level (0 before the probe) */
 } tbc_stats;
 

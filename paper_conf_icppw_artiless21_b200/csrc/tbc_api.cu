@@ -189,6 +189,7 @@ void free_graph(tbc_graph *g) {
     cudaFree(g->in_col);
     if (g->out_row != g->in_col) cudaFree(g->out_row);
     engine_free(g);
+    if (g->h_bovf) cudaFreeHost(g->h_bovf);
     cudaFree(g->bfs_depth);
     cudaFree(g->bfs_sigma);
     cudaFree(g->bc_tmp);
@@ -547,6 +548,13 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->batch = v;
         return TBC_OK;
     }
+    if (key == TBC_OPT_BATCH_LIST) {
+        int v = (int)value;
+        if (v < 1 || v > 64 || (double)v != value) return set_error(TBC_ERR_INVALID, "batch list factor %g not in [1, 64]", value);
+        g->blist_factor = v;
+        for (int q = 0; q < kMaxPartitions; ++q) batch_free_one(g, q);  // resized at the next call
+        return TBC_OK;
+    }
     if (key == TBC_OPT_NARROW_WIDTH) {
         if (!(value >= 0)) return set_error(TBC_ERR_INVALID, "narrow width %g", value);
         g->narrow_width = value;
@@ -738,6 +746,7 @@ tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
         TBC_CUDA(cudaMemcpy(&c, src, sizeof c, cudaMemcpyDeviceToHost));
         out->bad_sources += (int64_t)c.bad_sources;
         if (c.st_list_peak > out->list_peak) out->list_peak = c.st_list_peak;
+        out->list_overflows += c.st_overflows;
         out->sources += c.st_sources;
         out->reached += c.st_reached;
         out->reached_edges += c.st_reached_edges;
@@ -791,7 +800,7 @@ fail:
 #endif
 }
 
-static constexpr size_t kStatBytes = offsetof(Ctrs, st_list_peak) + sizeof(long long) - offsetof(Ctrs, st_sources);
+static constexpr size_t kStatBytes = offsetof(Ctrs, st_overflows) + sizeof(long long) - offsetof(Ctrs, st_sources);
 
 tbc_status tbc_stats_reset(tbc_graph *g) {
     if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
@@ -802,7 +811,7 @@ tbc_status tbc_stats_reset(tbc_graph *g) {
         Ctrs *c = i < g->ws_count ? g->ws[i].ctr
                   : i < g->ws_count + kMaxPartitions ? g->bws[i - g->ws_count].ctr : g->sws.ctr;
         if (!c) continue;
-        TBC_CUDA(cudaMemset(&c->st_sources, 0, kStatBytes));  // st_sources .. st_list_peak
+        TBC_CUDA(cudaMemset(&c->st_sources, 0, kStatBytes));  // st_sources .. st_overflows
         TBC_CUDA(cudaMemset(&c->bad_sources, 0, sizeof(unsigned long long)));
     }
     return TBC_OK;

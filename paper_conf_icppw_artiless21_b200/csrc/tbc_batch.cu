@@ -73,7 +73,7 @@ template <> struct MaskT<64> { using T = unsigned long long; };
 // 0 barrier, 1 B phase, 2 push pass, 3 pull pass, 4 backward pass, 5 retire, 6 init/other,
 // 8 + {0 window, 1 index+masks, 2 claims/append, 3 owner loop} inside the edge passes
 enum { BR_BAR = 0, BR_BPHASE = 1, BR_PASS = 2, BR_CLEAR = 5, BR_OTHER = 6, BR_WIN = 8, BR_IDX = 9, BR_APP = 10,
-       BR_OWN = 11, BR_SLOTS = 16 };
+       BR_OWN = 11, BR_OGATH = 12, BR_OEPI = 13, BR_SLOTS = 16 };
 #ifdef TBC_PROF
 __shared__ unsigned long long tbc_bprof[kBWarps][BR_SLOTS];
 #define BPROF_START() unsigned long long _bt = clock64()
@@ -208,6 +208,7 @@ struct BOut {
     uint32_t *pre, *beg;
     int32_t *tiles;
     int64_t cap, tcap;
+    unsigned *ovf;  // set when an entry or a tile start does not fit (the batch is re-run in halves)
 };
 
 // warp-aggregated append of the entries lanes hold (item i of lane l: v[i], degree dg[i],
@@ -244,12 +245,14 @@ __device__ __forceinline__ void bappend(const bool (&take)[kBI], const int32_t (
         if (take[i]) {
             const int64_t pp = p + __popc(msk & lt);
             const int64_t ee = e + (int64_t)(inc - x);
-            if (pp < o.cap) {  // capacities are sufficient by construction (batch_alloc)
+            const int64_t k0 = ee + pp, k1 = k0 + x;
+            if (pp < o.cap && k1 / kBT < o.tcap) {
                 o.v[pp] = v[i];
                 o.pre[pp] = (uint32_t)ee;
                 o.beg[pp] = bg[i];
-                const int64_t k0 = ee + pp, k1 = k0 + x;
-                for (int64_t t = (k0 + kBT - 1) / kBT; t <= k1 / kBT && t < o.tcap; ++t) o.tiles[t] = (int32_t)pp;
+                for (int64_t t = (k0 + kBT - 1) / kBT; t <= k1 / kBT; ++t) o.tiles[t] = (int32_t)pp;
+            } else {  // capacity exceeded: the kernel re-runs the batch in halves (k_bcb)
+                *o.ovf = 1u;
             }
         }
         p += __popc(msk);
@@ -437,11 +440,17 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
         __syncwarp();
         BPROF(BR_APP);
         int nc = 0;  // PULL: discovered owners of this tile
+#ifdef TBC_PROF
+        unsigned n_own = 0;
+#endif
         for (int j = 0; j < nwin; ++j) {
             uint64_t bits = act & slot_range(ws.first[j], ws.first[j + 1]);
             const int fl = ws.fl[j];
             if (MODE != B_BWD && bits == 0) continue;
             if (MODE == B_BWD && bits == 0 && !(fl & 1)) continue;
+#ifdef TBC_PROF
+            ++n_own;
+#endif
             const int32_t v = ws.v[j];
             const MT m = (MT)ws.msk[j];
             const int64_t row = (int64_t)v * W + lane;  // + 32 k: the lane's word of source k
@@ -479,6 +488,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             }
             // the two 32-slot halves of the tile, U2 gathers in flight per lane and source;
             // __ffs(0) = 0 marks the exhausted positions
+            BPROF(BR_OWN);
 #pragma unroll
             for (int h = 0; h < kBI; ++h) {
                 uint32_t mm[NS];
@@ -513,6 +523,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                         for (int q = 0; q < U2; ++q) acc[k] += a[k][q];
                 }
             }
+            BPROF(BR_OGATH);
             if (MODE == B_PULL) {
                 // Alg.1 l.20-25: lanes with a non-zero masked sum are discovered on this level
                 MT newm = 0;
@@ -559,7 +570,11 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                     if (fl & 1) atomicOr(&fr_out[v], m);
                 }
             }
+            BPROF(BR_OEPI);
         }
+#ifdef TBC_PROF
+        if (lane == 0) atomicAdd(&P.gctr->prof[16 + MODE], (unsigned long long)n_own);
+#endif
         if (MODE == B_PULL) {
             __syncwarp();
             bool cl[kBI];
@@ -658,19 +673,28 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
     const unsigned long long t_kernel0 = clock64();
 #endif
     for (int64_t b = part; b < nb; b += MULTI ? S.nparts : 1) {
+      // the batch's lane sets still to run: all W lanes, or -- after a level list or its tile starts
+      // outgrew the workspace (BOut::ovf) -- the two halves of the set that overflowed (a single
+      // source always fits: batch_alloc sizes the lists for at least n entries)
+      MT pend[8];
+      int npend = 0;
+      pend[npend++] = ~(MT)0;
+      unsigned valid = 0;  // thread 0 of CTA 0: valid sources of the lane set being run
+      while (npend > 0) {
+        const MT bmask = pend[--npend];
         // ---------------- level 0: the batch's sources (Alg.1 l.15-18): source b*W + 32k + l is
         // lane l's source k; a vertex repeated in the batch is appended once, by its lowest source
         if (cta0 && tid < 32) {
             int32_t s[NS];
-            unsigned valid = 0;
+            valid = 0;
 #pragma unroll
             for (int k = 0; k < NS; ++k) {
                 const int64_t si = b * W + 32 * k + lane;
                 s[k] = -1;
-                if (si < P.k) {
+                if (si < P.k && ((bmask >> (32 * k + lane)) & 1u)) {
                     const int32_t sc = P.sources[si];
                     if (sc >= 0 && sc < P.n) s[k] = (P.perm && !P.src_internal) ? P.perm[sc] : sc;
-                    else atomicAdd(&C->bad_sources, 1ull);
+                    else if (bmask == ~(MT)0) atomicAdd(&C->bad_sources, 1ull);
                 }
                 if (s[k] >= 0) {
                     atomicOr(&fr[0][s[k]], (MT)1 << (32 * k + lane));
@@ -715,7 +739,6 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
                 C->ilist = 0;
                 C->cand[0] = 0;
                 C->dyn[0] = C->dyn[1] = 0;
-                C->st_sources += valid;
             }
         }
         unsigned ph = 0;  // edge passes of this batch so far (selects the dynamic-tile counter)
@@ -733,6 +756,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
         int d = 0;
         MT active = ~(MT)0;
         int64_t fwd_edges = 0, pulls = 0;
+        bool overflow = false;
         for (;;) {
             // direction of level d+1 (uniform: every CTA computes it from the same snapshot)
             const bool pull = d + 1 >= 2 && P.dir_mode != 1 &&
@@ -768,7 +792,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
                 }
                 if (pull) {  // candidates: vertices with in-edges and an unvisited active lane
                     const BOut co{&C->cand[0], P.cand_v, P.cand_pre, P.cand_beg, P.cand_tiles, P.n + kPad,
-                                  P.cand_tiles_cap};
+                                  P.cand_tiles_cap, &C->ovf};
                     for (int64_t base = gwarp * kBT; base < P.n_scan; base += nwarps * kBT) {
                         bool tk[kBI];
                         int32_t vv[kBI];
@@ -801,7 +825,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             }
             Lv nxt{cur.p0 + cur.N, 0, 0, cur.tb + cdiv(cur.N + cur.E, kBT)};
             const BOut lo{&C->list, P.list_v + nxt.p0, P.list_pre + nxt.p0, P.list_beg + nxt.p0, P.tiles + nxt.tb,
-                          P.list_cap - nxt.p0, P.tiles_cap - nxt.tb};
+                          P.list_cap - nxt.p0, P.tiles_cap - nxt.tb, &C->ovf};
             MT *fro = fr[(d + 1) & 1];
             if (cta0 && tid == 0) C->dyn[(ph + 1) & 1] = 0;  // the next pass's counter (its last user is done)
             if (pull) {
@@ -818,6 +842,10 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             }
             ++ph;
             bsync(C, gen, ncta);
+            if (*(volatile unsigned *)&C->ovf) {  // level d+1 did not fit (uniform: read after the barrier)
+                overflow = true;
+                break;
+            }
             {
                 const unsigned long long lv = ld_volatile_u64(&C->snap[0]);
                 nxt.N = (int64_t)(lv >> P.ebits);
@@ -835,6 +863,30 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             prev = cur;
             cur = nxt;
         }
+        if (overflow) {
+            // drop the lane set's partial forward state (grid-wide, no list needed), then run its halves
+            for (int64_t i = gtid; i < P.n * W; i += nthreads) P.sig[i] = 0.0;
+            for (int64_t i = gtid; i < P.n; i += nthreads) {
+                vis[i] = 0;
+                fr[0][i] = 0;
+                fr[1][i] = 0;
+            }
+            bsync(C, gen, ncta);
+            if (cta0 && tid == 0) {  // every CTA has read the flag (before the barrier above)
+                C->ovf = 0;
+                C->st_overflows += 1;
+                C->ovf_total += 1;
+            }
+            MT lo = 0, x = bmask;
+            for (int i = __popcll((unsigned long long)bmask) / 2; i > 0; --i) {
+                lo |= x & (~x + 1);
+                x &= x - 1;
+            }
+            if (lo == 0 || npend + 2 > 8) __trap();  // one source always fits (batch_alloc)
+            pend[npend++] = bmask ^ lo;
+            pend[npend++] = lo;
+            continue;
+        }
         const int D = d;  // deepest non-empty level of the batch
         if (cta0 && tid == 0) {
             C->st_levels += D + 2;
@@ -849,7 +901,10 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
                 const int64_t *l = P.lvl + 4 * (int64_t)L;
                 bclear<W, true>(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps, L, b);
             }
-            if (cta0 && tid == 0) C->st_scans += pulls;
+            if (cta0 && tid == 0) {
+                C->st_scans += pulls;
+                C->st_sources += valid;
+            }
             bsync(C, gen, ncta);
             continue;
         }
@@ -858,7 +913,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
         for (int L = D; L >= 1; --L) {
             const int64_t *l = P.lvl + 4 * (int64_t)L;
             const Lv lv{l[0], l[1], l[2], l[3]};
-            const BOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0};
+            const BOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0, nullptr};
             if (cta0 && tid == 0) C->dyn[(ph + 1) & 1] = 0;  // the next pass's counter (its last user is done)
             bpass<B_BWD, W>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.list_beg + lv.p0, list_m + lv.p0,
                          P.tiles + lv.tb, lv.N, lv.E, P.out_idx, fr[(L + 1) & 1], fr[L & 1], 0u, gwarp, nwarps, none,
@@ -882,15 +937,17 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
         if (cta0 && tid == 0) {
             C->st_bwd_edges += bwd_edges;
             C->st_scans += pulls;
+            C->st_sources += valid;
         }
         bsync(C, gen, ncta);
         btrace(P, tr, 5, 0, 0, 0, 0, 0);
+      }
     }
 #ifdef TBC_PROF
     if ((tid & 31) == 0) {
         unsigned long long busy = 0;
         for (int r = 0; r < BR_OTHER; ++r) busy += tbc_bprof[tid >> 5][r];
-        for (int r = BR_WIN; r <= BR_OWN; ++r) busy += tbc_bprof[tid >> 5][r];
+        for (int r = BR_WIN; r <= BR_OEPI; ++r) busy += tbc_bprof[tid >> 5][r];
         tbc_bprof[tid >> 5][BR_OTHER] = clock64() - t_kernel0 - busy;
         for (int r = 0; r < BR_SLOTS; ++r) atomicAdd(&P.gctr->prof[r], tbc_bprof[tid >> 5][r]);
     }
@@ -915,11 +972,14 @@ static tbc_status batch_alloc(tbc_graph *g, int q, int W) {
         if (r == cudaSuccess) w.bytes += bytes;
         return r;
     };
-    // every (vertex, level) pair of a batch has at least one source: <= W n list entries, and the
-    // levels' tiles sum to <= (W n + W m) / kBT + (levels <= n + 1)
+    // level lists: a batch uses one entry per (vertex, level) with any of its sources on it -- at most
+    // W n, but about n on low-diameter graphs (cfg 3: 1.07 n); sized at blist_factor n (>= n: one
+    // source always fits) and grown by the next call after a sweep overflowed (k_bcb re-runs it in
+    // halves).  Tile starts: <= (entries + their out-edges) / kBT + one partial tile per level.
     w.width = W;
-    w.list_cap = (int64_t)W * n + kPad;
-    w.tiles_cap = ((int64_t)W * (n + m)) / kBT + n + 2 + kPad;
+    const int64_t f = g->blist_factor < W ? g->blist_factor : W;
+    w.list_cap = f * n + kPad;
+    w.tiles_cap = (w.list_cap + f * m) / kBT + n + 2 + kPad;
     w.cand_tiles_cap = (n + m) / kBT + 2 + kPad;
     if ((e = alloc(&w.sig, (size_t)n * W)) || (e = alloc(&w.du, (size_t)n * W)) || (e = alloc(&w.vis, n * nw)) ||
         (e = alloc(&w.fr[0], n * nw)) || (e = alloc(&w.fr[1], n * nw)) || (e = alloc(&w.list_v, w.list_cap)) ||
@@ -981,8 +1041,9 @@ void batch_free(tbc_graph *g) {
 // back to 32 if the W = 64 workspace then fails to allocate (batch_run).
 static int64_t batch_ws_bytes(const tbc_graph *g, int W) {  // batch_alloc's sizes, one partition
     const int64_t n = g->n, m = g->m, nw = W / 32;
-    const int64_t list_cap = (int64_t)W * n + kPad;
-    const int64_t tiles_cap = ((int64_t)W * (n + m)) / kBT + n + 2 + kPad;
+    const int64_t f = g->blist_factor < W ? g->blist_factor : W;
+    const int64_t list_cap = f * n + kPad;
+    const int64_t tiles_cap = (list_cap + f * m) / kBT + n + 2 + kPad;
     return 16 * W * n + 12 * n * nw + list_cap * (12 + 4 * nw) + 4 * tiles_cap + 16 * (n + kPad) +
            4 * ((n + m) / kBT + 2 + kPad) + 32 * (n + 2) + (int64_t)sizeof(Ctrs);
 }
@@ -1094,6 +1155,15 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
                      int32_t *bfs_depth, double *bfs_sigma) {
     int W = batch_width(g);
     const int32_t *src = d_sources;
+    {  // sweeps of earlier calls that outgrew the level lists: grow them (x2) before this call
+        unsigned long long seen = 0;
+        for (int q = 0; q < kMaxPartitions; ++q) seen += g->h_bovf ? g->h_bovf[q] : 0;
+        if (seen > g->bovf_seen && g->blist_factor < W) {
+            g->blist_factor *= 2;
+            for (int q = 0; q < kMaxPartitions; ++q) batch_free_one(g, q);
+        }
+        g->bovf_seen = seen;
+    }
     // tbc_bfs_batch exports per list index: batches are cut from the list as given
     const bool grouped = g->batch_order && k > 1 && k < (1ll << 31) && !bfs_depth;
     if (grouped) {
@@ -1182,6 +1252,14 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
                             : (W == 64 ? (const void *)k_bcb<64, false> : (const void *)k_bcb<32, false>);
     cudaError_t e = cudaLaunchCooperativeKernel(fn, dim3(S.cta_per_part * np), dim3(kBB), args, kBSmem, stream);
     if (e != cudaSuccess) return cuda_error(e, "cudaLaunchCooperativeKernel(k_bcb)");
+    if (!g->h_bovf && (e = cudaMallocHost(&g->h_bovf, sizeof(unsigned long long) * kMaxPartitions)) == cudaSuccess)
+        for (int q = 0; q < kMaxPartitions; ++q) g->h_bovf[q] = 0;
+    (void)cudaGetLastError();
+    if (g->h_bovf)  // overflow totals, read by the next call (no synchronisation here)
+        for (int q = 0; q < np; ++q)
+            if ((e = cudaMemcpyAsync(&g->h_bovf[q], &g->bws[q].ctr->ovf_total, sizeof(unsigned long long),
+                                     cudaMemcpyDeviceToHost, stream)))
+                return cuda_error(e, "overflow counter copy");
     return TBC_OK;
 }
 

@@ -30,10 +30,12 @@ struct Ctrs {
     unsigned long long snap[4];
     unsigned long long bad_sources;
     unsigned long long dyn[2];    // batched engine: dynamic tile counters of consecutive edge passes
+    unsigned int ovf;             // batched engine: a level list outgrew the workspace (re-run in halves)
+    unsigned long long ovf_total; // batched engine: such re-runs since the workspace was allocated
     unsigned long long trace_n;   // entries written to the trace buffer
     // accumulated statistics (tbc_stats)
     long long st_sources, st_reached, st_reached_edges, st_fwd_edges, st_bwd_edges, st_levels, st_pull_levels,
-        st_scans, st_max_depth, st_list_peak;
+        st_scans, st_max_depth, st_list_peak, st_overflows;
     unsigned long long prof[32];  // TBC_PROF builds: warp-cycles per code region (gctr only)
 };
 
@@ -218,6 +220,9 @@ struct tbc_graph {
     int bgrid = 0;
     int auto_width = 0;           // batch width the auto rule settled on for this graph (0: not yet)
     int last_width = 0, last_parts = 0;  // of the latest batched call (tbc_stats)
+    int64_t blist_factor = 2;     // batched engine: level-list entries per vertex allocated (grows x2)
+    unsigned long long *h_bovf = nullptr;  // pinned: per-partition overflow totals after the latest call
+    unsigned long long bovf_seen = 0;
     int32_t *bfs_depth = nullptr; // tbc_bfs_batch device outputs (grow-only)
     double *bfs_sigma = nullptr;
     int64_t bfs_cap = 0;          // elements of bfs_depth / bfs_sigma

@@ -260,3 +260,27 @@ def test_dist_bc_real_kernel(tmp_path, backend, world):
     # each rank ran only its contiguous slice, twice (host and device API)
     from paper_conf_icppw_artiless21_b200 import dist as tdist
     assert per_rank == [2 * (hi - lo) for lo, hi in (tdist.partition(len(src), world, r) for r in range(world))]
+
+
+@pytest.mark.parametrize("width", [32, 64])
+def test_batched_list_overflow_reruns_halves(width):
+    """Level lists sized below a sweep's need (TBC_OPT_BATCH_LIST = 1 on a deep lattice, where the W
+    sources of a sweep sit on different levels): k_bcb re-runs overflowing sweeps as halves, bc stays
+    exact, the overflow is reported, and the next call grows the lists."""
+    g = gg.road_lattice(128, 0.10, seed=4)
+    src = gg.sources(g, 70, seed=2)
+    want = oracle.bc(g.col_ptr, g.row_idx, False, src)
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+        G.set_batch(tbc.ENGINE_BATCHED)
+        G.set_batch_width(width)
+        G.set_batch_parts(1)
+        G.set_batch_list(1)
+        assert_bc(G.bc(src), want)
+        st = G.stats()
+        assert st["list_overflows"] > 0 and st["sources"] == len(src)
+        depth, sigma = G.bfs_batch(src[:9])
+        assert_bfs_rows(g, src[:9], depth, sigma)
+        for _ in range(8):  # the lists grow call by call until a sweep fits
+            G.reset_stats()
+            assert_bc(G.bc(src), want)
+        assert G.stats()["list_overflows"] == 0

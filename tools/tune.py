@@ -91,9 +91,11 @@ for setting in a.settings.split(";"):
         tot = sum(pr.values()) or 1
         if int(kv.get("batch", 1)):
             names = ["barrier", "bphase", "r2", "r3", "r4", "retire", "other", "r7",
-                     "tile_window", "tile_index", "tile_append", "tile_owners"]
-            pr = {**{n: v for n, v in zip(names, pr.values()) if not n.startswith("r")},
-                  **{k: v for k, v in pr.items() if k.startswith("b_")}}
+                     "tile_window", "tile_index", "tile_append", "tile_owners", "owner_gather", "owner_epilogue"]
+            vals = list(pr.values())
+            pr = {**{n: v for n, v in zip(names, vals) if not n.startswith("r")},
+                  **{k: v for k, v in pr.items() if k.startswith("b_")},
+                  "b_owners_push": vals[16], "b_owners_pull": vals[17], "b_owners_bwd": vals[18]}
         reg = {k: v for k, v in pr.items() if not k.startswith("b_")}
         tot = sum(reg.values()) or 1
         print("PROFILE " + setting + " " + " ".join(f"{k}={100 * v / tot:.1f}" for k, v in reg.items() if v), flush=True)

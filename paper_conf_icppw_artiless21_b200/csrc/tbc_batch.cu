@@ -1024,6 +1024,10 @@ void batch_free_one(tbc_graph *g, int q) {
     for (void *p : ps) cudaFree(p);
     g->device_bytes -= w.bytes;
     w = BatchWorkspace{};
+    // the partition's overflow total restarts with its counters (after cudaFree: a copy still in
+    // flight from the last launch has landed by now)
+    if (g->h_bovf) g->h_bovf[q] = 0;
+    g->bovf_seen[q] = 0;
 }
 
 void batch_free(tbc_graph *g) {
@@ -1156,13 +1160,13 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
     int W = batch_width(g);
     const int32_t *src = d_sources;
     {  // sweeps of earlier calls that outgrew the level lists: grow them (x2) before this call
-        unsigned long long seen = 0;
-        for (int q = 0; q < kMaxPartitions; ++q) seen += g->h_bovf ? g->h_bovf[q] : 0;
-        if (seen > g->bovf_seen && g->blist_factor < W) {
+        bool grew = false;
+        for (int q = 0; q < kMaxPartitions; ++q) grew |= g->h_bovf && g->h_bovf[q] > g->bovf_seen[q];
+        if (grew && g->blist_factor < W) {
             g->blist_factor *= 2;
-            for (int q = 0; q < kMaxPartitions; ++q) batch_free_one(g, q);
+            for (int q = 0; q < kMaxPartitions; ++q) batch_free_one(g, q);  // reallocated below
         }
-        g->bovf_seen = seen;
+        for (int q = 0; q < kMaxPartitions; ++q) g->bovf_seen[q] = g->h_bovf ? g->h_bovf[q] : 0;
     }
     // tbc_bfs_batch exports per list index: batches are cut from the list as given
     const bool grouped = g->batch_order && k > 1 && k < (1ll << 31) && !bfs_depth;

@@ -203,12 +203,41 @@ def kronecker(scale: int, edgefactor: int, seed: int, directed: bool, device: st
     perm = torch.sort(mix64(torch.arange(n, dtype=torch.int64, device=device) + key_perm), stable=True).indices
     src = perm[src]
     dst = perm[dst]
+    del perm
     if device == "cpu":
-        cp, ri = csc_from_edges(n, src.numpy(), dst.numpy(), directed)
+        cp, ri = _csc_lean_host(n, src, dst, directed)
     else:
         cp, ri = csc_from_edges_torch(n, src, dst, directed)
     kind = "dir" if directed else "undir"
     return Graph(f"kron_s{scale}_ef{edgefactor}_{kind}_seed{seed}", n, cp, ri, directed)
+
+
+def _csc_lean_host(n: int, src, dst, directed: bool):
+    """csc_from_edges for large host tensors with a small memory peak: keys (column-major) built
+    in place, sorted in place, duplicates compressed out.  Same result as csc_from_edges_torch."""
+    s = src.numpy()
+    d = dst.numpy()
+    keep = s != d
+    m = int(keep.sum())
+    key = np.empty(m if directed else 2 * m, dtype=np.int64)
+    np.multiply(d[keep], n, out=key[:m])
+    key[:m] += s[keep]
+    if not directed:
+        np.multiply(s[keep], n, out=key[m:])
+        key[m:] += d[keep]
+    del s, d, keep, src, dst
+    key.sort()  # introsort, in place (no second copy of the keys)
+    uniq = np.empty(key.size, dtype=bool)
+    uniq[:1] = True
+    np.not_equal(key[1:], key[:-1], out=uniq[1:])
+    key = key[uniq]
+    del uniq
+    col = key // n
+    row = (key - col * n).astype(np.int32)
+    del key
+    col_ptr = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(np.bincount(col, minlength=n), out=col_ptr[1:])
+    return col_ptr, row
 
 
 def road_lattice(side: int, q: float, seed: int) -> Graph:

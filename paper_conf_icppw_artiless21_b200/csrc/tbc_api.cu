@@ -739,11 +739,13 @@ tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
     out->probe_width = (int64_t)g->probe_width;
     for (int q = 0; q < kMaxPartitions; ++q) out->workspace_bytes += (int64_t)g->bws[q].bytes;
     out->workspace_bytes += (int64_t)g->ws_bytes + (int64_t)g->sws.bytes;
-    for (int i = 0; i < g->ws_count + kMaxPartitions + 1; ++i) {  // per-source, batched, narrow-level
+    for (int i = 0; i < g->ws_count + kMaxPartitions + 2; ++i) {  // per-source, batched, narrow-level, retired
         Ctrs *src = i < g->ws_count ? g->ws[i].ctr
-                    : i < g->ws_count + kMaxPartitions ? g->bws[i - g->ws_count].ctr : g->sws.ctr;
-        if (!src) continue;
-        TBC_CUDA(cudaMemcpy(&c, src, sizeof c, cudaMemcpyDeviceToHost));
+                    : i < g->ws_count + kMaxPartitions ? g->bws[i - g->ws_count].ctr
+                    : i == g->ws_count + kMaxPartitions ? g->sws.ctr : nullptr;
+        if (i == g->ws_count + kMaxPartitions + 1) c = g->retired;
+        else if (!src) continue;
+        else TBC_CUDA(cudaMemcpy(&c, src, sizeof c, cudaMemcpyDeviceToHost));
         out->bad_sources += (int64_t)c.bad_sources;
         if (c.st_list_peak > out->list_peak) out->list_peak = c.st_list_peak;
         out->list_overflows += c.st_overflows;
@@ -814,6 +816,7 @@ tbc_status tbc_stats_reset(tbc_graph *g) {
         TBC_CUDA(cudaMemset(&c->st_sources, 0, kStatBytes));  // st_sources .. st_overflows
         TBC_CUDA(cudaMemset(&c->bad_sources, 0, sizeof(unsigned long long)));
     }
+    g->retired = Ctrs{};
     return TBC_OK;
 fail:
     return st;

@@ -1019,6 +1019,24 @@ static tbc_status batch_alloc(tbc_graph *g, int q, int W) {
 
 void batch_free_one(tbc_graph *g, int q) {
     BatchWorkspace &w = g->bws[q];
+    if (w.ctr) {  // keep the partition's accumulated statistics (tbc_stats) across a reallocation
+        Ctrs c;
+        if (cudaMemcpy(&c, w.ctr, sizeof c, cudaMemcpyDeviceToHost) == cudaSuccess) {
+            g->retired.st_sources += c.st_sources;
+            g->retired.st_reached += c.st_reached;
+            g->retired.st_reached_edges += c.st_reached_edges;
+            g->retired.st_fwd_edges += c.st_fwd_edges;
+            g->retired.st_bwd_edges += c.st_bwd_edges;
+            g->retired.st_levels += c.st_levels;
+            g->retired.st_pull_levels += c.st_pull_levels;
+            g->retired.st_scans += c.st_scans;
+            g->retired.st_overflows += c.st_overflows;
+            g->retired.bad_sources += c.bad_sources;
+            if (c.st_max_depth > g->retired.st_max_depth) g->retired.st_max_depth = c.st_max_depth;
+            if (c.st_list_peak > g->retired.st_list_peak) g->retired.st_list_peak = c.st_list_peak;
+        }
+        (void)cudaGetLastError();
+    }
     void *ps[] = {w.sig, w.du, w.vis, w.fr[0], w.fr[1], w.list_v, w.list_pre, w.list_beg, w.list_m, w.tiles,
                   w.cand_v, w.cand_pre, w.cand_beg, w.cand_tiles, w.lvl, w.ctr};
     for (void *p : ps) cudaFree(p);

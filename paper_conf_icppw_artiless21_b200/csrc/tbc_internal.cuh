@@ -223,6 +223,7 @@ struct tbc_graph {
     int64_t blist_factor = 2;     // batched engine: level-list entries per vertex allocated (grows x2)
     unsigned long long *h_bovf = nullptr;  // pinned: per-partition overflow totals after the latest call
     unsigned long long bovf_seen[tbc::kMaxPartitions] = {};
+    tbc::Ctrs retired = {};       // statistics of freed batched workspaces (kept for tbc_stats)
     int32_t *bfs_depth = nullptr; // tbc_bfs_batch device outputs (grow-only)
     double *bfs_sigma = nullptr;
     int64_t bfs_cap = 0;          // elements of bfs_depth / bfs_sigma

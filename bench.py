@@ -29,7 +29,8 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "BC GTEPS and sec/source at 1/2/4/8 B200; HBM GB/s fraction of peak"
-SOURCES_PER_GPU = {1: 1024, 2: 1024, 3: 4096, 4: 1024, 5: 1024, 6: None, 7: 1024}
+# the configs' source lists (BASELINE.json configs); strong scaling splits them over the ranks
+SOURCES_TOTAL = {1: 1024, 2: 1024, 3: 4096, 4: 1024, 5: 8192, 6: None, 7: 1024}
 # the paper's printed figure for the SAME workload (context: Titan Xp), GTEPS
 PAPER_GTEPS = {6: (10.257, "Table 5 P:452: exact BC of mycielski16, 159.8 s, 10,257 MTEPs on a Titan Xp"),
                7: (18.470, "Table 3 P:380: one source of mycielski19, 48.9 ms, 18,470 MTEPs on a Titan Xp")}
@@ -42,7 +43,12 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", type=int, default=3)
-    ap.add_argument("--sources", type=int, default=None, help="sources per GPU (default: the config's)")
+    ap.add_argument("--sources", type=int, default=None,
+                    help="sources per step (strong) or per GPU (weak); default: the config's list")
+    ap.add_argument("--scaling", choices=["strong", "weak"], default="strong",
+                    help="strong: the config's list split over the ranks; weak: that many per rank")
+    ap.add_argument("--assign", choices=["contiguous", "interleaved"], default="contiguous",
+                    help="rank r takes a contiguous range of the list, or every world-th source")
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=None, help="sources in the CPU-oracle sample")
@@ -130,17 +136,33 @@ def source_list(g, cfg, total):
     return gg.sources(g, total, seed=gg.CONFIGS[cfg]["src_seed"])
 
 
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
+
+
 def cpu_baseline(g, sources, sample):
-    """The oracle as it stands on this host's cores, bounded sample of the same workload."""
+    """The oracle as it stands on this host's cores, bounded sample of the same workload: all-core
+    throughput (one source per thread) and the single-thread sec/source (the comparator of the
+    paper's "(sequential)x", P:326, P:332)."""
     import oracle
     cores = os.cpu_count() or 1
     k = sample or min(max(cores, 4), 64)
     src = sources[:k]
     _, secs = oracle.bc_timed(g.col_ptr, g.row_idx, g.directed, src, nthreads=min(cores, k))
+    k1 = 2 if g.nnz > 2e8 else 4
+    _, secs1 = oracle.bc_timed(g.col_ptr, g.row_idx, g.directed, sources[:k1], nthreads=1)
     return {"value": k * g.nnz / secs / 1e9, "unit": "GTEPS", "cores": min(cores, k), "kind": "oracle",
             "sample": f"{k} sources of the same graph (first {k} of the rank-0 source list), "
-                      f"{secs:.2f} s of C Brandes oracle, one source per thread, graph build excluded",
-            "sec_per_source": secs / k}
+                      f"{secs:.2f} s of C Brandes oracle, one source per thread, graph build excluded; "
+                      f"single-thread: {k1} sources in {secs1:.2f} s",
+            "sec_per_source": secs / k, "single_thread_sec_per_source": secs1 / k1,
+            "cpu_model": cpu_model(), "host_cores": cores}
 
 
 def run_reference(args):
@@ -153,8 +175,8 @@ def run_reference(args):
     if args.config in EXACT:
         srcs = np.arange(g.n, dtype=np.int32)
     else:
-        per_gpu = args.sources or SOURCES_PER_GPU[args.config]
-        srcs = source_list(g, args.config, per_gpu * args.gpus)
+        total = args.sources or SOURCES_TOTAL[args.config]
+        srcs = source_list(g, args.config, total * (args.gpus if args.scaling == "weak" else 1))
     cores = os.cpu_count() or 1
     k = args.cpu_sample or min(max(cores, 4), 64)
     times = []
@@ -167,7 +189,7 @@ def run_reference(args):
     val = g.nnz / spp / 1e9
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "GTEPS", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": spp * k * 1e3,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f64",
             "data": "synthetic", "sec_per_source": spp,
             "config": {"workload": _workload_name(args.config), "n": g.n, "m": g.nnz,
                        "sources_per_step": k},
@@ -185,6 +207,23 @@ def _gen_device():
 def _workload_name(cfg):
     import graphgen as gg
     return gg.CONFIGS[cfg]["name"]
+
+
+def traffic_signature(cfg, engine, k, eng, width):
+    """Key of a measured-traffic file: the exact launch (workload, engine, sources per launch, W)."""
+    return f"cfg{cfg}_{engine}_k{k}_e{eng}_w{width}"
+
+
+def load_traffic(sig):
+    """DRAM bytes of the exact launch from tools/measure_traffic.py (an ncu capture of this launch
+    configuration, committed under profiles/), or None."""
+    path = os.path.join(ROOT, "profiles", f"traffic_{sig}.json")
+    if not os.path.exists(path):
+        return None, None
+    try:
+        return json.load(open(path)), os.path.relpath(path, ROOT)
+    except Exception:
+        return None, None
 
 
 def main():
@@ -206,20 +245,26 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("NCCL_DEBUG", "INFO")  # communicator init lines: the rank count is on record
         dist.init_process_group("nccl", device_id=dev)
 
     g, gen_s = make_graph(args.config, "cuda")
-    if args.config in EXACT:  # exact BC: all n sources per step, split across the ranks
+    # the source list and this rank's share: strong scaling splits the config's list
+    # over the ranks, weak scaling gives every rank a list of that size
+    if args.config in EXACT:  # exact BC: all n sources per step
         all_src = np.arange(g.n, dtype=np.int32)
-        my_src = np.array_split(all_src, world)[rank]
-        per_gpu = len(my_src)
-        n_sources = g.n
     else:
-        per_gpu = args.sources or SOURCES_PER_GPU[args.config]
-        all_src = source_list(g, args.config, per_gpu * world)
-        lo, hi = rank * per_gpu, (rank + 1) * per_gpu
+        total = args.sources or SOURCES_TOTAL[args.config]
+        if args.scaling == "weak":
+            total *= world
+        all_src = source_list(g, args.config, total)
+    n_sources = len(all_src)
+    if args.assign == "interleaved":
+        my_src = all_src[rank::world]
+    else:
+        lo, hi = tdist.partition(n_sources, world, rank)
         my_src = all_src[lo:hi]
-        n_sources = per_gpu * world
+    per_gpu = len(my_src)
     t0 = time.time()
     engine = tbc.ENGINE_COOT if args.engine == "coot" else tbc.ENGINE_CSC
     G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, engine=engine, device=local)
@@ -231,7 +276,7 @@ def main():
     G.set_batch_order(args.order)
     if args.cost:
         G.set_cost(**{k: float(v) for k, v in (kv.split("=") for kv in args.cost.split(","))})
-    src_d = torch.from_numpy(my_src).to(dev)
+    src_d = torch.from_numpy(np.ascontiguousarray(my_src)).to(dev)
     bc = torch.zeros(g.n, dtype=torch.float64, device=dev)
     stream = torch.cuda.current_stream(dev)
 
@@ -266,10 +311,16 @@ def main():
     step_ms = [a.elapsed_time(b) for a, b in ev]
     kern_ms = [a.elapsed_time(b) for a, b in kev]
     total_ms = sum(step_ms)
+    busy_ms = sum(kern_ms)  # this rank's time in the hot path (its source slice)
+    busy = [busy_ms]
     if world > 1:
         t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
+        bt = torch.zeros(world, dtype=torch.float64, device=dev)
+        bt[rank] = busy_ms
+        dist.all_reduce(bt, op=dist.ReduceOp.SUM)
+        busy = bt.tolist()
     st = G.stats()
     eng = st["engine"] if args.engine == "csc" else 0
     batched = eng == 1
@@ -278,27 +329,32 @@ def main():
     gteps = sources_total * g.nnz / (total_ms / 1e3) / 1e9
     ms_per_step = total_ms / args.steps
 
-    # roofline of the hot-path kernel (k_bcb batched, or k_bc per source): SURVEY 8(d) algorithmic bytes
-    # B_min = 8 B per out-edge of the reached set (4 B index read once per stage) + 80 B per
-    # reached vertex, summed over the launch's sources; / the kernel's event-timed duration.
+    # roofline of the hot-path kernel: SURVEY 8(d) algorithmic bytes B_min = 8 B per
+    # out-edge of the reached set (4 B index read once per stage) + 80 B per reached vertex, summed
+    # over the launch's sources, / the kernel's event-timed duration on its stream.  The batched
+    # engine shares the index stream between the W sources of a sweep, so its own compulsory
+    # traffic is 8 B per reached edge / W + 80 B per reached (vertex, source).
     alg_bytes_per_launch = (8.0 * st["reached_edges"] + 80.0 * st["reached"]) / args.steps
-    # the batched engine's own compulsory traffic: the index stream once per stage per BATCH of W
-    # sources (8 B per reached edge / W per source) + the per-(vertex, source) state (80 B)
-    # mirrors csrc/tbc_batch.cu batch_width (64 up to 8 M vertices, or average degree >= 8 when the
-    # W = 64 workspace fits the device; the library's exact rule uses the free memory at the call)
     wdt = st["batch_width"] if batched else 1
     alg_bytes_batched = (8.0 * st["reached_edges"] / wdt + 80.0 * st["reached"]) / args.steps
     k_avg_s = statistics.mean(kern_ms) / 1e3
     peak, peak_kind = peaks()
     achieved = alg_bytes_per_launch / k_avg_s / 1e9
-    traffic = None
-    tpath = os.path.join(ROOT, "profiles", f"traffic_cfg{args.config}_{kname}.json")
-    if os.path.exists(tpath):
-        try:
-            tj = json.load(open(tpath))
-            traffic = tj["dram_bytes_per_source"] * per_gpu
-        except Exception:
-            traffic = None
+    # measured DRAM bytes of this exact launch (ncu, profiles/traffic_<signature>.json)
+    sig = traffic_signature(args.config, args.engine, per_gpu, eng, wdt)
+    tj, tpath = load_traffic(sig)
+    traffic = hbm = None
+    stages = None
+    if tj:
+        traffic = tj["full"]["dram_bytes"]
+        hbm = traffic / k_avg_s / 1e9 / peak
+        if tj.get("forward"):
+            fw, fu = tj["forward"], tj["full"]
+            stages = {"forward_bytes": fw["dram_bytes"], "forward_ms": fw["ms"],
+                      "backward_bytes": fu["dram_bytes"] - fw["dram_bytes"], "backward_ms": fu["ms"] - fw["ms"],
+                      "forward_hbm_frac": fw["dram_bytes"] / (fw["ms"] / 1e3) / 1e9 / peak,
+                      "backward_hbm_frac": (fu["dram_bytes"] - fw["dram_bytes"]) / ((fu["ms"] - fw["ms"]) / 1e3)
+                      / 1e9 / peak if fu["ms"] > fw["ms"] else None}
 
     # end to end through the public host API: H2D sources, run, all-reduce, D2H bc
     e2e_times = []
@@ -325,15 +381,18 @@ def main():
         line = {
             "metric": METRIC, "value": gteps, "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-            "scaling": "strong" if args.config in EXACT else "weak",
+            "scaling": "strong" if (args.config in EXACT or args.scaling == "strong") else "weak",
             "vs_baseline": gteps / PAPER_GTEPS[args.config][0] if args.config in PAPER_GTEPS else None,
             "dtype": "f64", "data": "synthetic",
             "sec_per_source": total_ms / 1e3 / sources_total,
             "config": {"workload": _workload_name(args.config), "n": g.n, "m": g.nnz,
-                       "directed": g.directed, "engine": args.engine, "sources_per_gpu": per_gpu,
+                       "directed": g.directed, "engine": args.engine, "sources_per_step": n_sources,
+                       "sources_per_gpu": per_gpu, "assign": args.assign,
                        "parallelism": f"source-partitioned x{world}, graph replicated, 1 NCCL all-reduce/step",
                        "l2": "inputs larger than L2 (CSC+CSR %.0f MB vs 126 MB L2); no flush" %
-                             ((8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) / 1e6),
+                             ((8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) / 1e6)
+                             if (8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) > 126e6 else
+                             "graph fits in L2 (small config); no flush",
                        "direction": args.direction, "format": args.format, "engine_kind": args.engine,
                        "engine_mode": (f"batched, {wdt} sources per sweep, {st['batch_parts']} SM partition(s)"
                                        + (", sources grouped by 2-hop out-volume" if args.order
@@ -345,28 +404,40 @@ def main():
                        "paper": PAPER_GTEPS[args.config][1] if args.config in PAPER_GTEPS else None,
                        "cost": args.cost},
             "clocks": clocks,
-            "gpu_launches": args.steps,
+            "gpu_launches": args.steps * (2 if eng == 2 else 1),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
                          "kernel": kname, "alg_bytes_per_launch": alg_bytes_per_launch,
                          "model": "SURVEY 8(d) B_min = 8 B per reached edge + 80 B per reached vertex, per "
-                                  "source; a batch shares the index stream, so frac may exceed 1",
+                                  "source (B_min-equivalent throughput); a batch shares the index stream, so "
+                                  "frac may exceed 1",
+                         "b_min_equiv_frac": achieved / peak,
+                         "hbm_frac": hbm,
+                         "hbm_frac_def": "ncu dram__bytes_read+write of this exact launch / its event-timed "
+                                         "duration / peak" if hbm is not None else
+                                         f"no measured traffic for launch {sig} (tools/measure_traffic.py)",
+                         "traffic_file": tpath, "stages": stages,
                          "achieved_batched_model": alg_bytes_batched / k_avg_s / 1e9,
                          "frac_batched_model": alg_bytes_batched / k_avg_s / 1e9 / peak,
                          "kernel_ms": statistics.mean(kern_ms)},
             "e2e": {"value": e2e_gteps, "unit": "GTEPS", "h2d_bytes_per_step": 4 * len(my_src),
                     "d2h_bytes_per_step": 8 * g.n},
             "cpu_baseline": cpu,
+            "ranks": {"busy_ms_max": max(busy), "busy_ms_mean": statistics.mean(busy),
+                      "imbalance": max(busy) / statistics.mean(busy) - 1.0 if statistics.mean(busy) > 0 else 0.0,
+                      "busy_ms": busy},
             "traversal": {"reached_per_source": st["reached"] / max(st["sources"], 1),
                           "reached_edges_per_source": st["reached_edges"] / max(st["sources"], 1),
                           "fwd_edges_per_source": st["fwd_edges"] / max(st["sources"], 1),
                           "bwd_edges_per_source": st["bwd_edges"] / max(st["sources"], 1),
                           "levels_per_source": st["levels"] / max(st["sources"], 1),
                           "pull_levels_per_source": st["pull_levels"] / max(st["sources"], 1),
+                          "list_peak": st["list_peak"], "list_overflows": st["list_overflows"],
                           "traversed_gteps": (st["reached_edges"] / args.steps) * world * args.steps
                           / (total_ms / 1e3) / 1e9},
             "setup": {"generate_s": gen_s, "create_s": create_s, "graph_bytes": G.device_bytes,
-                      "device_bytes": G.info()["device_bytes"], "workspace_bytes": st["workspace_bytes"]},
+                      "device_bytes": G.info()["device_bytes"], "workspace_bytes": st["workspace_bytes"],
+                      "paper_word_model_bytes": 4 * (7 * g.n + g.nnz)},
         }
         print(json.dumps(line), flush=True)
     if args.trace >= 0 and rank == 0:

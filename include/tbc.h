@@ -126,9 +126,12 @@ enum {
                                 0 in the given order */
     TBC_OPT_NARROW_WIDTH = 18, /* auto engine: probe vertices per level below which the narrow-level
                                 engine runs (default 4096; setting it re-runs the probe next call) */
-    TBC_OPT_BATCH_LIST = 19  /* batched engine: level-list entries allocated per vertex (1..64, default 2;
+    TBC_OPT_BATCH_LIST = 19, /* batched engine: level-list entries allocated per vertex (1..64, default 2;
                                 capped at W).  A sweep whose lists outgrow them is re-run as two half
                                 sweeps (tbc_stats.list_overflows) and the next call doubles them. */
+    TBC_OPT_STAGE = 20       /* measurement: 0 (default) forward + backward; 1 forward stage only --
+                                the batched and narrow-level engines run Alg.1 l.11-28 and skip the
+                                backward stage, leaving bc untouched (per-stage HBM traffic with ncu) */
 };
 
 /* counters accumulated on the device by every tbc_bc / tbc_bc_device / tbc_bfs call since

@@ -26,7 +26,7 @@ ENGINE_CSC, ENGINE_COOT = 0, 1
 FLAG_ONE_FORMAT, FLAG_NO_VALIDATE, FLAG_NO_REORDER = 1, 2, 4
 OPT_DIRECTION, OPT_BWD_DIRECTION, OPT_TRACE, OPT_FORMAT, OPT_PARTITIONS = 1, 2, 3, 4, 11
 OPT_BATCH, OPT_BATCH_PULL, OPT_BATCH_WIDTH, OPT_BATCH_PARTS, OPT_BATCH_ORDER = 12, 13, 14, 16, 17
-OPT_NARROW_WIDTH, OPT_BATCH_LIST = 18, 19
+OPT_NARROW_WIDTH, OPT_BATCH_LIST, OPT_STAGE = 18, 19, 20
 ENGINE_AUTO, ENGINE_PER_SOURCE, ENGINE_BATCHED, ENGINE_NARROW = -1, 0, 1, 2
 OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8, "scan": 9, "bpush": 10}
 FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
@@ -193,6 +193,10 @@ class Graph:
     def set_batch_list(self, factor: int):
         """Batched engine: level-list entries allocated per vertex (TBC_OPT_BATCH_LIST, 1..64, default 2)."""
         _check(lib().tbc_graph_set_option(self._h, OPT_BATCH_LIST, float(factor)))
+
+    def set_stage(self, stage: int):
+        """Measurement: 0 forward + backward (default), 1 forward stage only (TBC_OPT_STAGE; bc untouched)."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_STAGE, float(stage)))
 
     def set_narrow_width(self, width: float):
         """Auto engine: probe vertices per level below which the narrow-level engine runs (TBC_OPT_NARROW_WIDTH)."""

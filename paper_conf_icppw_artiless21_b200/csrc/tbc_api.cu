@@ -548,6 +548,12 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->batch = v;
         return TBC_OK;
     }
+    if (key == TBC_OPT_STAGE) {
+        int v = (int)value;
+        if (v < 0 || v > 1 || (double)v != value) return set_error(TBC_ERR_INVALID, "stage %g not 0 or 1", value);
+        g->stage = v;
+        return TBC_OK;
+    }
     if (key == TBC_OPT_BATCH_LIST) {
         int v = (int)value;
         if (v < 1 || v > 64 || (double)v != value) return set_error(TBC_ERR_INVALID, "batch list factor %g not in [1, 64]", value);

@@ -122,6 +122,7 @@ struct BParams {
     // exported to bfs_depth[i n + v], bfs_sigma[i n + v] (pre-set to -1 / 0 by the host)
     int32_t *bfs_depth;
     double *bfs_sigma;
+    int fwd_only;  // TBC_OPT_STAGE = 1: forward stage only (measurement), bc untouched
 };
 
 // one launch: a BParams per SM partition (its own workspace and counters/barrier); partition q
@@ -896,10 +897,11 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             const int64_t used = nxt_p0_end(P, D);
             if (used > C->st_list_peak) C->st_list_peak = used;
         }
-        if (P.bfs_depth) {  // tbc_bfs_batch: export depth / sigma level by level, retire, next batch
-            for (int L = 0; L <= D; ++L) {
+        if (P.bfs_depth || P.fwd_only) {  // tbc_bfs_batch (export depth / sigma) or forward-only
+            for (int L = 0; L <= D; ++L) {  // measurement (TBC_OPT_STAGE): retire, next batch
                 const int64_t *l = P.lvl + 4 * (int64_t)L;
-                bclear<W, true>(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps, L, b);
+                if (P.bfs_depth) bclear<W, true>(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps, L, b);
+                else bclear<W>(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps);
             }
             if (cta0 && tid == 0) {
                 C->st_scans += pulls;
@@ -1266,6 +1268,7 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
         P.trace_b = g->trace_src >= 0 ? g->trace_src / W : -1;
         P.bfs_depth = bfs_depth;
         P.bfs_sigma = bfs_sigma;
+        P.fwd_only = g->stage == 1;
     }
     g->last_width = W;
     g->last_parts = np;

@@ -205,6 +205,7 @@ struct tbc_graph {
     int bwd_mode = 0;
     int fmt_mode = 0;
     double c_list = 12.0, c_stream = 4.0, c_atom = 18.0, c_vert = 10.0, c_scan = 3.0, c_bpush = 6.0;
+    int stage = 0;                // TBC_OPT_STAGE: 0 forward + backward, 1 forward only (measurement)
     int batch = -1;               // TBC_OPT_BATCH: -1 auto, 0 per source, 1 batched, 2 narrow-level
     int narrow = -1;              // auto choice, settled by the first call's probe: 1 narrow-level engine
     double narrow_width = 4096.0; // TBC_OPT_NARROW_WIDTH: probe's vertices per level below which auto is narrow

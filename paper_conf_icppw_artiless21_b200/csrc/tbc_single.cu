@@ -55,6 +55,7 @@ struct SParams {
     double bc_scale;
     int32_t *bfs_depth;  // tbc_bfs_batch: forward only, export [source index][caller label]
     double *bfs_sigma;
+    int fwd_only;        // TBC_OPT_STAGE = 1: forward stage only (measurement), bc untouched
     int64_t probe_cap;   // > 0: probe run (one source, forward only, stop after ~probe_cap vertices)
     int64_t *probe_out;  // {levels completed, vertices discovered}
 };
@@ -190,8 +191,8 @@ __global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) 
             atomicAdd((unsigned long long *)&P.ctr->st_levels, (unsigned long long)(D + 2));
             atomicMax((unsigned long long *)&P.ctr->st_max_depth, (unsigned long long)D);
         }
-        if (P.bfs_depth) {  // tbc_bfs_batch: export depth / sigma, reset, next source
-            for (int L = 0; L <= D; ++L) {
+        if (P.bfs_depth || P.fwd_only) {  // tbc_bfs_batch: export depth / sigma; or forward only
+            for (int L = 0; L <= D && P.bfs_depth; ++L) {
                 const int b0 = lvl[L], b1 = lvl[L + 1];
                 for (int i = b0 + tid; i < b1; i += kSB) {
                     const int32_t x = order[i];
@@ -360,12 +361,13 @@ tbc_status single_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double 
     SParams P = single_params(g, d_sources, k, d_bc);
     P.bfs_depth = bfs_depth;
     P.bfs_sigma = bfs_sigma;
+    P.fwd_only = g->stage == 1;
     const int grid = (int)(k < g->sws.slots ? k : g->sws.slots);
     if (grid < 1) return TBC_OK;
     k_bcs<<<grid, kSB, 0, stream>>>(P);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_error(e, "k_bcs launch");
-    if (!bfs_depth) {
+    if (!bfs_depth && !P.fwd_only) {
         k_bcs_reduce<<<148 * 8, 256, 0, stream>>>(g->n, grid, g->sws.rec, d_bc, g->inv);
         if ((e = cudaGetLastError()) != cudaSuccess) return cuda_error(e, "k_bcs_reduce launch");
     }

@@ -78,7 +78,11 @@ def main():
                  "nsecond": 1e-6, "usecond": 1e-3, "msecond": 1.0, "second": 1e3}.get(r[iu], 1.0)
         d[r[im]] = val * scale
     meta = json.load(open(args.meta))
-    hot = [launches[i] for i in sorted(launches) if launches[i]["kernel"] == meta["kernel"]]
+    import re
+    pat = re.compile(r"(^|::|\s)" + meta["kernel"] + r"(<|\(|$)")
+    hot = [launches[i] for i in sorted(launches) if pat.search(launches[i]["kernel"])]
+    if len(hot) < 2:
+        sys.exit("hot kernel launches not found: " + json.dumps(sorted({d["kernel"] for d in launches.values()})))
     full, fwd = hot[-2], hot[-1]
 
     def rec(d):

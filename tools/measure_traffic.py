@@ -75,7 +75,11 @@ def main():
         d = launches.setdefault(int(r[ii]), {"kernel": r[ik]})
         val = float(r[iv].replace(",", ""))
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
-                 "nsecond": 1e-6, "usecond": 1e-3, "msecond": 1.0, "second": 1e3}.get(r[iu], 1.0)
+                 "B": 1, "KB": 1e3, "MB": 1e6, "GB": 1e9, "TB": 1e12,
+                 "nsecond": 1e-6, "usecond": 1e-3, "msecond": 1.0, "second": 1e3,
+                 "ns": 1e-6, "us": 1e-3, "ms": 1.0, "s": 1e3}.get(r[iu])
+        if scale is None:
+            sys.exit(f"unknown ncu unit {r[iu]!r} for {r[im]}")
         d[r[im]] = val * scale
     meta = json.load(open(args.meta))
     import re

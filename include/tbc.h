@@ -57,7 +57,13 @@ enum {
 
 /* create flags */
 enum {
-    TBC_FLAG_ONE_FORMAT = 1u << 0,  /* reserved (strict single-format directed mode, not yet built) */
+    TBC_FLAG_ONE_FORMAT = 1u << 0,  /* strict single format: a directed
+                                       TBC_ENGINE_CSC graph keeps its CSC alone -- no CSR copy, no
+                                       owner arrays (graph ~ 16 n + 4 m bytes: col_ptr, row_idx,
+                                       degrees).  bc then runs the batched engine only: every forward
+                                       level is a pull over in-edges (Alg.3's masked A^T f) and the
+                                       backward pushes delta_u over in-edges with fp64 atomics;
+                                       TBC_OPT_BATCH must stay 1.  No effect on undirected graphs. */
     TBC_FLAG_NO_VALIDATE = 1u << 1, /* skip host-side input validation (caller guarantees it) */
     TBC_FLAG_NO_REORDER = 1u << 2   /* keep the caller's vertex labels internally (default: relabel by
                                        decreasing degree when the degree distribution is skewed --

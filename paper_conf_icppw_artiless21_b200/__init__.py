@@ -112,12 +112,14 @@ class Graph:
 
     @classmethod
     def from_csc(cls, col_ptr, row_idx, directed: bool, engine: int = ENGINE_CSC, device: int = 0,
-                 validate: bool = True, reorder: bool = True):
+                 validate: bool = True, reorder: bool = True, one_format: bool = False):
+        """one_format: directed graphs keep the CSC alone (TBC_FLAG_ONE_FORMAT, batched engine only)."""
         cp = np.ascontiguousarray(col_ptr, dtype=np.int64)
         ri = np.ascontiguousarray(row_idx, dtype=np.int32)
         n = cp.size - 1
         h = ctypes.c_void_p()
-        flags = (0 if validate else FLAG_NO_VALIDATE) | (0 if reorder else FLAG_NO_REORDER)
+        flags = ((0 if validate else FLAG_NO_VALIDATE) | (0 if reorder else FLAG_NO_REORDER)
+                 | (FLAG_ONE_FORMAT if one_format else 0))
         _check(lib().tbc_graph_create_csc(n, int(cp[-1]) if n >= 0 else 0, _p(cp, ctypes.c_int64),
                                           _p(ri, ctypes.c_int32) if ri.size else None, int(directed),
                                           engine, flags, device, ctypes.byref(h)))
@@ -125,11 +127,12 @@ class Graph:
 
     @classmethod
     def from_coo(cls, n, src, dst, directed: bool, engine: int = ENGINE_CSC, device: int = 0,
-                 validate: bool = True, reorder: bool = True):
+                 validate: bool = True, reorder: bool = True, one_format: bool = False):
         s = np.ascontiguousarray(src, dtype=np.int32)
         d = np.ascontiguousarray(dst, dtype=np.int32)
         h = ctypes.c_void_p()
-        flags = (0 if validate else FLAG_NO_VALIDATE) | (0 if reorder else FLAG_NO_REORDER)
+        flags = ((0 if validate else FLAG_NO_VALIDATE) | (0 if reorder else FLAG_NO_REORDER)
+                 | (FLAG_ONE_FORMAT if one_format else 0))
         _check(lib().tbc_graph_create_coo(int(n), s.size, _p(s, ctypes.c_int32) if s.size else None,
                                           _p(d, ctypes.c_int32) if d.size else None, int(directed), engine,
                                           flags, device, ctypes.byref(h)))

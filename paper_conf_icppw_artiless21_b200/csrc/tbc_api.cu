@@ -203,6 +203,9 @@ void free_graph(tbc_graph *g) {
 // Consumes d_keys (device, nnz entries).  Runs on g->stream.
 tbc_status build_from_keys(tbc_graph *g, unsigned long long *d_keys, int64_t nnz) {
     tbc_status st = TBC_OK;
+    // strict single format (NEXT-4): a directed graph keeps the CSC alone (no CSR, no
+    // owner arrays); undirected graphs are one format anyway (the CSC is its own transpose)
+    const bool one_format = (g->flags & TBC_FLAG_ONE_FORMAT) && g->directed;
     cudaStream_t s = g->stream;
     unsigned long long *alt = nullptr, *tkeys = nullptr, *d_bad = nullptr;
     int64_t *d_num = nullptr;
@@ -278,11 +281,12 @@ tbc_status build_from_keys(tbc_graph *g, unsigned long long *d_keys, int64_t nnz
     // CSC of A (in-neighbours)
     TBC_CUDA(dmalloc(g, &g->in_ptr, g->n + 1));
     TBC_CUDA(dmalloc(g, &g->in_idx, m + kPad));  // +pad: 16-byte bulk copies of the last chunk
-    TBC_CUDA(dmalloc(g, &g->in_col, m + kPad));  // column (owner) of every CSC entry: the COOC col_A
+    if (!one_format)  // column (owner) of every CSC entry: the COOC col_A, for edge streams
+        TBC_CUDA(dmalloc(g, &g->in_col, m + kPad));
     k_keys_to_ptr<<<grid_for(m > g->n ? m : g->n + 1), 256, 0, s>>>(g->n, m, d_keys, g->in_ptr,
                                                                    g->in_idx, g->in_col);
     TBC_CUDA(cudaGetLastError());
-    if (!g->directed || g->engine == TBC_ENGINE_CSC) {
+    if (!g->directed || (g->engine == TBC_ENGINE_CSC && !one_format)) {
         // transpose (row << 32 | col), sorted: the CSR of A; compared to the CSC when undirected
         tkeys = alt;  // reuse: alt is free after Unique
         alt = nullptr;
@@ -325,7 +329,7 @@ tbc_status build_from_keys(tbc_graph *g, unsigned long long *d_keys, int64_t nnz
             TBC_CUDA(cudaGetLastError());
         }
     } else {
-        g->out_ptr = nullptr;  // COO^T directed: one format only
+        g->out_ptr = nullptr;  // COO^T or TBC_FLAG_ONE_FORMAT directed: one format only
         g->out_idx = nullptr;
         g->out_row = nullptr;
     }
@@ -355,8 +359,8 @@ tbc_status create_common(int64_t n, int directed, int engine, unsigned flags, in
     if (n <= 0 || n >= (1ll << 31)) return set_error(TBC_ERR_INVALID, "n=%lld out of [1, 2^31)", (long long)n);
     if (engine != TBC_ENGINE_CSC && engine != TBC_ENGINE_COOT)
         return set_error(TBC_ERR_INVALID, "unknown engine %d", engine);
-    if (flags & TBC_FLAG_ONE_FORMAT)
-        return set_error(TBC_ERR_UNSUPPORTED, "TBC_FLAG_ONE_FORMAT is not implemented in this build");
+    if ((flags & TBC_FLAG_ONE_FORMAT) && engine != TBC_ENGINE_CSC)
+        return set_error(TBC_ERR_UNSUPPORTED, "TBC_FLAG_ONE_FORMAT applies to TBC_ENGINE_CSC (COO^T is one format already)");
     int ndev = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev);
     if (e != cudaSuccess) return cuda_error(e, "cudaGetDeviceCount");
@@ -545,6 +549,8 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
     if (key == TBC_OPT_BATCH) {
         int v = (int)value;
         if (v < -1 || v > 2 || (double)v != value) return set_error(TBC_ERR_INVALID, "engine %g not in [-1, 2]", value);
+        if (g->engine == TBC_ENGINE_CSC && g->directed && !g->out_idx && v != 1)
+            return set_error(TBC_ERR_UNSUPPORTED, "one-format graphs run the batched engine only");
         g->batch = v;
         return TBC_OK;
     }
@@ -648,6 +654,11 @@ tbc_status tbc_bfs(tbc_graph *g, int32_t source, int32_t *depth_out, double *sig
     if (source < 0 || source >= g->n) return set_error(TBC_ERR_INVALID, "source %d out of range", source);
     tbc_status st = TBC_OK;
     TBC_CUDA(cudaSetDevice(g->device));
+    if (g->ws_count == 0) {  // one-format graphs carry no per-source engine: the batched forward stage
+        std::vector<int32_t> d(depth_out ? 0 : g->n);
+        std::vector<double> sg(sigma_out ? 0 : g->n);
+        return tbc_bfs_batch(g, &source, 1, depth_out ? depth_out : d.data(), sigma_out ? sigma_out : sg.data());
+    }
     if (g->src_cap < 1) {
         TBC_CUDA(cudaMalloc(&g->src_tmp, sizeof(int32_t)));
         g->src_cap = 1;
@@ -687,7 +698,8 @@ tbc_status tbc_bfs_batch(tbc_graph *g, const int32_t *sources, int64_t k, int32_
     if (k < 0) return set_error(TBC_ERR_INVALID, "k < 0");
     if (k > 0 && (!sources || !depth_out || !sigma_out)) return set_error(TBC_ERR_INVALID, "NULL pointer");
     if (g->engine != TBC_ENGINE_CSC) return set_error(TBC_ERR_UNSUPPORTED, "tbc_bfs_batch: CSC engine only");
-    if (g->batch == 0) return set_error(TBC_ERR_UNSUPPORTED, "tbc_bfs_batch: per-source engine selected (use tbc_bfs)");
+    if (g->batch == 0 && g->ws_count > 0)
+        return set_error(TBC_ERR_UNSUPPORTED, "tbc_bfs_batch: per-source engine selected (use tbc_bfs)");
     for (int64_t i = 0; i < k; ++i)
         if (sources[i] < 0 || sources[i] >= g->n)
             return set_error(TBC_ERR_INVALID, "sources[%lld] = %d out of range", (long long)i, sources[i]);

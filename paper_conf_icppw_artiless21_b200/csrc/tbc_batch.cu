@@ -63,7 +63,7 @@ constexpr int kPad = 8;
 constexpr int kBU = TBC_BUNROLL;
 constexpr int kBU64 = TBC_BUNROLL64;
 
-enum { B_PUSH = 0, B_PULL = 1, B_BWD = 2 };
+enum { B_PUSH = 0, B_PULL = 1, B_BWD = 2, B_BPUSH = 3 };  // B_BPUSH: one-format backward push
 
 // lane-mask word of a batch of W sources: lane l of a warp holds sources l and (W = 64) l + 32
 template <int W> struct MaskT { using T = uint32_t; };
@@ -123,6 +123,11 @@ struct BParams {
     int32_t *bfs_depth;
     double *bfs_sigma;
     int fwd_only;  // TBC_OPT_STAGE = 1: forward stage only (measurement), bc untouched
+    // TBC_FLAG_ONE_FORMAT (directed): the CSC is the only adjacency -- list entries carry in-edge
+    // spans (adj_ptr = in_ptr), every forward level is a pull, the backward pushes delta_u of level
+    // L+1 over its in-edges into level L's rows, then an owner pass finishes level L
+    int one_format;
+    const int64_t *__restrict__ adj_ptr;  // spans of list entries: out_ptr, or in_ptr (one format)
 };
 
 // one launch: a BParams per SM partition (its own workspace and counters/barrier); partition q
@@ -396,7 +401,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
         for (int i = 0; i < kBI; ++i) {
             const int sl = i * 32 + lane;
             if (sl < ne) {
-                const MT g = (MODE == B_PUSH) ? (MT)~vis[xs[i]] : emsk[xs[i]];
+                const MT g = (MODE == B_PUSH) ? (MT)~vis[xs[i]] : emsk[xs[i]];  // BPUSH: M_L(u)
                 ems[i] = g & (MT)ws.msk[ws.own[sl]];
             }
             ws.x[sl] = xs[i];
@@ -434,7 +439,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                 cdg[i] = 0;
                 cbg[i] = 0;
                 if (ems[i] != (MT)0) cl[i] = atomicOr(&fr_out[xs[i]], ems[i]) == (MT)0;
-                if (cl[i]) span(P.out_ptr, xs[i], cdg[i], cbg[i]);
+                if (cl[i]) span(P.adj_ptr, xs[i], cdg[i], cbg[i]);
             }
             bappend(cl, xs, cdg, cbg, out, P.ebits);
         }
@@ -449,6 +454,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             const int fl = ws.fl[j];
             if (MODE != B_BWD && bits == 0) continue;
             if (MODE == B_BWD && bits == 0 && !(fl & 1)) continue;
+            (void)fl;
 #ifdef TBC_PROF
             ++n_own;
 #endif
@@ -464,17 +470,21 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                 // collectives inside): warp iterations = the busiest lane's count, not the slots'
                 mine[k] = lm[k] & bits;
             }
-            if (MODE == B_PUSH) {
+            if (MODE == B_PUSH || MODE == B_BPUSH) {
+                // PUSH: sigma(x) += sigma(u) (Alg.1 l.19 as a scatter); BPUSH (one format): the owner
+                // w of level L+1 adds delta_u(w) into the accumulator row of each in-neighbour u on
+                // level L (A delta_u of l.37, R1, as a scatter over the CSC)
+                double *const dst = MODE == B_PUSH ? sig : P.du;
 #pragma unroll
                 for (int k = 0; k < NS; ++k) {
-                    const double su = in[k] ? sig[row + 32 * k] : 0.0;
+                    const double su = in[k] ? (MODE == B_PUSH ? sig : P.du)[row + 32 * k] : 0.0;
 #pragma unroll
                     for (int h = 0; h < kBI; ++h) {
                         uint32_t mm = (uint32_t)(mine[k] >> (32 * h));
                         while (mm) {
                             const int sl = 32 * h + __ffs(mm) - 1;
                             mm &= mm - 1;
-                            atomicAdd(&sig[(int64_t)ws.x[sl] * W + 32 * k + lane], su);
+                            atomicAdd(&dst[(int64_t)ws.x[sl] * W + 32 * k + lane], su);
                         }
                     }
                 }
@@ -588,7 +598,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                 cv[i] = cl[i] ? ws.claim[q] : 0;
                 cdg[i] = 0;
                 cbg[i] = 0;
-                if (cl[i]) span(P.out_ptr, cv[i], cdg[i], cbg[i]);
+                if (cl[i]) span(P.adj_ptr, cv[i], cdg[i], cbg[i]);
             }
             bappend(cl, cv, cdg, cbg, out, P.ebits);
         }
@@ -638,6 +648,44 @@ __device__ __forceinline__ void bclear(const BParams &P, const Lv &l, void *fr_,
                     P.du[row] = 0.0;
                 }
             }
+        }
+    }
+}
+
+// one-format owner pass of level L: for each (v, lane s) on level L the row of du holds
+// acc_s(v) = sum of delta_u over v's level-(L+1) out-neighbours (pushed there by B_BPUSH);
+// bc(v) += scale * sum_s sigma_s(v) acc_s(v) (Alg.1 l.39, l.45) and du_s(v) = 1/sigma + acc (l.35)
+template <int W>
+__device__ __forceinline__ void bowner(const BParams &P, const Lv &l, int64_t gwarp, int64_t nwarps) {
+    using MT = typename MaskT<W>::T;
+    constexpr int NS = W / 32;
+    const MT *lm = static_cast<const MT *>(P.list_m);
+    const int lane = threadIdx.x & 31;
+    for (int64_t base = gwarp * 32; base < l.N; base += nwarps * 32) {
+        const int64_t p = base + lane;
+        int32_t v = -1;
+        MT m = 0;
+        if (p < l.N) {
+            v = P.list_v[l.p0 + p];
+            m = lm[l.p0 + p];
+        }
+        const int cnt = (int)min((int64_t)32, l.N - base);
+        for (int q = 0; q < cnt; ++q) {
+            const int32_t vq = __shfl_sync(FULL, v, q);
+            const MT mq = __shfl_sync(FULL, m, q);
+            double c = 0.0;
+#pragma unroll
+            for (int k = 0; k < NS; ++k) {
+                if ((mq >> (32 * k + lane)) & 1u) {
+                    const int64_t row = (int64_t)vq * W + 32 * k + lane;
+                    const double sv = P.sig[row], acc = P.du[row];
+                    c += sv * acc;
+                    P.du[row] = 1.0 / sv + acc;
+                }
+            }
+#pragma unroll
+            for (int o = 16; o >= 1; o >>= 1) c += __shfl_xor_sync(FULL, c, o);
+            if (lane == 0 && c != 0.0) atomicAdd(&P.bc[P.inv ? P.inv[vq] : vq], c * P.bc_scale);
         }
     }
 }
@@ -716,7 +764,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
                     }
                 }
                 uint32_t dg = 0, bg = 0;
-                if (take) span(P.out_ptr, s[k], dg, bg);
+                if (take) span(P.adj_ptr, s[k], dg, bg);
                 const unsigned tm = __ballot_sync(FULL, take);
                 uint32_t inc = take ? dg : 0u;
                 for (int o = 1; o < 32; o <<= 1) {
@@ -760,8 +808,8 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
         bool overflow = false;
         for (;;) {
             // direction of level d+1 (uniform: every CTA computes it from the same snapshot)
-            const bool pull = d + 1 >= 2 && P.dir_mode != 1 &&
-                              (P.dir_mode == 2 || (double)cur.E * P.pull_ratio > (double)P.m);
+            const bool pull = P.one_format || (d + 1 >= 2 && P.dir_mode != 1 &&
+                              (P.dir_mode == 2 || (double)cur.E * P.pull_ratio > (double)P.m));
             // ---- B(d): lanes of level d -> list masks and visited; retire M_{d-1}; candidates
             BPROF_START();
             if (cta0 && tid == 0) C->list = 0;  // relative counter of level d+1 (snapshot already taken)
@@ -912,7 +960,40 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
         }
         // ---------------- backward, L = D..1 (Alg.1 l.29-47); level L+2 retired on the way
         int64_t bwd_edges = 0;
-        for (int L = D; L >= 1; --L) {
+        for (int L = D; L >= 1 && P.one_format; --L) {
+            // one format (CSC only): P(L) pushes delta_u of level L+1 over its in-edges into the rows
+            // of level L (masked M_{L+1}(w) & M_L(u)); O(L) finishes level L (owner pass)
+            const BOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0, nullptr};
+            if (L < D) {
+                const int64_t *l1 = P.lvl + 4 * (int64_t)(L + 1);
+                const Lv lw{l1[0], l1[1], l1[2], l1[3]};
+                if (cta0 && tid == 0) C->dyn[(ph + 1) & 1] = 0;
+                bpass<B_BPUSH, W>(P, ws, P.list_v + lw.p0, P.list_pre + lw.p0, P.list_beg + lw.p0, list_m + lw.p0,
+                                  P.tiles + lw.tb, lw.N, lw.E, P.in_idx, fr[L & 1], nullptr, 0u, gwarp, nwarps, none,
+                                  &C->dyn[ph & 1]);
+                ++ph;
+                bwd_edges += lw.E;
+                bsync(C, gen, ncta);
+            }
+            const int64_t *l = P.lvl + 4 * (int64_t)L;
+            bowner<W>(P, Lv{l[0], l[1], l[2], l[3]}, gwarp, nwarps);
+            {  // scatter M_{L-1} (P(L-1)'s in-neighbour masks) and drop M_{L+1}: the same parity array
+                const int64_t *lp = P.lvl + 4 * (int64_t)(L - 1);
+                for (int64_t p = gtid; p < lp[1]; p += nthreads) atomicOr(&fr[(L - 1) & 1][P.list_v[lp[0] + p]], list_m[lp[0] + p]);
+                if (L + 1 <= D) {
+                    const int64_t *ln = P.lvl + 4 * (int64_t)(L + 1);
+                    for (int64_t p = gtid; p < ln[1]; p += nthreads)
+                        atomicAnd(&fr[(L + 1) & 1][P.list_v[ln[0] + p]], ~list_m[ln[0] + p]);
+                }
+            }
+            if (L + 2 <= D) {
+                const int64_t *l2 = P.lvl + 4 * (int64_t)(L + 2);
+                bclear<W>(P, Lv{l2[0], l2[1], l2[2], l2[3]}, fr[L & 1], gwarp, nwarps);
+            }
+            bsync(C, gen, ncta);
+            btrace(P, tr, 4, L, l[1], l[2], 0, 0);
+        }
+        for (int L = D; L >= 1 && !P.one_format; --L) {
             const int64_t *l = P.lvl + 4 * (int64_t)L;
             const Lv lv{l[0], l[1], l[2], l[3]};
             const BOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0, nullptr};
@@ -1105,7 +1186,8 @@ __global__ void k_source_keys(int64_t k, int64_t n, const int32_t *__restrict__ 
         }
         const int32_t v = perm ? perm[sc] : sc;
         unsigned long long vol = 0;
-        for (int64_t e = out_ptr[v] + lane; e < out_ptr[v + 1]; e += 32) vol += (unsigned)deg2[out_idx[e]].x;
+        if (out_idx)  // one-format graphs (no CSR): the out-degree alone
+            for (int64_t e = out_ptr[v] + lane; e < out_ptr[v + 1]; e += 32) vol += (unsigned)deg2[out_idx[e]].x;
 #pragma unroll
         for (int o = 16; o >= 1; o >>= 1) vol += __shfl_xor_sync(0xffffffffu, vol, o);
         if (lane == 0) {
@@ -1269,6 +1351,8 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
         P.bfs_depth = bfs_depth;
         P.bfs_sigma = bfs_sigma;
         P.fwd_only = g->stage == 1;
+        P.one_format = g->out_idx == nullptr ? 1 : 0;
+        P.adj_ptr = P.one_format ? g->in_ptr : g->out_ptr;
     }
     g->last_width = W;
     g->last_parts = np;

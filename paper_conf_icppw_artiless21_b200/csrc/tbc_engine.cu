@@ -1281,6 +1281,10 @@ tbc_status engine_setup(tbc_graph *g) {
         return cuda_error(e, "workspace cudaMalloc");
     g->device_bytes += sizeof(Ctrs) + sizeof(int64_t) * 8 * kTraceCap;
     if ((e = cudaMemsetAsync(g->gctr, 0, sizeof(Ctrs), s))) return cuda_error(e, "workspace init");
+    if (g->engine == TBC_ENGINE_CSC && g->directed && !g->out_idx) {
+        g->batch = 1;  // one format: the batched engine only (no per-source workspace)
+        return TBC_OK;
+    }
     tbc_status st = engine_workspaces(g, 1);
     if (st != TBC_OK) return st;
     {  // vertices that can have in-edges: [0, n_scan); count of in-degree > 0 (scan cost model)
@@ -1315,7 +1319,9 @@ tbc_status engine_choose(tbc_graph *g, const int32_t *d_sources, int64_t k, cuda
         *mode = g->last_mode = 0;
         return TBC_OK;
     }
-    if (g->batch >= 0) {
+    if (g->batch >= 0 || (g->directed && !g->out_idx)) {  // forced, or one format (batched only)
+        if (g->directed && !g->out_idx && g->batch != 1)
+            return set_error(TBC_ERR_UNSUPPORTED, "one-format graphs run the batched engine only (TBC_OPT_BATCH = 1)");
         *mode = g->last_mode = g->batch;
         return TBC_OK;
     }

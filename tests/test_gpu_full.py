@@ -284,3 +284,57 @@ def test_batched_list_overflow_reruns_halves(width):
             G.reset_stats()
             assert_bc(G.bc(src), want)
         assert G.stats()["list_overflows"] == 0
+
+
+# ------------------------------------------------------------------ strict single format (NEXT-4)
+
+def _one_format_cases():
+    rng = np.random.default_rng(8)
+    out = [gg.path(7, directed=True), gg.star(9, directed_both=True),
+           gg.from_edges("dstar_d", 3000, [(0, 1)] + [(0, i) for i in range(2, 1500)] + [(1, i) for i in range(1500, 3000)]
+                         + [(i, 1) for i in range(2, 1500)], True)]
+    for t in range(6):
+        n = int(rng.integers(5, 80))
+        A = rng.random((n, n)) < float(rng.choice([0.03, 0.1, 0.3]))
+        np.fill_diagonal(A, False)
+        u, v = np.nonzero(A)
+        out.append(gg.from_edges(f"rd{t}", n, np.stack([u, v], 1), True))
+    out.append(gg.kronecker(14, 16, seed=6, directed=True, device="cuda"))
+    return out
+
+
+@pytest.mark.parametrize("width", [32, 64])
+def test_one_format_directed_parity(width):
+    """TBC_FLAG_ONE_FORMAT: CSC only; pull-only forward, backward push over in-edges (fp64 atomics)."""
+    for g in _one_format_cases():
+        src = gg.sources(g, min(3 * g.n, 150), seed=1) if g.n > 5 else np.arange(g.n, dtype=np.int32)
+        want = oracle.bc(g.col_ptr, g.row_idx, True, src)
+        with tbc.Graph.from_csc(g.col_ptr, g.row_idx, True, one_format=True) as G:
+            G.set_batch_width(width)
+            assert_bc(G.bc(src), want)
+            depth, sigma = G.bfs_batch(src[:5])
+            assert_bfs_rows(g, src[:5], depth, sigma)
+            d1, s1 = G.bfs(int(src[0]))  # tbc_bfs routes to the batched forward stage
+            np.testing.assert_array_equal(d1, depth[0])
+            with pytest.raises(tbc.TBCError):
+                G.set_batch(0)
+
+
+def test_one_format_footprint_and_cfg3_full_list():
+    """Config 3 in strict single-format mode: graph bytes against the paper's 7n+m word model
+     and the two-format graph, and the full 4096-source list against the cached oracle."""
+    meta, z = _fixture("oracle_cfg3")
+    g, src = gg.make_config(3, device="cuda")
+    n, m = g.n, g.nnz
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, True) as G2:
+        two = G2.info()["device_bytes"]
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, True, one_format=True) as G:
+        one = G.info()["device_bytes"]
+        assert one <= 16 * n + 4 * m + (16 << 20), (one, 16 * n + 4 * m)
+        assert one < 0.5 * two, (one, two)
+        got = G.bc(src)
+        assert G.stats()["sources"] == len(src)
+    zero = got == 0.0
+    assert _sha(np.packbits(zero)) == meta["zero_sha"]
+    assert_bc(got[z["sample_idx"]], z["sample_val"])
+    assert_bc(got[z["top_idx"]], z["top_val"])

@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--direction", type=int, default=0)
     ap.add_argument("--format", type=int, default=0, help="0 auto, 1 list passes, 2 edge streams")
     ap.add_argument("--engine", choices=["csc", "coot"], default="csc")
+    ap.add_argument("--one-format", action="store_true",
+                    help="directed graphs keep the CSC alone (TBC_FLAG_ONE_FORMAT; batched engine)")
     ap.add_argument("--batch", type=int, default=-1,
                     help="engine: -1 auto (level-width probe), 0 per source, 1 batched, 2 narrow-level")
     ap.add_argument("--width", type=int, default=0, help="batched engine: sources per sweep (32, 64; 0 auto)")
@@ -267,11 +269,12 @@ def main():
     per_gpu = len(my_src)
     t0 = time.time()
     engine = tbc.ENGINE_COOT if args.engine == "coot" else tbc.ENGINE_CSC
-    G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, engine=engine, device=local)
+    G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, engine=engine, device=local,
+                           one_format=args.one_format)
     create_s = time.time() - t0
     G.set_direction(args.direction)
     G.set_format(args.format)
-    G.set_batch(args.batch)
+    G.set_batch(1 if args.one_format and g.directed else args.batch)
     G.set_batch_width(args.width)
     G.set_batch_order(args.order)
     if args.cost:
@@ -394,6 +397,7 @@ def main():
                              if (8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) > 126e6 else
                              "graph fits in L2 (small config); no flush",
                        "direction": args.direction, "format": args.format, "engine_kind": args.engine,
+                       "one_format": bool(args.one_format and g.directed),
                        "engine_mode": (f"batched, {wdt} sources per sweep, {st['batch_parts']} SM partition(s)"
                                        + (", sources grouped by 2-hop out-volume" if args.order
                                           else ", sources in the given order")) if eng == 1

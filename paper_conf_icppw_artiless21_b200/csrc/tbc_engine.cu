@@ -1281,12 +1281,6 @@ tbc_status engine_setup(tbc_graph *g) {
         return cuda_error(e, "workspace cudaMalloc");
     g->device_bytes += sizeof(Ctrs) + sizeof(int64_t) * 8 * kTraceCap;
     if ((e = cudaMemsetAsync(g->gctr, 0, sizeof(Ctrs), s))) return cuda_error(e, "workspace init");
-    if (g->engine == TBC_ENGINE_CSC && g->directed && !g->out_idx) {
-        g->batch = 1;  // one format: the batched engine only (no per-source workspace)
-        return TBC_OK;
-    }
-    tbc_status st = engine_workspaces(g, 1);
-    if (st != TBC_OK) return st;
     {  // vertices that can have in-edges: [0, n_scan); count of in-degree > 0 (scan cost model)
         unsigned long long *d_cnt = nullptr;
         if ((e = cudaMalloc(&d_cnt, 2 * sizeof(unsigned long long))) ||
@@ -1301,6 +1295,12 @@ tbc_status engine_setup(tbc_graph *g) {
         g->n_scan = (int64_t)h[0];
         g->n_in = (int64_t)h[1];
     }
+    if (g->engine == TBC_ENGINE_CSC && g->directed && !g->out_idx) {
+        g->batch = 1;  // one format: the batched engine only (no per-source workspace)
+        return TBC_OK;
+    }
+    tbc_status st = engine_workspaces(g, 1);
+    if (st != TBC_OK) return st;
     int per_sm = 0, sms = 0;
     if ((e = cudaFuncSetAttribute(k_bc, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes)) ||
         (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_bc, kBlock, kSmemBytes)) ||

@@ -6,7 +6,8 @@ Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline``
 
 Contents
   * ``brandes.c``  -- textbook Brandes (Eq. 2-4) in plain C / fp64,
-    exposed here as :func:`bc`, :func:`bfs`, :func:`delta`.
+    exposed here as :func:`bc`, :func:`bfs`, :func:`delta`; and the same algorithm in C long
+    double (extended exponent range, NEXT-2) as :func:`bc_ld`, :func:`bfs_ld`.
   * ``brute.py``   -- exact brute force of Freeman's Eq. 1 with rationals
     for graphs of <= 12 vertices (a second, independent oracle used to pin the first).
 
@@ -32,7 +33,7 @@ def build(force: bool = False) -> str:
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
         subprocess.check_call(["gcc", "-O3", "-march=native", "-std=c11", "-fPIC", "-shared",
-                               "-o", tmp, _SRC, "-lpthread"])
+                               "-o", tmp, _SRC, "-lpthread", "-lm"])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -52,6 +53,10 @@ def _load():
         lib.oracle_bfs.restype = ctypes.c_int
         lib.oracle_delta.argtypes = [i64, P(i64), P(i32), i32, P(dbl)]
         lib.oracle_delta.restype = ctypes.c_int
+        lib.oracle_bfs_ld.argtypes = [i64, P(i64), P(i32), i32, P(i32), P(dbl), P(i32)]
+        lib.oracle_bfs_ld.restype = ctypes.c_int
+        lib.oracle_bc_ld.argtypes = [i64, P(i64), P(i32), ctypes.c_int, P(i32), i64, P(dbl)]
+        lib.oracle_bc_ld.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -126,4 +131,36 @@ def delta(col_ptr, row_idx, source: int) -> np.ndarray:
                           _ptr(out, ctypes.c_double))
     if rc != 0:
         raise ValueError("oracle_delta: invalid input")
+    return out
+
+
+def bfs_ld(col_ptr, row_idx, source: int):
+    """Extended range (C long double, NEXT-2): (depth int32[n], sigma mantissa float64[n] in [0.5, 1),
+    sigma binary exponent int32[n]); sigma = mantissa * 2**exponent, also beyond fp64's range."""
+    lib = _load()
+    cp, ri = _csc(col_ptr, row_idx)
+    n = cp.size - 1
+    depth = np.empty(n, dtype=np.int32)
+    mant = np.empty(n, dtype=np.float64)
+    expo = np.empty(n, dtype=np.int32)
+    rc = lib.oracle_bfs_ld(n, _ptr(cp, ctypes.c_int64), _ptr(ri, ctypes.c_int32), int(source),
+                           _ptr(depth, ctypes.c_int32), _ptr(mant, ctypes.c_double), _ptr(expo, ctypes.c_int32))
+    if rc != 0:
+        raise ValueError("oracle_bfs_ld: invalid input")
+    return depth, mant, expo
+
+
+def bc_ld(col_ptr, row_idx, directed: bool, sources) -> np.ndarray:
+    """bc with long double sigma / delta / accumulation (single thread), rounded to float64."""
+    lib = _load()
+    cp, ri = _csc(col_ptr, row_idx)
+    n = cp.size - 1
+    src = np.ascontiguousarray(sources, dtype=np.int32)
+    out = np.zeros(n, dtype=np.float64)
+    if src.size == 0:
+        return out
+    rc = lib.oracle_bc_ld(n, _ptr(cp, ctypes.c_int64), _ptr(ri, ctypes.c_int32), int(bool(directed)),
+                          _ptr(src, ctypes.c_int32), src.size, _ptr(out, ctypes.c_double))
+    if rc != 0:
+        raise ValueError("oracle_bc_ld: invalid input")
     return out

@@ -30,6 +30,7 @@
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
+#include <math.h>
 #include <pthread.h>
 #include <time.h>
 
@@ -249,4 +250,98 @@ int oracle_bc_timed(int64_t n, const int64_t *col_ptr, const int32_t *row_idx, i
     for (int t = 0; t < nthreads; ++t) free(tasks[t].bc);
     free(tasks); free(th); og_free(&g);
     return rc;
+}
+
+/* ---------------------------------------------------------------- extended range (NEXT-2)
+ * The same textbook Brandes in C long double (x86-64: 64-bit mantissa, 15-bit exponent, range
+ * ~2^16383), for graphs whose shortest-path counts overflow fp64: on a P_a x P_b mesh sigma from a
+ * corner is C(i+j, i), ~2^8190 at 4096 x 4096 (the paper's int sigma, and fp64
+ * both overflow).  Same passages as og_forward / og_backward (Alg.1, Eq. 4); only the
+ * number type differs.  sigma is exported as mantissa in [0.5, 1) and a binary exponent (frexpl). */
+
+typedef struct {
+    int32_t *dist;
+    long double *sigma;
+    long double *acc;
+    int32_t *order;
+} og_work_ld;
+
+static int og_work_ld_alloc(int64_t n, og_work_ld *w) {
+    size_t nn = (size_t)(n > 0 ? n : 1);
+    w->dist = (int32_t *)malloc(sizeof(int32_t) * nn);
+    w->sigma = (long double *)malloc(sizeof(long double) * nn);
+    w->acc = (long double *)malloc(sizeof(long double) * nn);
+    w->order = (int32_t *)malloc(sizeof(int32_t) * nn);
+    return (w->dist && w->sigma && w->acc && w->order) ? 0 : -1;
+}
+static void og_work_ld_free(og_work_ld *w) { free(w->dist); free(w->sigma); free(w->acc); free(w->order); }
+
+static int64_t og_forward_ld(const og_graph *g, int32_t s, og_work_ld *w) {
+    int64_t n = g->n;
+    for (int64_t v = 0; v < n; ++v) { w->dist[v] = -1; w->sigma[v] = 0.0L; w->acc[v] = 0.0L; }
+    w->dist[s] = 0;
+    w->sigma[s] = 1.0L;                                  /* Alg.1 l.17 */
+    int64_t head = 0, tail = 0;
+    w->order[tail++] = s;
+    while (head < tail) {
+        int32_t v = w->order[head++];
+        for (int64_t k = g->out_ptr[v]; k < g->out_ptr[v + 1]; ++k) {
+            int32_t x = g->out_idx[k];
+            if (w->dist[x] < 0) { w->dist[x] = w->dist[v] + 1; w->order[tail++] = x; }
+            if (w->dist[x] == w->dist[v] + 1) w->sigma[x] += w->sigma[v];
+        }
+    }
+    return tail;
+}
+
+static void og_backward_ld(const og_graph *g, int32_t s, og_work_ld *w, int64_t reached, int directed,
+                           long double *bc) {
+    for (int64_t i = reached - 1; i >= 0; --i) {
+        int32_t x = w->order[i];
+        long double delta_x = w->sigma[x] * w->acc[x];      /* Alg.1 l.39 */
+        if (x != s) bc[x] += directed ? delta_x : 0.5L * delta_x;   /* Alg.1 l.45 */
+        long double coef = (1.0L + delta_x) / w->sigma[x];  /* Alg.1 l.35 */
+        for (int64_t k = g->in_ptr[x]; k < g->in_ptr[x + 1]; ++k) {
+            int32_t v = g->in_idx[k];
+            if (w->dist[v] == w->dist[x] - 1) w->acc[v] += coef;
+        }
+    }
+}
+
+/* depth and sigma (as mantissa * 2^exponent) from one source, long double. */
+int oracle_bfs_ld(int64_t n, const int64_t *col_ptr, const int32_t *row_idx, int32_t source,
+                  int32_t *depth_out, double *sigma_mant, int32_t *sigma_exp) {
+    if (n <= 0 || source < 0 || source >= n) return -1;
+    og_graph g; og_work_ld w;
+    if (og_build(n, col_ptr, row_idx, &g)) return -1;
+    if (og_work_ld_alloc(n, &w)) { og_free(&g); return -1; }
+    og_forward_ld(&g, source, &w);
+    for (int64_t v = 0; v < n; ++v) {
+        int e = 0;
+        long double m = frexpl(w.sigma[v], &e);
+        if (depth_out) depth_out[v] = w.dist[v];
+        if (sigma_mant) sigma_mant[v] = (double)m;
+        if (sigma_exp) sigma_exp[v] = (int32_t)e;
+    }
+    og_work_ld_free(&w); og_free(&g);
+    return 0;
+}
+
+/* bc over a source list, long double accumulation, rounded to double at the end (single thread). */
+int oracle_bc_ld(int64_t n, const int64_t *col_ptr, const int32_t *row_idx, int directed,
+                 const int32_t *sources, int64_t k, double *bc_out) {
+    if (n <= 0 || k < 0 || !bc_out) return -1;
+    for (int64_t i = 0; i < k; ++i) if (sources[i] < 0 || sources[i] >= n) return -1;
+    og_graph g; og_work_ld w;
+    if (og_build(n, col_ptr, row_idx, &g)) return -1;
+    if (og_work_ld_alloc(n, &w)) { og_free(&g); return -1; }
+    long double *bc = (long double *)calloc((size_t)n, sizeof(long double));
+    if (!bc) { og_work_ld_free(&w); og_free(&g); return -1; }
+    for (int64_t i = 0; i < k; ++i) {                        /* Alg.1 l.6 */
+        int64_t r = og_forward_ld(&g, sources[i], &w);
+        og_backward_ld(&g, sources[i], &w, r, directed, bc);
+    }
+    for (int64_t v = 0; v < n; ++v) bc_out[v] = (double)bc[v];
+    free(bc); og_work_ld_free(&w); og_free(&g);
+    return 0;
 }

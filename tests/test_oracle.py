@@ -323,3 +323,67 @@ def test_edge_cases(oracle_lib):
     assert list(depth) == [0, -1, -1, -1] and list(sigma) == [1, 0, 0, 0]
     with pytest.raises(ValueError):
         oracle_lib.bc(g.col_ptr, g.row_idx, False, [7])
+
+
+# ------------------------------------------------------------------ extended-range oracle (NEXT-2)
+
+def _ld_value_vs_int(mant, expo, exact: int, rel: float):
+    """|mant * 2^expo - exact| <= rel * exact, in exact integer arithmetic (values beyond fp64)."""
+    M = int(float(mant) * 2 ** 53)  # the double mantissa times 2^53 is an integer
+    e = int(expo) - 53
+    approx_num, approx_den = (M << e, 1) if e >= 0 else (M, 1 << -e)
+    diff = abs(approx_num - exact * approx_den)
+    return diff * (10 ** 15) <= int(rel * 1e15) * exact * approx_den
+
+
+def test_ld_grid_sigma_binomial_beyond_fp64(oracle_lib):
+    """700 x 700 mesh from the corner: sigma(i,j) = C(i+j, i) up to ~2^1393 (> DBL_MAX ~ 2^1024),
+    depth(i,j) = i+j.  Exact below 2^64, relative 1e-15 above (64-bit long double mantissa)."""
+    a = b = 700
+    g = gg.grid(a, b)
+    depth, mant, expo = oracle_lib.bfs_ld(g.col_ptr, g.row_idx, 0)
+    assert expo.max() > 1300
+    rng = np.random.default_rng(3)
+    cells = [(i, j) for i in range(0, a, 37) for j in range(0, b, 41)] + [(a - 1, b - 1), (a - 1, 0), (0, b - 1)]
+    cells += [tuple(x) for x in rng.integers(0, a, size=(200, 2))]
+    for i, j in cells:
+        v = i * b + j
+        assert depth[v] == i + j
+        assert _ld_value_vs_int(mant[v], expo[v], math.comb(i + j, i), 1e-15), (i, j)
+
+
+def test_ld_matches_fp64_and_bruteforce_small(oracle_lib):
+    """Where fp64 does not overflow, the long double oracle equals the fp64 oracle and Eq. 1."""
+    rng = random.Random(5)
+    for trial in range(40):
+        n = rng.randint(1, 11)
+        directed = trial % 2 == 1
+        edges = [(u, v) for u in range(n) for v in range(n) if u != v and rng.random() < 0.3]
+        if not directed:
+            edges = [(u, v) for u, v in edges if u < v]
+        g = gg.from_edges("r", n, edges, directed)
+        src = np.asarray([rng.randrange(n) for _ in range(rng.randint(0, 2 * n))], dtype=np.int32)
+        exact = brute.bc_exact(brute.adjacency_from_csc(g.col_ptr, g.row_idx), directed, sources=list(src))
+        got = oracle_lib.bc_ld(g.col_ptr, g.row_idx, directed, src)
+        assert_bc_close(got, exact)
+        np.testing.assert_allclose(got, oracle_lib.bc(g.col_ptr, g.row_idx, directed, src), rtol=1e-13, atol=0)
+        if n:
+            d1, s1 = oracle_lib.bfs(g.col_ptr, g.row_idx, 0)
+            d2, m2, e2 = oracle_lib.bfs_ld(g.col_ptr, g.row_idx, 0)
+            np.testing.assert_array_equal(d1, d2)
+            np.testing.assert_array_equal(np.ldexp(m2, e2), s1)
+
+
+def test_ld_delta_sum_invariant_on_overflowing_mesh(oracle_lib):
+    """Backward stage in extended range: on a 600 x 600 mesh (sigma ~2^1195 from a corner), one source's
+    sum_v delta_s(v) = sum_t (depth_s(t) - 1) (each shortest path's interior vertices), halved if
+    undirected -- exact integer, checked to 1e-12 relative; and delta is finite everywhere."""
+    g = gg.grid(600, 600)
+    for s in (0, 600 * 300 + 300, 600 * 599 + 17):
+        depth, _, expo = oracle_lib.bfs_ld(g.col_ptr, g.row_idx, s)
+        bc = oracle_lib.bc_ld(g.col_ptr, g.row_idx, False, [s])
+        want = 0.5 * float(np.sum(depth[depth > 0] - 1))
+        assert np.all(np.isfinite(bc))
+        assert abs(bc.sum() - want) <= 1e-12 * want
+        if s == 0:
+            assert expo.max() > 1100

@@ -364,6 +364,9 @@ CONFIGS = {
     # exact BC of mycielski16 (Table 5) and single sources of mycielski19 (Table 3)
     6: dict(name="cfg6_mycielski16_exact", kind="myc", myc=16, directed=False, k=None, src_seed=None),
     7: dict(name="cfg7_mycielski19_sources", kind="myc", myc=19, directed=False, k=1024, src_seed=17),
+    # the literal average-degree-4 mesh of BASELINE configs[3] (4096 x 4096 grid): sigma overflows
+    # fp64 (C(i+j, i) ~ 2^8190 from a corner), runnable with extended-range sigma
+    8: dict(name="cfg8_mesh4096_literal", kind="mesh", side=4096, directed=False, k=1024, src_seed=18),
 }
 
 
@@ -380,6 +383,10 @@ def make_config(cfg: int, device: str = "cpu", scale_override: int | None = None
     elif c["kind"] == "myc":
         g = mycielski(c["myc"], device=device)
         src = np.arange(g.n, dtype=np.int32) if c["k"] is None else sources(g, c["k"], c["src_seed"])
+    elif c["kind"] == "mesh":
+        side = side_override or c["side"]
+        g = grid(side, side)
+        src = sources(g, c["k"], c["src_seed"])
     else:
         g = road_lattice(side_override or c["side"], c["q"], c["seed"])
         src = sources(g, c["k"], c["src_seed"])

@@ -135,6 +135,11 @@ enum {
     TBC_OPT_BATCH_LIST = 19, /* batched engine: level-list entries allocated per vertex (1..64, default 2;
                                 capped at W).  A sweep whose lists outgrow them is re-run as two half
                                 sweeps (tbc_stats.list_overflows) and the next call doubles them. */
+    TBC_OPT_SIGMA = 21,      /* narrow-level engine: 0 (default) fp64 sigma, and a source whose sigma
+                                leaves the fp64 range (inf; meshes: sigma = C(i+j, i) from a corner) is
+                                re-run with extended-range sigma and delta_u (mantissa + int32
+                                exponent, exact below 2^53 like fp64; tbc_stats.xr_sources); 1 always
+                                extended range.  The other engines compute in fp64 only. */
     TBC_OPT_STAGE = 20       /* measurement: 0 (default) forward + backward; 1 forward stage only --
                                 the batched and narrow-level engines run Alg.1 l.11-28 and skip the
                                 backward stage, leaving bc untouched (per-stage HBM traffic with ncu) */
@@ -163,6 +168,7 @@ typedef struct {
     int64_t list_overflows; /* batched engine: sweeps whose level lists outgrew the workspace and were
                                re-run as two half sweeps (the next call grows the lists) */
     int64_t probe_width; /* auto engine: the probe's vertices per level (0 before the probe) */
+    int64_t xr_sources;  /* narrow-level engine: sources run with extended-range sigma (TBC_OPT_SIGMA) */
 } tbc_stats;
 
 /* Create a graph from the CSC of A (CP_A = col_ptr, row_A = row_idx, here 0-based).
@@ -220,6 +226,12 @@ tbc_status tbc_bfs(tbc_graph *g, int32_t source, int32_t *depth_out, double *sig
  * TBC_ERR_UNSUPPORTED for TBC_ENGINE_COOT graphs and for TBC_OPT_BATCH = 0 (use tbc_bfs). */
 tbc_status tbc_bfs_batch(tbc_graph *g, const int32_t *sources, int64_t k, int32_t *depth_out,
                          double *sigma_out);
+
+/* tbc_bfs_batch with sigma as mantissa and binary exponent, for sigma beyond the fp64 range
+ * (NEXT-2): sigma = sigma_mant_out[i n + v] * 2^sigma_exp_out[i n + v], mantissa in [0.5, 1) or 0.
+ * The narrow-level engine exports its extended-range values; the fp64 engines split fp64 sigma. */
+tbc_status tbc_bfs_batch_ext(tbc_graph *g, const int32_t *sources, int64_t k, int32_t *depth_out,
+                             double *sigma_mant_out, int32_t *sigma_exp_out);
 
 /* Graph properties after canonicalisation; any output pointer may be NULL.
  *   nnz = stored entries of A after deduplication; device_bytes = device memory owned now: the

@@ -26,7 +26,7 @@ ENGINE_CSC, ENGINE_COOT = 0, 1
 FLAG_ONE_FORMAT, FLAG_NO_VALIDATE, FLAG_NO_REORDER = 1, 2, 4
 OPT_DIRECTION, OPT_BWD_DIRECTION, OPT_TRACE, OPT_FORMAT, OPT_PARTITIONS = 1, 2, 3, 4, 11
 OPT_BATCH, OPT_BATCH_PULL, OPT_BATCH_WIDTH, OPT_BATCH_PARTS, OPT_BATCH_ORDER = 12, 13, 14, 16, 17
-OPT_NARROW_WIDTH, OPT_BATCH_LIST, OPT_STAGE = 18, 19, 20
+OPT_NARROW_WIDTH, OPT_BATCH_LIST, OPT_STAGE, OPT_SIGMA = 18, 19, 20, 21
 ENGINE_AUTO, ENGINE_PER_SOURCE, ENGINE_BATCHED, ENGINE_NARROW = -1, 0, 1, 2
 OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8, "scan": 9, "bpush": 10}
 FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
@@ -35,7 +35,7 @@ STATUS = {0: "TBC_OK", 1: "TBC_ERR_INVALID", 2: "TBC_ERR_OOM", 3: "TBC_ERR_CUDA"
 
 # every symbol include/tbc.h declares (checked by tests/test_abi.py)
 SYMBOLS = ["tbc_graph_create_csc", "tbc_graph_create_coo", "tbc_bc", "tbc_bc_device", "tbc_bfs",
-           "tbc_bfs_batch", "tbc_graph_info", "tbc_graph_set_option", "tbc_stats_get", "tbc_stats_reset", "tbc_trace_get",
+           "tbc_bfs_batch", "tbc_bfs_batch_ext", "tbc_graph_info", "tbc_graph_set_option", "tbc_stats_get", "tbc_stats_reset", "tbc_trace_get",
            "tbc_profile_get", "tbc_destroy", "tbc_status_string", "tbc_last_error"]
 
 
@@ -49,7 +49,7 @@ class Stats(ctypes.Structure):
     _fields_ = [(f, ctypes.c_int64) for f in
                 ("sources", "reached", "reached_edges", "fwd_edges", "bwd_edges", "levels", "pull_levels", "scans",
                  "max_depth", "list_peak", "bad_sources", "batch_width", "batch_parts", "workspace_bytes",
-                 "engine", "list_overflows", "probe_width")]
+                 "engine", "list_overflows", "probe_width", "xr_sources")]
 
     def as_dict(self):
         return {f: int(getattr(self, f)) for f, _ in self._fields_}
@@ -75,6 +75,7 @@ def lib():
         L.tbc_bc_device.argtypes = [vp, vp, i64, vp, vp]
         L.tbc_bfs.argtypes = [vp, i32, P(i32), P(ctypes.c_double)]
         L.tbc_bfs_batch.argtypes = [vp, P(i32), i64, P(i32), P(ctypes.c_double)]
+        L.tbc_bfs_batch_ext.argtypes = [vp, P(i32), i64, P(i32), P(ctypes.c_double), P(i32)]
         L.tbc_graph_info.argtypes = [vp, P(i64), P(i64), P(ctypes.c_int), P(ctypes.c_size_t)]
         L.tbc_graph_set_option.argtypes = [vp, ctypes.c_int, ctypes.c_double]
         L.tbc_stats_get.argtypes = [vp, P(Stats)]
@@ -85,7 +86,7 @@ def lib():
         L.tbc_status_string.argtypes = [ctypes.c_int]
         L.tbc_status_string.restype = ctypes.c_char_p
         L.tbc_last_error.restype = ctypes.c_char_p
-        for name in SYMBOLS[:13]:
+        for name in SYMBOLS[:14]:
             getattr(L, name).restype = ctypes.c_int
         _LIB = L
     return _LIB
@@ -174,6 +175,21 @@ class Graph:
         _check(lib().tbc_bfs_batch(self._h, _p(src, ctypes.c_int32) if src.size else None, src.size,
                                    _p(depth, ctypes.c_int32), _p(sigma, ctypes.c_double)))
         return depth, sigma
+
+    def bfs_batch_ext(self, sources):
+        """tbc_bfs_batch_ext: (depth int32[k, n], sigma mantissa float64[k, n], sigma exponent int32[k, n])."""
+        src = np.ascontiguousarray(sources, dtype=np.int32)
+        depth = np.empty((src.size, self.n), dtype=np.int32)
+        mant = np.empty((src.size, self.n), dtype=np.float64)
+        expo = np.empty((src.size, self.n), dtype=np.int32)
+        _check(lib().tbc_bfs_batch_ext(self._h, _p(src, ctypes.c_int32) if src.size else None, src.size,
+                                       _p(depth, ctypes.c_int32), _p(mant, ctypes.c_double), _p(expo, ctypes.c_int32)))
+        return depth, mant, expo
+
+    def set_sigma_mode(self, mode: int):
+        """Narrow-level engine: 0 fp64 sigma with an extended-range re-run on overflow (default), 1 always
+        extended range (TBC_OPT_SIGMA)."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_SIGMA, float(mode)))
 
     def info(self) -> dict:
         """tbc_graph_info now (device_bytes includes the engine workspaces allocated so far)."""

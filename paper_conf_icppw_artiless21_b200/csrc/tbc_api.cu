@@ -1,6 +1,7 @@
 // tbc_api.cu -- the extern "C" boundary of libturbobc: graph creation (device-side
 // canonicalisation of the CSC / COOC input of P:95-97), the tbc_bc / tbc_bfs drivers,
 // options, statistics and error reporting.  Declarations and contracts: include/tbc.h.
+#include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstddef>
@@ -192,6 +193,7 @@ void free_graph(tbc_graph *g) {
     if (g->h_bovf) cudaFreeHost(g->h_bovf);
     cudaFree(g->bfs_depth);
     cudaFree(g->bfs_sigma);
+    cudaFree(g->bfs_sexp);
     cudaFree(g->bc_tmp);
     cudaFree(g->src_tmp);
     if (g->stream) cudaStreamDestroy(g->stream);
@@ -554,6 +556,12 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->batch = v;
         return TBC_OK;
     }
+    if (key == TBC_OPT_SIGMA) {
+        int v = (int)value;
+        if (v < 0 || v > 1 || (double)v != value) return set_error(TBC_ERR_INVALID, "sigma mode %g not 0 or 1", value);
+        g->sigma_mode = v;
+        return TBC_OK;
+    }
     if (key == TBC_OPT_STAGE) {
         int v = (int)value;
         if (v < 0 || v > 1 || (double)v != value) return set_error(TBC_ERR_INVALID, "stage %g not 0 or 1", value);
@@ -692,8 +700,23 @@ fail:
     return st;
 }
 
+static tbc_status bfs_batch_impl(tbc_graph *g, const int32_t *sources, int64_t k, int32_t *depth_out,
+                                 double *sigma_out, int32_t *sexp_out);
+
 tbc_status tbc_bfs_batch(tbc_graph *g, const int32_t *sources, int64_t k, int32_t *depth_out, double *sigma_out) {
     g_err[0] = 0;
+    return bfs_batch_impl(g, sources, k, depth_out, sigma_out, nullptr);
+}
+
+tbc_status tbc_bfs_batch_ext(tbc_graph *g, const int32_t *sources, int64_t k, int32_t *depth_out,
+                             double *sigma_mant_out, int32_t *sigma_exp_out) {
+    g_err[0] = 0;
+    if (k > 0 && !sigma_exp_out) return set_error(TBC_ERR_INVALID, "NULL pointer");
+    return bfs_batch_impl(g, sources, k, depth_out, sigma_mant_out, sigma_exp_out);
+}
+
+static tbc_status bfs_batch_impl(tbc_graph *g, const int32_t *sources, int64_t k, int32_t *depth_out,
+                                 double *sigma_out, int32_t *sexp_out) {
     if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
     if (k < 0) return set_error(TBC_ERR_INVALID, "k < 0");
     if (k > 0 && (!sources || !depth_out || !sigma_out)) return set_error(TBC_ERR_INVALID, "NULL pointer");
@@ -708,14 +731,17 @@ tbc_status tbc_bfs_batch(tbc_graph *g, const int32_t *sources, int64_t k, int32_
     tbc_status st = TBC_OK;
     const int64_t kn = k * g->n;
     TBC_CUDA(cudaSetDevice(g->device));
-    if (kn > g->bfs_cap) {
+    if (kn > g->bfs_cap || (sexp_out && !g->bfs_sexp)) {
         cudaFree(g->bfs_depth);
         cudaFree(g->bfs_sigma);
+        cudaFree(g->bfs_sexp);
         g->bfs_depth = nullptr;
         g->bfs_sigma = nullptr;
+        g->bfs_sexp = nullptr;
         g->bfs_cap = 0;
         TBC_CUDA(cudaMalloc(&g->bfs_depth, sizeof(int32_t) * kn));
         TBC_CUDA(cudaMalloc(&g->bfs_sigma, sizeof(double) * kn));
+        if (sexp_out) TBC_CUDA(cudaMalloc(&g->bfs_sexp, sizeof(int32_t) * kn));
         g->bfs_cap = kn;
     }
     if (k > g->src_cap) {
@@ -732,13 +758,22 @@ tbc_status tbc_bfs_batch(tbc_graph *g, const int32_t *sources, int64_t k, int32_
         int mode = 1;
         st = engine_choose(g, g->src_tmp, k, g->stream, &mode);
         if (st != TBC_OK) return st;
-        st = mode == 2 ? single_run(g, g->src_tmp, k, nullptr, g->stream, g->bfs_depth, g->bfs_sigma)
+        st = mode == 2 ? single_run(g, g->src_tmp, k, nullptr, g->stream, g->bfs_depth, g->bfs_sigma,
+                                    sexp_out ? g->bfs_sexp : nullptr)
                        : batch_run(g, g->src_tmp, k, nullptr, g->stream, g->bfs_depth, g->bfs_sigma);
         if (st != TBC_OK) return st;
+        TBC_CUDA(cudaMemcpyAsync(depth_out, g->bfs_depth, sizeof(int32_t) * kn, cudaMemcpyDeviceToHost, g->stream));
+        TBC_CUDA(cudaMemcpyAsync(sigma_out, g->bfs_sigma, sizeof(double) * kn, cudaMemcpyDeviceToHost, g->stream));
+        if (sexp_out && mode == 2)
+            TBC_CUDA(cudaMemcpyAsync(sexp_out, g->bfs_sexp, sizeof(int32_t) * kn, cudaMemcpyDeviceToHost, g->stream));
+        TBC_CUDA(cudaStreamSynchronize(g->stream));
+        if (sexp_out && mode != 2)  // fp64 engines: split the (finite) sigma into mantissa and exponent
+            for (int64_t i = 0; i < kn; ++i) {
+                int e = 0;
+                sigma_out[i] = frexp(sigma_out[i], &e);
+                sexp_out[i] = e;
+            }
     }
-    TBC_CUDA(cudaMemcpyAsync(depth_out, g->bfs_depth, sizeof(int32_t) * kn, cudaMemcpyDeviceToHost, g->stream));
-    TBC_CUDA(cudaMemcpyAsync(sigma_out, g->bfs_sigma, sizeof(double) * kn, cudaMemcpyDeviceToHost, g->stream));
-    TBC_CUDA(cudaStreamSynchronize(g->stream));
     return TBC_OK;
 fail:
     return st;
@@ -767,6 +802,7 @@ tbc_status tbc_stats_get(tbc_graph *g, tbc_stats *out) {
         out->bad_sources += (int64_t)c.bad_sources;
         if (c.st_list_peak > out->list_peak) out->list_peak = c.st_list_peak;
         out->list_overflows += c.st_overflows;
+        out->xr_sources += c.st_xr_sources;
         out->sources += c.st_sources;
         out->reached += c.st_reached;
         out->reached_edges += c.st_reached_edges;
@@ -820,7 +856,7 @@ fail:
 #endif
 }
 
-static constexpr size_t kStatBytes = offsetof(Ctrs, st_overflows) + sizeof(long long) - offsetof(Ctrs, st_sources);
+static constexpr size_t kStatBytes = offsetof(Ctrs, st_xr_sources) + sizeof(long long) - offsetof(Ctrs, st_sources);
 
 tbc_status tbc_stats_reset(tbc_graph *g) {
     if (!g) return set_error(TBC_ERR_INVALID, "graph is NULL");
@@ -831,7 +867,7 @@ tbc_status tbc_stats_reset(tbc_graph *g) {
         Ctrs *c = i < g->ws_count ? g->ws[i].ctr
                   : i < g->ws_count + kMaxPartitions ? g->bws[i - g->ws_count].ctr : g->sws.ctr;
         if (!c) continue;
-        TBC_CUDA(cudaMemset(&c->st_sources, 0, kStatBytes));  // st_sources .. st_overflows
+        TBC_CUDA(cudaMemset(&c->st_sources, 0, kStatBytes));  // st_sources .. st_xr_sources
         TBC_CUDA(cudaMemset(&c->bad_sources, 0, sizeof(unsigned long long)));
     }
     g->retired = Ctrs{};

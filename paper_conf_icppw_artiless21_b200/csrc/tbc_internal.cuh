@@ -35,7 +35,7 @@ struct Ctrs {
     unsigned long long trace_n;   // entries written to the trace buffer
     // accumulated statistics (tbc_stats)
     long long st_sources, st_reached, st_reached_edges, st_fwd_edges, st_bwd_edges, st_levels, st_pull_levels,
-        st_scans, st_max_depth, st_list_peak, st_overflows;
+        st_scans, st_max_depth, st_list_peak, st_overflows, st_xr_sources;
     unsigned long long prof[32];  // TBC_PROF builds: warp-cycles per code region (gctr only)
 };
 
@@ -154,9 +154,10 @@ struct BatchWorkspace {
 // concurrently running source (one per resident CTA)
 // per (slot, vertex) state of the narrow-level engine: one 32-byte DRAM sector
 struct __align__(32) VRec {
-    double sd;     // sigma (forward), then delta_u (backward); 0 between sources
+    double sd;     // sigma (forward), then delta_u (backward); 0 between sources (extended range:
+                   // the mantissa)
     int32_t depth; // -1 between sources
-    int32_t pad;
+    int32_t sexp;  // extended range (NEXT-2): binary exponent of sd (value = sd * 2^sexp), else 0
     double bc;     // the slot's partial bc, summed into the caller's bc after each call
     double pad2;
 };
@@ -205,6 +206,7 @@ struct tbc_graph {
     int bwd_mode = 0;
     int fmt_mode = 0;
     double c_list = 12.0, c_stream = 4.0, c_atom = 18.0, c_vert = 10.0, c_scan = 3.0, c_bpush = 6.0;
+    int sigma_mode = 0;           // TBC_OPT_SIGMA: 0 fp64 + extended re-run on overflow, 1 extended range
     int stage = 0;                // TBC_OPT_STAGE: 0 forward + backward, 1 forward only (measurement)
     int batch = -1;               // TBC_OPT_BATCH: -1 auto, 0 per source, 1 batched, 2 narrow-level
     int narrow = -1;              // auto choice, settled by the first call's probe: 1 narrow-level engine
@@ -227,6 +229,7 @@ struct tbc_graph {
     tbc::Ctrs retired = {};       // statistics of freed batched workspaces (kept for tbc_stats)
     int32_t *bfs_depth = nullptr; // tbc_bfs_batch device outputs (grow-only)
     double *bfs_sigma = nullptr;
+    int32_t *bfs_sexp = nullptr;  // tbc_bfs_batch_ext: sigma exponents
     int64_t bfs_cap = 0;          // elements of bfs_depth / bfs_sigma
     int64_t *trace = nullptr;     // device, 8 * kTraceCap int64
     int64_t trace_src = -1;       // index in the next call's source list to trace (-1: off)
@@ -250,7 +253,7 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
 int batch_width(const tbc_graph *g);  // sources per sweep the next batched call uses
 // narrow-level engine (tbc_single.cu)
 tbc_status single_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
-                      int32_t *bfs_depth = nullptr, double *bfs_sigma = nullptr);
+                      int32_t *bfs_depth = nullptr, double *bfs_sigma = nullptr, int32_t *bfs_sexp = nullptr);
 tbc_status single_probe(tbc_graph *g, const int32_t *d_sources, cudaStream_t stream, double *width);
 void single_free(tbc_graph *g);
 // engine the next bc call on these sources runs (auto: probes once per graph): 0 per source,

@@ -54,13 +54,57 @@ struct SParams {
     int64_t k;
     double bc_scale;
     int32_t *bfs_depth;  // tbc_bfs_batch: forward only, export [source index][caller label]
-    double *bfs_sigma;
+    double *bfs_sigma;   // sigma, or its mantissa when bfs_sexp is set
+    int32_t *bfs_sexp;   // tbc_bfs_batch_ext: binary exponent of sigma
+    const int64_t *__restrict__ in_ptr;   // CSC (in-edges): the extended-range sigma pull
+    const int32_t *__restrict__ in_idx;
+    int sigma_mode;      // TBC_OPT_SIGMA: 0 fp64 with extended-range re-run on overflow, 1 extended
     int fwd_only;        // TBC_OPT_STAGE = 1: forward stage only (measurement), bc untouched
     int64_t probe_cap;   // > 0: probe run (one source, forward only, stop after ~probe_cap vertices)
     int64_t *probe_out;  // {levels completed, vertices discovered}
 };
 
-// relax the out-edge u -> w of frontier level d: claim w for level d+1, add sigma(u)
+// ---- extended-range numbers (NEXT-2): value = f * 2^e with f = 0 or 0.5 <= |f| < 1.  sigma and
+// delta_u of a source on a mesh leave the fp64 range (sigma = C(i+j, i) ~ 2^8190 from a corner of a
+// 4096^2 mesh; delta_u = (1 + delta) / sigma ~ 2^-8190), while delta = sigma * acc and bc stay in
+// range.  Integer sums below 2^53 stay exact (aligned adds of integers), as in fp64.
+struct Xr {
+    double f;
+    int e;
+};
+
+__device__ __forceinline__ Xr xr_norm(double f, int e) {
+    int k = 0;
+    const double m = frexp(f, &k);
+    return Xr{m, f == 0.0 ? 0 : e + k};
+}
+
+__device__ __forceinline__ Xr xr_add(Xr a, Xr b) {
+    if (a.f == 0.0) return b;
+    if (b.f == 0.0) return a;
+    if (a.e < b.e) {
+        const Xr t = a;
+        a = b;
+        b = t;
+    }
+    const int d = a.e - b.e;
+    if (d > 1100) return a;  // b is below a's last mantissa bit
+    return xr_norm(a.f + ldexp(b.f, -d), a.e);
+}
+
+__device__ __forceinline__ Xr xr_mul(Xr a, Xr b) { return xr_norm(a.f * b.f, a.e + b.e); }
+__device__ __forceinline__ Xr xr_inv(Xr a) { return xr_norm(1.0 / a.f, -a.e); }
+__device__ __forceinline__ Xr xr_shfl_xor(Xr a, int o) {
+    return Xr{__shfl_xor_sync(FULL, a.f, o), __shfl_xor_sync(FULL, a.e, o)};
+}
+__device__ __forceinline__ Xr rec_xr(const VRec *r) {  // one 16-byte load: {sd, depth, sexp}
+    const double2 q = __ldcg(reinterpret_cast<const double2 *>(r));
+    return Xr{q.x, __double2hiint(q.y)};
+}
+
+// relax the out-edge u -> w of frontier level d: claim w for level d+1 (the claimer appends it), and
+// in fp64 mode add sigma(u) (Alg.1 l.19-25 as a push); the extended mode sums sigma in a pull
+template <bool XR>
 __device__ __forceinline__ void relax(VRec *rec, int32_t *order, int32_t w, int d, double su, int *cnt, int end) {
     int dw = __ldcg(&rec[w].depth);
     if (dw == -1) {
@@ -70,13 +114,18 @@ __device__ __forceinline__ void relax(VRec *rec, int32_t *order, int32_t w, int 
             dw = d + 1;
         }
     }
-    if (dw == d + 1) atomicAdd(&rec[w].sd, su);
+    if (!XR && dw == d + 1) atomicAdd(&rec[w].sd, su);
 }
 
-// delta_u(w) if w is on level L+1, else 0 (one 16-byte load: sd and depth share it)
+// delta_u(w) if w is on level L+1, else 0 (one 16-byte load: sd and depth share it); in the
+// extended-range sigma pull the same test selects the in-neighbours on level d (L = d - 1)
 __device__ __forceinline__ double child(const VRec *rec, int32_t w, int L) {
     const double2 r = __ldcg(reinterpret_cast<const double2 *>(rec + w));
     return __double2loint(r.y) == L + 1 ? r.x : 0.0;
+}
+__device__ __forceinline__ Xr child_xr(const VRec *rec, int32_t w, int L) {
+    const double2 r = __ldcg(reinterpret_cast<const double2 *>(rec + w));
+    return __double2loint(r.y) == L + 1 ? Xr{r.x, __double2hiint(r.y)} : Xr{0.0, 0};
 }
 
 // Alg.1 l.35-45 for v with acc = sum of delta_u over its level-(L+1) out-neighbours
@@ -86,171 +135,263 @@ __device__ __forceinline__ void finish(const SParams &P, VRec *rec, int32_t v, d
     if (delta != 0.0) rec[v].bc += delta * P.bc_scale;
     rec[v].sd = 1.0 / sv + acc;
 }
+__device__ __forceinline__ void finish_xr(const SParams &P, VRec *rec, int32_t v, Xr acc) {
+    const Xr sv = rec_xr(rec + v);
+    const Xr dl = xr_mul(sv, acc);
+    const double delta = ldexp(dl.f, dl.e);  // delta_s(v) <= n: in range
+    if (delta != 0.0) rec[v].bc += delta * P.bc_scale;
+    const Xr du = xr_add(xr_inv(sv), acc);
+    rec[v].sd = du.f;
+    rec[v].sexp = du.e;
+}
 
 __device__ __forceinline__ void reset_level(VRec *rec, const int32_t *order, int b0, int b1) {
     for (int i = b0 + (int)threadIdx.x; i < b1; i += kSB) {
         const int32_t x = order[i];
-        *reinterpret_cast<int4 *>(rec + x) = make_int4(0, 0, -1, 0);  // sd = 0, depth = -1, pad = 0
+        *reinterpret_cast<int4 *>(rec + x) = make_int4(0, 0, -1, 0);  // sd = 0, depth = -1, sexp = 0
     }
 }
 
-__global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) {
+struct SShared {
+    int cnt[2], hcnt[2];
+    int ovf;  // fp64 mode: a sigma left the fp64 range (the source is re-run in extended range)
+    int32_t heavy[kHeavyCap];
+    unsigned long long edges[2];
+};
+
+// One source on one CTA (Alg.1 l.7-47).  XR = false: fp64 sigma / delta_u; returns false (nothing
+// accumulated, state reset) if a sigma overflowed, so that the caller re-runs the source with XR.
+template <bool XR>
+__device__ bool bcs_source(const SParams &P, SShared &sh, int64_t si, int32_t s, VRec *rec, int32_t *order,
+                           int32_t *lvl) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int64_t n = P.n;
-    const int64_t slot = blockIdx.x;
-    VRec *rec = P.rec + slot * n;
-    int32_t *order = P.order + slot * n;
-    int32_t *lvl = P.lvl + slot * (n + 2);
-    __shared__ int s_cnt[2], s_hcnt[2];
-    __shared__ int32_t s_heavy[kHeavyCap];
-    __shared__ unsigned long long s_edges[2];
-    for (int64_t si = blockIdx.x; si < P.k; si += gridDim.x) {
-        int32_t s = P.sources[si];
-        if (s < 0 || s >= n) {  // skipped and counted (tbc_bc_device does not validate on the host)
-            if (tid == 0) atomicAdd(&P.ctr->bad_sources, 1ull);
-            continue;
-        }
-        if (P.perm) s = P.perm[s];
-        if (tid == 0) {  // level 0 (Alg.1 l.15-18)
-            rec[s].depth = 0;
-            rec[s].sd = 1.0;
-            order[0] = s;
-            lvl[0] = 0;
-            lvl[1] = 1;
-            s_cnt[0] = s_cnt[1] = 0;
-            s_hcnt[0] = s_hcnt[1] = 0;
-            s_edges[0] = s_edges[1] = 0;
+    if (tid == 0) {  // level 0 (Alg.1 l.15-18)
+        rec[s].depth = 0;
+        rec[s].sd = XR ? 0.5 : 1.0;  // 1 = 0.5 * 2^1
+        rec[s].sexp = XR ? 1 : 0;
+        order[0] = s;
+        lvl[0] = 0;
+        lvl[1] = 1;
+        sh.cnt[0] = sh.cnt[1] = 0;
+        sh.hcnt[0] = sh.hcnt[1] = 0;
+        sh.edges[0] = sh.edges[1] = 0;
+        sh.ovf = 0;
+    }
+    __syncthreads();
+    // ---------------- forward (Alg.1 l.11-28)
+    int d = 0, beg = 0, end = 1;
+    unsigned long long my_edges = 0;
+    bool probe_stop = false;
+    for (;;) {
+        const int par = d & 1;
+        for (int i = beg + tid; i < end; i += kSB) {
+            if (P.probe_cap > 0 && end + *(volatile int *)&sh.cnt[par] > P.probe_cap) break;
+            const int32_t u = order[i];
+            const int64_t e0 = P.out_ptr[u], e1 = P.out_ptr[u + 1];
+            my_edges += (unsigned long long)(e1 - e0);
+            const double su = XR ? 0.0 : __ldcg(&rec[u].sd);
+            if (!XR && !(su <= 1.7976931348623157e308)) sh.ovf = 1;  // inf: out of the fp64 range
+            if (e1 - e0 > kHeavy) {
+                const int h = atomicAdd(&sh.hcnt[par], 1);
+                if (h < kHeavyCap) {
+                    sh.heavy[h] = u;
+                    continue;
+                }
+            }
+            for (int64_t e = e0; e < e1; ++e) relax<XR>(rec, order, P.out_idx[e], d, su, &sh.cnt[par], end);
         }
         __syncthreads();
-        // ---------------- forward (Alg.1 l.11-28)
-        int d = 0, beg = 0, end = 1;
-        unsigned long long my_edges = 0;
-        bool probe_stop = false;
-        for (;;) {
-            const int par = d & 1;
-            for (int i = beg + tid; i < end; i += kSB) {
-                if (P.probe_cap > 0 && end + *(volatile int *)&s_cnt[par] > P.probe_cap) break;
-                const int32_t u = order[i];
-                const int64_t e0 = P.out_ptr[u], e1 = P.out_ptr[u + 1];
-                my_edges += (unsigned long long)(e1 - e0);
+        if (tid == 0) {  // counters of level d+2 (their level-d readers are past the barrier)
+            sh.cnt[par ^ 1] = 0;
+            sh.hcnt[par ^ 1] = 0;
+        }
+        const int nh = min(sh.hcnt[par], kHeavyCap);
+        for (int h = warp; h < nh; h += kSWarps) {
+            const int32_t u = sh.heavy[h];
+            const double su = XR ? 0.0 : __ldcg(&rec[u].sd);
+            const int64_t e1 = P.out_ptr[u + 1];
+            for (int64_t e = P.out_ptr[u] + lane; e < e1; e += 32)
+                relax<XR>(rec, order, P.out_idx[e], d, su, &sh.cnt[par], end);
+        }
+        __syncthreads();
+        const int nn = sh.cnt[par];
+        if (P.probe_cap > 0 && end + nn > P.probe_cap) {
+            probe_stop = true;
+            end += nn;  // every claimed vertex is in the list (reset below)
+            break;
+        }
+        if (nn == 0) break;
+        if (XR) {
+            // sigma(w) = sum of sigma(u) over the in-neighbours u on level d (Alg.1 l.19 as a pull,
+            // extended-range adds); in-degrees above kHeavy by a warp with a shuffle reduction
+            for (int i = end + tid; i < end + nn; i += kSB) {
+                const int32_t w = order[i];
+                const int64_t e0 = P.in_ptr[w], e1 = P.in_ptr[w + 1];
                 if (e1 - e0 > kHeavy) {
-                    const int h = atomicAdd(&s_hcnt[par], 1);
+                    const int h = atomicAdd(&sh.hcnt[par], 1);
                     if (h < kHeavyCap) {
-                        s_heavy[h] = u;
+                        sh.heavy[h] = w;
                         continue;
                     }
                 }
-                const double su = __ldcg(&rec[u].sd);
-                for (int64_t e = e0; e < e1; ++e) relax(rec, order, P.out_idx[e], d, su, &s_cnt[par], end);
+                Xr sg{0.0, 0};
+                for (int64_t e = e0; e < e1; ++e) sg = xr_add(sg, child_xr(rec, P.in_idx[e], d - 1));  // depth d
+                rec[w].sd = sg.f;
+                rec[w].sexp = sg.e;
             }
             __syncthreads();
-            if (tid == 0) {  // counters of level d+2 (their level-d readers are past the barrier)
-                s_cnt[par ^ 1] = 0;
-                s_hcnt[par ^ 1] = 0;
-            }
-            const int nh = min(s_hcnt[par], kHeavyCap);
-            for (int h = warp; h < nh; h += kSWarps) {
-                const int32_t u = s_heavy[h];
-                const double su = __ldcg(&rec[u].sd);
-                const int64_t e1 = P.out_ptr[u + 1];
-                for (int64_t e = P.out_ptr[u] + lane; e < e1; e += 32)
-                    relax(rec, order, P.out_idx[e], d, su, &s_cnt[par], end);
-            }
-            __syncthreads();
-            const int nn = s_cnt[par];
-            if (P.probe_cap > 0 && end + nn > P.probe_cap) {
-                probe_stop = true;
-                end += nn;  // every claimed vertex is in the list (reset below)
-                break;
-            }
-            if (nn == 0) break;
-            beg = end;
-            end += nn;
-            ++d;
-            if (tid == 0) lvl[d + 1] = end;
-        }
-        const int D = d;  // deepest non-empty level
-        atomicAdd(&s_edges[0], my_edges);
-        if (tid == 0) s_hcnt[0] = s_hcnt[1] = 0;  // their forward readers are past the last barrier
-        __syncthreads();
-        if (P.probe_cap > 0) {  // probe: report, reset every listed vertex, done
-            if (tid == 0) {
-                P.probe_out[0] = D + 1;  // levels whose expansion ran
-                P.probe_out[1] = end;    // vertices discovered
-                P.probe_out[2] = probe_stop ? 0 : 1;
-            }
-            reset_level(rec, order, 0, end);
-            __syncthreads();
-            return;
-        }
-        if (tid == 0) {
-            atomicAdd((unsigned long long *)&P.ctr->st_sources, 1ull);
-            atomicAdd((unsigned long long *)&P.ctr->st_reached, (unsigned long long)end);
-            atomicAdd((unsigned long long *)&P.ctr->st_reached_edges, s_edges[0]);
-            atomicAdd((unsigned long long *)&P.ctr->st_fwd_edges, s_edges[0]);
-            atomicAdd((unsigned long long *)&P.ctr->st_levels, (unsigned long long)(D + 2));
-            atomicMax((unsigned long long *)&P.ctr->st_max_depth, (unsigned long long)D);
-        }
-        if (P.bfs_depth || P.fwd_only) {  // tbc_bfs_batch: export depth / sigma; or forward only
-            for (int L = 0; L <= D && P.bfs_depth; ++L) {
-                const int b0 = lvl[L], b1 = lvl[L + 1];
-                for (int i = b0 + tid; i < b1; i += kSB) {
-                    const int32_t x = order[i];
-                    const int64_t o = si * n + (P.inv ? P.inv[x] : x);
-                    P.bfs_depth[o] = L;
-                    P.bfs_sigma[o] = __ldcg(&rec[x].sd);
+            const int nh2 = min(sh.hcnt[par], kHeavyCap);
+            for (int h = warp; h < nh2; h += kSWarps) {
+                const int32_t w = sh.heavy[h];
+                const int64_t e1 = P.in_ptr[w + 1];
+                Xr sg{0.0, 0};
+                for (int64_t e = P.in_ptr[w] + lane; e < e1; e += 32) sg = xr_add(sg, child_xr(rec, P.in_idx[e], d - 1));
+#pragma unroll
+                for (int o = 16; o >= 1; o >>= 1) sg = xr_add(sg, xr_shfl_xor(sg, o));
+                if (lane == 0) {
+                    rec[w].sd = sg.f;
+                    rec[w].sexp = sg.e;
                 }
             }
             __syncthreads();
-            reset_level(rec, order, 0, end);
-            if (tid == 0) s_edges[0] = 0;
-            __syncthreads();
-            continue;
+            if (tid == 0) sh.hcnt[par] = 0;
         }
-        // ---------------- backward, L = D..1 (Alg.1 l.29-47)
-        unsigned long long my_bwd = 0;
-        for (int L = D; L >= 1; --L) {
-            const int par = L & 1;
+        beg = end;
+        end += nn;
+        ++d;
+        if (tid == 0) lvl[d + 1] = end;
+    }
+    const int D = d;  // deepest non-empty level
+    atomicAdd(&sh.edges[0], my_edges);
+    if (tid == 0) sh.hcnt[0] = sh.hcnt[1] = 0;  // their forward readers are past the last barrier
+    __syncthreads();
+    if (P.probe_cap > 0) {  // probe: report, reset every listed vertex, done
+        if (tid == 0) {
+            P.probe_out[0] = D + 1;  // levels whose expansion ran
+            P.probe_out[1] = end;    // vertices discovered
+            P.probe_out[2] = probe_stop ? 0 : 1;
+        }
+        reset_level(rec, order, 0, end);
+        __syncthreads();
+        return true;
+    }
+    if (!XR && sh.ovf) {  // a sigma overflowed fp64: drop this run (nothing accumulated yet)
+        reset_level(rec, order, 0, end);
+        if (tid == 0) sh.edges[0] = 0;
+        __syncthreads();
+        return false;
+    }
+    if (tid == 0) {
+        atomicAdd((unsigned long long *)&P.ctr->st_sources, 1ull);
+        atomicAdd((unsigned long long *)&P.ctr->st_reached, (unsigned long long)end);
+        atomicAdd((unsigned long long *)&P.ctr->st_reached_edges, sh.edges[0]);
+        atomicAdd((unsigned long long *)&P.ctr->st_fwd_edges, sh.edges[0]);
+        atomicAdd((unsigned long long *)&P.ctr->st_levels, (unsigned long long)(D + 2));
+        atomicMax((unsigned long long *)&P.ctr->st_max_depth, (unsigned long long)D);
+        if (XR) atomicAdd((unsigned long long *)&P.ctr->st_xr_sources, 1ull);
+    }
+    if (P.bfs_depth || P.fwd_only) {  // tbc_bfs_batch: export depth / sigma; or forward only
+        for (int L = 0; L <= D && P.bfs_depth; ++L) {
             const int b0 = lvl[L], b1 = lvl[L + 1];
             for (int i = b0 + tid; i < b1; i += kSB) {
-                const int32_t v = order[i];
-                const int64_t e0 = P.out_ptr[v], e1 = P.out_ptr[v + 1];
-                my_bwd += (unsigned long long)(e1 - e0);
-                if (e1 - e0 > kHeavy) {
-                    const int h = atomicAdd(&s_hcnt[par], 1);
-                    if (h < kHeavyCap) {
-                        s_heavy[h] = v;
-                        continue;
-                    }
+                const int32_t x = order[i];
+                const int64_t o = si * n + (P.inv ? P.inv[x] : x);
+                P.bfs_depth[o] = L;
+                const Xr sg = XR ? rec_xr(rec + x) : xr_norm(__ldcg(&rec[x].sd), 0);
+                if (P.bfs_sexp) {  // mantissa and exponent (any range)
+                    P.bfs_sigma[o] = sg.f;
+                    P.bfs_sexp[o] = sg.e;
+                } else {
+                    P.bfs_sigma[o] = ldexp(sg.f, sg.e);
                 }
+            }
+        }
+        __syncthreads();
+        reset_level(rec, order, 0, end);
+        if (tid == 0) sh.edges[0] = 0;
+        __syncthreads();
+        return true;
+    }
+    // ---------------- backward, L = D..1 (Alg.1 l.29-47)
+    unsigned long long my_bwd = 0;
+    for (int L = D; L >= 1; --L) {
+        const int par = L & 1;
+        const int b0 = lvl[L], b1 = lvl[L + 1];
+        for (int i = b0 + tid; i < b1; i += kSB) {
+            const int32_t v = order[i];
+            const int64_t e0 = P.out_ptr[v], e1 = P.out_ptr[v + 1];
+            my_bwd += (unsigned long long)(e1 - e0);
+            if (e1 - e0 > kHeavy) {
+                const int h = atomicAdd(&sh.hcnt[par], 1);
+                if (h < kHeavyCap) {
+                    sh.heavy[h] = v;
+                    continue;
+                }
+            }
+            if (XR) {
+                Xr acc{0.0, 0};
+                for (int64_t e = e0; e < e1; ++e) acc = xr_add(acc, child_xr(rec, P.out_idx[e], L));
+                finish_xr(P, rec, v, acc);
+            } else {
                 double acc = 0.0;
                 for (int64_t e = e0; e < e1; ++e) acc += child(rec, P.out_idx[e], L);
                 finish(P, rec, v, acc);
             }
-            if (L + 2 <= D) reset_level(rec, order, lvl[L + 2], lvl[L + 3]);
-            __syncthreads();
-            if (tid == 0) s_hcnt[par ^ 1] = 0;
-            const int nh = min(s_hcnt[par], kHeavyCap);
-            for (int h = warp; h < nh; h += kSWarps) {
-                const int32_t v = s_heavy[h];
-                const int64_t e1 = P.out_ptr[v + 1];
+        }
+        if (L + 2 <= D) reset_level(rec, order, lvl[L + 2], lvl[L + 3]);
+        __syncthreads();
+        if (tid == 0) sh.hcnt[par ^ 1] = 0;
+        const int nh = min(sh.hcnt[par], kHeavyCap);
+        for (int h = warp; h < nh; h += kSWarps) {
+            const int32_t v = sh.heavy[h];
+            const int64_t e1 = P.out_ptr[v + 1];
+            if (XR) {
+                Xr acc{0.0, 0};
+                for (int64_t e = P.out_ptr[v] + lane; e < e1; e += 32) acc = xr_add(acc, child_xr(rec, P.out_idx[e], L));
+#pragma unroll
+                for (int o = 16; o >= 1; o >>= 1) acc = xr_add(acc, xr_shfl_xor(acc, o));
+                if (lane == 0) finish_xr(P, rec, v, acc);
+            } else {
                 double acc = 0.0;
                 for (int64_t e = P.out_ptr[v] + lane; e < e1; e += 32) acc += child(rec, P.out_idx[e], L);
 #pragma unroll
                 for (int o = 16; o >= 1; o >>= 1) acc += __shfl_xor_sync(FULL, acc, o);
                 if (lane == 0) finish(P, rec, v, acc);
             }
-            __syncthreads();
-        }
-        reset_level(rec, order, 0, lvl[min(D, 2) + 1]);
-        atomicAdd(&s_edges[1], my_bwd);
-        __syncthreads();
-        if (tid == 0) {
-            atomicAdd((unsigned long long *)&P.ctr->st_bwd_edges, s_edges[1]);
-            s_edges[0] = s_edges[1] = 0;
-            s_hcnt[0] = s_hcnt[1] = 0;
         }
         __syncthreads();
+    }
+    reset_level(rec, order, 0, lvl[min(D, 2) + 1]);
+    atomicAdd(&sh.edges[1], my_bwd);
+    __syncthreads();
+    if (tid == 0) {
+        atomicAdd((unsigned long long *)&P.ctr->st_bwd_edges, sh.edges[1]);
+        sh.edges[0] = sh.edges[1] = 0;
+        sh.hcnt[0] = sh.hcnt[1] = 0;
+    }
+    __syncthreads();
+    return true;
+}
+
+__global__ void __launch_bounds__(kSB) k_bcs(const __grid_constant__ SParams P) {
+    const int64_t n = P.n;
+    const int64_t slot = blockIdx.x;
+    VRec *rec = P.rec + slot * n;
+    int32_t *order = P.order + slot * n;
+    int32_t *lvl = P.lvl + slot * (n + 2);
+    __shared__ SShared sh;
+    for (int64_t si = blockIdx.x; si < P.k; si += gridDim.x) {
+        int32_t s = P.sources[si];
+        if (s < 0 || s >= n) {  // skipped and counted (tbc_bc_device does not validate on the host)
+            if (threadIdx.x == 0) atomicAdd(&P.ctr->bad_sources, 1ull);
+            continue;
+        }
+        if (P.perm) s = P.perm[s];
+        // fp64 first; a source whose sigma leaves the fp64 range runs again in extended range
+        if (P.sigma_mode == 1 || !bcs_source<false>(P, sh, si, s, rec, order, lvl))
+            bcs_source<true>(P, sh, si, s, rec, order, lvl);
+        if (P.probe_cap > 0) return;
     }
 }
 
@@ -269,7 +410,7 @@ __global__ void k_bcs_reduce(int64_t n, int64_t slots, VRec *rec, double *bc, co
 
 __global__ void k_rec_init(int64_t count, VRec *rec) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x)
-        rec[i] = VRec{0.0, -1, 0, 0.0, 0.0};
+        rec[i] = VRec{0.0, -1, 0, 0.0, 0.0};  // sd, depth, sexp, bc, pad
 }
 
 }  // namespace
@@ -350,17 +491,21 @@ static SParams single_params(tbc_graph *g, const int32_t *d_sources, int64_t k, 
     P.k = k;
     P.bc_scale = g->directed ? 1.0 : 0.5;
     P.probe_out = w.probe_out;
+    P.in_ptr = g->in_ptr;
+    P.in_idx = g->in_idx;
+    P.sigma_mode = g->sigma_mode;
     return P;
 }
 
 tbc_status single_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc, cudaStream_t stream,
-                      int32_t *bfs_depth, double *bfs_sigma) {
+                      int32_t *bfs_depth, double *bfs_sigma, int32_t *bfs_sexp) {
     if (!g->out_ptr) return set_error(TBC_ERR_UNSUPPORTED, "narrow-level engine needs the out-edge format");
     tbc_status st = single_alloc(g);
     if (st != TBC_OK) return st;
     SParams P = single_params(g, d_sources, k, d_bc);
     P.bfs_depth = bfs_depth;
     P.bfs_sigma = bfs_sigma;
+    P.bfs_sexp = bfs_sexp;
     P.fwd_only = g->stage == 1;
     const int grid = (int)(k < g->sws.slots ? k : g->sws.slots);
     if (grid < 1) return TBC_OK;

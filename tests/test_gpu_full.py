@@ -340,3 +340,85 @@ def test_one_format_footprint_and_cfg3_full_list():
     assert _sha(np.packbits(zero)) == meta["zero_sha"]
     assert_bc(got[z["sample_idx"]], z["sample_val"])
     assert_bc(got[z["top_idx"]], z["top_val"])
+
+
+# ------------------------------------------------------------------ extended-range sigma (NEXT-2)
+
+def _assert_sigma_ext(mant, expo, m_ora, e_ora):
+    """sigma as (mantissa, exponent): exact below 2^53, relative 1e-12 above (any range)."""
+    zero = m_ora == 0
+    assert np.all(mant[zero] == 0)
+    small = ~zero & (e_ora <= 53)
+    np.testing.assert_array_equal(np.ldexp(mant[small], expo[small]), np.ldexp(m_ora[small], e_ora[small]))
+    big = ~zero & ~small
+    rel = np.abs(mant[big] / m_ora[big] * np.exp2((expo[big] - e_ora[big]).astype(np.float64)) - 1.0)
+    assert rel.size == 0 or rel.max() <= 1e-12, rel.max()
+
+
+def test_xr_mesh_sigma_beyond_fp64():
+    """700^2 mesh: sigma up to ~2^1393 from a corner, exported as mantissa + exponent, against the long
+    double oracle; auto mode re-runs the overflowing sources in extended range."""
+    g = gg.grid(700, 700)
+    src = np.array([0, 699, 700 * 350 + 350, 700 * 700 - 1, 12345], dtype=np.int32)
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, False) as G:
+        G.set_batch(tbc.ENGINE_NARROW)
+        depth, mant, expo = G.bfs_batch_ext(src)
+        assert G.stats()["xr_sources"] >= 3  # the corners overflow fp64
+    assert expo.max() > 1300
+    for i, s in enumerate(src):
+        d_o, m_o, e_o = oracle.bfs_ld(g.col_ptr, g.row_idx, int(s))
+        np.testing.assert_array_equal(depth[i], d_o)
+        _assert_sigma_ext(mant[i], expo[i], m_o, e_o)
+
+
+def test_xr_mesh_bc_vs_long_double_oracle():
+    """bc on a 560^2 mesh (sigma ~2^1113 from a corner) with sources that overflow fp64 and others that
+    do not, against the long double oracle (1e-9), in auto and forced extended mode."""
+    g = gg.grid(560, 560)
+    src = np.concatenate([[0, 559, 560 * 559, 560 * 560 - 1], gg.sources(g, 20, seed=3)]).astype(np.int32)
+    want = oracle.bc_ld(g.col_ptr, g.row_idx, False, src)
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, False) as G:
+        G.set_batch(tbc.ENGINE_NARROW)
+        assert_bc(G.bc(src), want)
+        assert G.stats()["xr_sources"] >= 4
+        G.set_sigma_mode(1)
+        G.reset_stats()
+        assert_bc(G.bc(src), want)
+        assert G.stats()["xr_sources"] == len(src)
+
+
+@pytest.mark.parametrize("directed", [False, True])
+def test_xr_forced_matches_fp64_oracle(directed):
+    """Extended-range arithmetic everywhere (TBC_OPT_SIGMA = 1) on graphs fp64 handles: scale-free
+    (hubs: warp paths of the sigma pull and the backward), small closed forms, random digraphs."""
+    cases = [gg.kronecker(14, 16, seed=11, directed=directed, device="cuda"), gg.grid(40, 40)]
+    if not directed:
+        cases += [gg.star(9), gg.cycle(9), gg.complete_bipartite(3, 5), gg.mycielski(7)]
+    for g in cases:
+        src = gg.sources(g, min(g.n, 120), seed=4)
+        with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+            G.set_batch(tbc.ENGINE_NARROW)
+            G.set_sigma_mode(1)
+            assert_bc(G.bc(src), oracle.bc(g.col_ptr, g.row_idx, g.directed, src))
+            depth, sigma = G.bfs_batch(src[:4])
+            assert_bfs_rows(g, src[:4], depth, sigma)
+
+
+def test_cfg8_literal_mesh_4096():
+    """BASELINE configs[3] taken literally: the 4096^2 average-degree-4 mesh (sigma ~2^8190 from a
+    corner).  One corner source's depth and sigma against the long double oracle, and the delta-sum
+    invariant sum_v bc_s(v) = 1/2 sum_t (depth_s(t) - 1) for three sources, in the auto engine."""
+    g, src = gg.make_config(8)
+    corner = 0
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, False) as G:
+        depth, mant, expo = G.bfs_batch_ext([corner])
+        d_o, m_o, e_o = oracle.bfs_ld(g.col_ptr, g.row_idx, corner)
+        np.testing.assert_array_equal(depth[0], d_o)
+        _assert_sigma_ext(mant[0], expo[0], m_o, e_o)
+        assert expo.max() > 8000
+        for s in (corner, int(src[0]), int(src[1])):
+            d = depth[0] if s == corner else G.bfs_batch([s])[0][0]
+            want = 0.5 * float(np.sum(d[d > 0] - 1))
+            got = G.bc([s]).sum()
+            assert abs(got - want) <= 1e-9 * want
+        assert G.stats()["engine"] == 2 and G.stats()["xr_sources"] >= 1

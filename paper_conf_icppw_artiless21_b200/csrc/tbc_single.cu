@@ -154,6 +154,7 @@ __device__ __forceinline__ void reset_level(VRec *rec, const int32_t *order, int
 
 struct SShared {
     int cnt[2], hcnt[2];
+    int pcnt;  // extended range: heavy vertices of the level's sigma pull
     int ovf;  // fp64 mode: a sigma left the fp64 range (the source is re-run in extended range)
     int32_t heavy[kHeavyCap];
     unsigned long long edges[2];
@@ -205,6 +206,7 @@ __device__ bool bcs_source(const SParams &P, SShared &sh, int64_t si, int32_t s,
         if (tid == 0) {  // counters of level d+2 (their level-d readers are past the barrier)
             sh.cnt[par ^ 1] = 0;
             sh.hcnt[par ^ 1] = 0;
+            sh.pcnt = 0;
         }
         const int nh = min(sh.hcnt[par], kHeavyCap);
         for (int h = warp; h < nh; h += kSWarps) {
@@ -229,7 +231,7 @@ __device__ bool bcs_source(const SParams &P, SShared &sh, int64_t si, int32_t s,
                 const int32_t w = order[i];
                 const int64_t e0 = P.in_ptr[w], e1 = P.in_ptr[w + 1];
                 if (e1 - e0 > kHeavy) {
-                    const int h = atomicAdd(&sh.hcnt[par], 1);
+                    const int h = atomicAdd(&sh.pcnt, 1);
                     if (h < kHeavyCap) {
                         sh.heavy[h] = w;
                         continue;
@@ -241,7 +243,7 @@ __device__ bool bcs_source(const SParams &P, SShared &sh, int64_t si, int32_t s,
                 rec[w].sexp = sg.e;
             }
             __syncthreads();
-            const int nh2 = min(sh.hcnt[par], kHeavyCap);
+            const int nh2 = min(sh.pcnt, kHeavyCap);
             for (int h = warp; h < nh2; h += kSWarps) {
                 const int32_t w = sh.heavy[h];
                 const int64_t e1 = P.in_ptr[w + 1];
@@ -255,7 +257,6 @@ __device__ bool bcs_source(const SParams &P, SShared &sh, int64_t si, int32_t s,
                 }
             }
             __syncthreads();
-            if (tid == 0) sh.hcnt[par] = 0;
         }
         beg = end;
         end += nn;

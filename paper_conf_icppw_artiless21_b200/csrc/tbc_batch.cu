@@ -57,6 +57,9 @@ constexpr int kPad = 8;
 #ifndef TBC_DYN_CHUNK
 #define TBC_DYN_CHUNK 1    // tiles taken per atomic in the dynamic share
 #endif
+#ifndef TBC_DYN_BIG
+#define TBC_DYN_BIG 4      // chunk multiplier on passes of > 4 M tiles
+#endif
 // gathers in flight per lane in the slot loop, by batch width (A/B on B200: W = 32 best at 6 --
 // Kronecker 25: 394 vs 389 at 4, 373 at 8; W = 64 best at 8, i.e. 4 per source -- Kronecker 22:
 // 332 vs 318 at 6, RMAT 18: 359 vs 350)
@@ -319,13 +322,16 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
     // counter by warps that ran out, so the costly tiles (many active lanes) do not leave most
     // warps waiting at the next grid barrier
     const int64_t nstat = (ntiles * TBC_STATIC_PCT) / 100;
-    int64_t dend = -1;  // end of the warp's current dynamic chunk of TBC_DYN_CHUNK tiles
+    // dynamic chunk: 1 tile per atomic, 4 on passes of > 4 M tiles (A/B on B200: Kronecker 22, whose
+    // largest passes have ~1 M tiles, is best at 1; Kronecker 25, ~16 M, at 4: 402 -> 426 GTEPS)
+    const int chunk = ntiles > (4ll << 20) ? TBC_DYN_BIG * TBC_DYN_CHUNK : TBC_DYN_CHUNK;
+    int64_t dend = -1;  // end of the warp's current dynamic chunk
     for (int64_t tile = gwarp;;) {
         if (tile >= nstat && tile >= dend) {
             unsigned long long t = 0;
             if (lane == 0) t = atomicAdd(dyn, 1ull);
-            tile = nstat + (int64_t)__shfl_sync(FULL, t, 0) * TBC_DYN_CHUNK;
-            dend = tile + TBC_DYN_CHUNK;
+            tile = nstat + (int64_t)__shfl_sync(FULL, t, 0) * chunk;
+            dend = tile + chunk;
         }
         if (tile >= ntiles) break;
         BPROF_START();

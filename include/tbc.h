@@ -135,6 +135,9 @@ enum {
     TBC_OPT_BATCH_LIST = 19, /* batched engine: level-list entries allocated per vertex (1..64, default 2;
                                 capped at W).  A sweep whose lists outgrow them is re-run as two half
                                 sweeps (tbc_stats.list_overflows) and the next call doubles them. */
+    TBC_OPT_NARROW_SLOTS = 22, /* narrow-level engine: sources run concurrently (one CTA each), 0 = auto
+                                (default: as many CTAs as are resident, within 60 % of the free memory,
+                                40 B/vertex each) */
     TBC_OPT_SIGMA = 21,      /* narrow-level engine: 0 (default) fp64 sigma, and a source whose sigma
                                 leaves the fp64 range (inf; meshes: sigma = C(i+j, i) from a corner) is
                                 re-run with extended-range sigma and delta_u (mantissa + int32

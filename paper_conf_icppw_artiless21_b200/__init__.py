@@ -26,7 +26,7 @@ ENGINE_CSC, ENGINE_COOT = 0, 1
 FLAG_ONE_FORMAT, FLAG_NO_VALIDATE, FLAG_NO_REORDER = 1, 2, 4
 OPT_DIRECTION, OPT_BWD_DIRECTION, OPT_TRACE, OPT_FORMAT, OPT_PARTITIONS = 1, 2, 3, 4, 11
 OPT_BATCH, OPT_BATCH_PULL, OPT_BATCH_WIDTH, OPT_BATCH_PARTS, OPT_BATCH_ORDER = 12, 13, 14, 16, 17
-OPT_NARROW_WIDTH, OPT_BATCH_LIST, OPT_STAGE, OPT_SIGMA = 18, 19, 20, 21
+OPT_NARROW_WIDTH, OPT_BATCH_LIST, OPT_STAGE, OPT_SIGMA, OPT_NARROW_SLOTS = 18, 19, 20, 21, 22
 ENGINE_AUTO, ENGINE_PER_SOURCE, ENGINE_BATCHED, ENGINE_NARROW = -1, 0, 1, 2
 OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8, "scan": 9, "bpush": 10}
 FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
@@ -185,6 +185,10 @@ class Graph:
         _check(lib().tbc_bfs_batch_ext(self._h, _p(src, ctypes.c_int32) if src.size else None, src.size,
                                        _p(depth, ctypes.c_int32), _p(mant, ctypes.c_double), _p(expo, ctypes.c_int32)))
         return depth, mant, expo
+
+    def set_narrow_slots(self, slots: int):
+        """Narrow-level engine: sources run concurrently, one CTA each (TBC_OPT_NARROW_SLOTS, 0 auto)."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_NARROW_SLOTS, float(slots)))
 
     def set_sigma_mode(self, mode: int):
         """Narrow-level engine: 0 fp64 sigma with an extended-range re-run on overflow (default), 1 always

@@ -556,6 +556,13 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->batch = v;
         return TBC_OK;
     }
+    if (key == TBC_OPT_NARROW_SLOTS) {
+        int v = (int)value;
+        if (v < 0 || (double)v != value) return set_error(TBC_ERR_INVALID, "narrow slots %g", value);
+        g->narrow_slots = v;
+        if (g->sws.slots > 1) single_free(g);  // re-sized at the next call
+        return TBC_OK;
+    }
     if (key == TBC_OPT_SIGMA) {
         int v = (int)value;
         if (v < 0 || v > 1 || (double)v != value) return set_error(TBC_ERR_INVALID, "sigma mode %g not 0 or 1", value);

@@ -210,6 +210,7 @@ struct tbc_graph {
     int stage = 0;                // TBC_OPT_STAGE: 0 forward + backward, 1 forward only (measurement)
     int batch = -1;               // TBC_OPT_BATCH: -1 auto, 0 per source, 1 batched, 2 narrow-level
     int narrow = -1;              // auto choice, settled by the first call's probe: 1 narrow-level engine
+    int narrow_slots = 0;         // TBC_OPT_NARROW_SLOTS: concurrent sources of the narrow engine (0 auto)
     double narrow_width = 4096.0; // TBC_OPT_NARROW_WIDTH: probe's vertices per level below which auto is narrow
     double probe_width = 0.0;     // the probe's measured vertices per level (tbc_stats)
     int last_mode = -1;           // engine of the latest bc call (0 per source, 1 batched, 2 narrow-level)

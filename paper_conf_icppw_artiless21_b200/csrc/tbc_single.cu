@@ -34,7 +34,10 @@ namespace tbc {
 namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
-constexpr int kSB = 512;            // threads per CTA
+#ifndef TBC_SBLOCK
+#define TBC_SBLOCK 512
+#endif
+constexpr int kSB = TBC_SBLOCK;     // threads per CTA
 constexpr int kSWarps = kSB / 32;
 constexpr int kHeavy = 32;          // out-degree above which a whole warp handles the vertex
 constexpr int kHeavyCap = 2048;     // heavy vertices queued per level (overflow: handled by one thread)
@@ -447,6 +450,7 @@ static tbc_status single_alloc(tbc_graph *g, bool probe_only = false) {
     size_t fr = 0, tot = 0;
     if ((e = cudaMemGetInfo(&fr, &tot))) return cuda_error(e, "cudaMemGetInfo");
     int64_t slots = probe_only ? 1 : (int64_t)per_sm * sms;
+    if (!probe_only && g->narrow_slots > 0 && slots > g->narrow_slots) slots = g->narrow_slots;
     const int64_t fit = (int64_t)(0.6 * (double)fr / (double)single_slot_bytes(g));
     if (slots > fit) slots = fit;
     if (slots < 1) slots = 1;

@@ -61,6 +61,8 @@ for setting in a.settings.split(";"):
     G.set_bwd_direction(int(kv.get("bwd", 0)))
     G.set_partitions(int(kv.get("parts", 8)))
     G.set_batch(int(kv.get("batch", 1)))
+    if "slots" in kv:
+        G.set_narrow_slots(int(kv["slots"]))
     G.set_batch_width(int(kv.get("width", 0)))
     G.set_batch_pull(float(kv.get("bpull", 8)))
     G.set_batch_parts(int(kv.get("bparts", 0)))

@@ -190,41 +190,68 @@ __device__ bool bcs_source(const SParams &P, SShared &sh, int64_t si, int32_t s,
     bool probe_stop = false;
     for (;;) {
         const int par = d & 1;
-        for (int i = beg + tid; i < end; i += kSB) {
+        // two frontier vertices per thread and iteration; low-degree ones (<= kLight out-edges: lattices,
+        // road networks) issue all their edge loads, then all depth loads, together
+        for (int i = beg + tid; i < end; i += 2 * kSB) {
             if (P.probe_cap > 0 && end + *(volatile int *)&sh.cnt[par] > P.probe_cap) break;
-            const int32_t u = order[i];
-            const int64_t e0 = P.out_ptr[u], e1 = P.out_ptr[u + 1];
-            my_edges += (unsigned long long)(e1 - e0);
-            const double su = XR ? 0.0 : __ldcg(&rec[u].sd);
-            if (!XR && !(su <= 1.7976931348623157e308)) sh.ovf = 1;  // inf: out of the fp64 range
-            if (e1 - e0 > kHeavy) {
-                const int h = atomicAdd(&sh.hcnt[par], 1);
-                if (h < kHeavyCap) {
-                    sh.heavy[h] = u;
-                    continue;
+            int32_t uu[2];
+            int64_t b0[2], b1[2];
+            double su[2];
+            bool lt[2];
+            uu[0] = order[i];
+            uu[1] = i + kSB < end ? order[i + kSB] : -1;
+#pragma unroll
+            for (int t = 0; t < 2; ++t) {
+                b0[t] = b1[t] = 0;
+                su[t] = 0.0;
+                if (uu[t] >= 0) {
+                    b0[t] = P.out_ptr[uu[t]];
+                    b1[t] = P.out_ptr[uu[t] + 1];
+                    su[t] = XR ? 0.0 : __ldcg(&rec[uu[t]].sd);
                 }
             }
-            if (e1 - e0 <= kLight) {  // low degree (lattices, road networks): all loads of a step in flight
-                int32_t w[kLight];
-                int dw[kLight];
 #pragma unroll
-                for (int q = 0; q < kLight; ++q) w[q] = e0 + q < e1 ? P.out_idx[e0 + q] : -1;
-#pragma unroll
-                for (int q = 0; q < kLight; ++q) dw[q] = w[q] >= 0 ? __ldcg(&rec[w[q]].depth) : -2;
-#pragma unroll
-                for (int q = 0; q < kLight; ++q) {
-                    if (dw[q] == -1) {
-                        dw[q] = atomicCAS(&rec[w[q]].depth, -1, d + 1);
-                        if (dw[q] == -1) {
-                            order[end + atomicAdd(&sh.cnt[par], 1)] = w[q];
-                            dw[q] = d + 1;
-                        }
+            for (int t = 0; t < 2; ++t) {
+                lt[t] = false;
+                if (uu[t] < 0) continue;
+                my_edges += (unsigned long long)(b1[t] - b0[t]);
+                if (!XR && !(su[t] <= 1.7976931348623157e308)) sh.ovf = 1;  // inf: out of the fp64 range
+                if (b1[t] - b0[t] > kHeavy) {
+                    const int h = atomicAdd(&sh.hcnt[par], 1);
+                    if (h < kHeavyCap) {
+                        sh.heavy[h] = uu[t];
+                        uu[t] = -1;
+                        continue;
                     }
-                    if (!XR && dw[q] == d + 1) atomicAdd(&rec[w[q]].sd, su);
                 }
-            } else {
-                for (int64_t e = e0; e < e1; ++e) relax<XR>(rec, order, P.out_idx[e], d, su, &sh.cnt[par], end);
+                lt[t] = b1[t] - b0[t] <= kLight;
             }
+            int32_t w[2 * kLight];
+            int dw[2 * kLight];
+#pragma unroll
+            for (int q = 0; q < 2 * kLight; ++q) {
+                const int t = q / kLight;
+                const int64_t e = b0[t] + q % kLight;
+                w[q] = (lt[t] && e < b1[t]) ? P.out_idx[e] : -1;
+            }
+#pragma unroll
+            for (int q = 0; q < 2 * kLight; ++q) dw[q] = w[q] >= 0 ? __ldcg(&rec[w[q]].depth) : -2;
+#pragma unroll
+            for (int q = 0; q < 2 * kLight; ++q) {
+                if (dw[q] == -1) {
+                    dw[q] = atomicCAS(&rec[w[q]].depth, -1, d + 1);
+                    if (dw[q] == -1) {
+                        order[end + atomicAdd(&sh.cnt[par], 1)] = w[q];
+                        dw[q] = d + 1;
+                    }
+                }
+                if (!XR && dw[q] == d + 1) atomicAdd(&rec[w[q]].sd, su[q / kLight]);
+            }
+#pragma unroll
+            for (int t = 0; t < 2; ++t)
+                if (uu[t] >= 0 && !lt[t])
+                    for (int64_t e = b0[t]; e < b1[t]; ++e)
+                        relax<XR>(rec, order, P.out_idx[e], d, su[t], &sh.cnt[par], end);
         }
         __syncthreads();
         if (tid == 0) {  // counters of level d+2 (their level-d readers are past the barrier)
@@ -343,36 +370,62 @@ __device__ bool bcs_source(const SParams &P, SShared &sh, int64_t si, int32_t s,
     for (int L = D; L >= 1; --L) {
         const int par = L & 1;
         const int b0 = lvl[L], b1 = lvl[L + 1];
-        for (int i = b0 + tid; i < b1; i += kSB) {
-            const int32_t v = order[i];
-            const int64_t e0 = P.out_ptr[v], e1 = P.out_ptr[v + 1];
-            my_bwd += (unsigned long long)(e1 - e0);
-            if (e1 - e0 > kHeavy) {
-                const int h = atomicAdd(&sh.hcnt[par], 1);
-                if (h < kHeavyCap) {
-                    sh.heavy[h] = v;
-                    continue;
+        for (int i = b0 + tid; i < b1; i += 2 * kSB) {
+            int32_t vv[2];
+            int64_t c0[2], c1[2];
+            bool lt[2];
+            vv[0] = order[i];
+            vv[1] = i + kSB < b1 ? order[i + kSB] : -1;
+#pragma unroll
+            for (int t = 0; t < 2; ++t) {
+                c0[t] = c1[t] = 0;
+                lt[t] = false;
+                if (vv[t] < 0) continue;
+                c0[t] = P.out_ptr[vv[t]];
+                c1[t] = P.out_ptr[vv[t] + 1];
+                my_bwd += (unsigned long long)(c1[t] - c0[t]);
+                if (c1[t] - c0[t] > kHeavy) {
+                    const int h = atomicAdd(&sh.hcnt[par], 1);
+                    if (h < kHeavyCap) {
+                        sh.heavy[h] = vv[t];
+                        vv[t] = -1;
+                        continue;
+                    }
+                }
+                lt[t] = !XR && c1[t] - c0[t] <= kLight;
+            }
+            if (!XR) {  // low-degree owners: every child load of both in flight together
+                int32_t w[2 * kLight];
+                double c[2 * kLight];
+#pragma unroll
+                for (int q = 0; q < 2 * kLight; ++q) {
+                    const int t = q / kLight;
+                    const int64_t e = c0[t] + q % kLight;
+                    w[q] = (lt[t] && e < c1[t]) ? P.out_idx[e] : -1;
+                }
+#pragma unroll
+                for (int q = 0; q < 2 * kLight; ++q) c[q] = w[q] >= 0 ? child(rec, w[q], L) : 0.0;
+#pragma unroll
+                for (int t = 0; t < 2; ++t) {
+                    if (!lt[t]) continue;
+                    double acc = 0.0;
+#pragma unroll
+                    for (int q = 0; q < kLight; ++q) acc += c[t * kLight + q];
+                    finish(P, rec, vv[t], acc);
                 }
             }
-            if (XR) {
-                Xr acc{0.0, 0};
-                for (int64_t e = e0; e < e1; ++e) acc = xr_add(acc, child_xr(rec, P.out_idx[e], L));
-                finish_xr(P, rec, v, acc);
-            } else {
-                double acc = 0.0;
-                if (e1 - e0 <= kLight) {
-                    int32_t w[kLight];
-                    double c[kLight];
 #pragma unroll
-                    for (int q = 0; q < kLight; ++q) w[q] = e0 + q < e1 ? P.out_idx[e0 + q] : -1;
-#pragma unroll
-                    for (int q = 0; q < kLight; ++q) c[q] = w[q] >= 0 ? child(rec, w[q], L) : 0.0;
-#pragma unroll
-                    for (int q = 0; q < kLight; ++q) acc += c[q];
+            for (int t = 0; t < 2; ++t) {
+                if (vv[t] < 0 || lt[t]) continue;
+                if (XR) {
+                    Xr acc{0.0, 0};
+                    for (int64_t e = c0[t]; e < c1[t]; ++e) acc = xr_add(acc, child_xr(rec, P.out_idx[e], L));
+                    finish_xr(P, rec, vv[t], acc);
                 } else {
-                    for (int64_t e = e0; e < e1; ++e) acc += child(rec, P.out_idx[e], L);
+                    double acc = 0.0;
+                    for (int64_t e = c0[t]; e < c1[t]; ++e) acc += child(rec, P.out_idx[e], L);
+                    finish(P, rec, vv[t], acc);
                 }
-                finish(P, rec, v, acc);
             }
         }
         if (L + 2 <= D) reset_level(rec, order, lvl[L + 2], lvl[L + 3]);

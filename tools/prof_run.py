@@ -16,6 +16,8 @@ kv = dict(x.split("=") for x in a.settings.split(",") if x)
 G.set_format(int(kv.get("fmt", 0)))
 G.set_direction(int(kv.get("dir", 0)))
 G.set_bwd_direction(int(kv.get("bwd", 0)))
+if "batch" in kv:
+    G.set_batch(int(kv["batch"]))
 s = torch.from_numpy(src).cuda()
 bc = torch.zeros(g.n, dtype=torch.float64, device="cuda")
 for _ in range(2):

@@ -40,7 +40,10 @@ constexpr unsigned FULL = 0xffffffffu;
 constexpr int kSB = TBC_SBLOCK;     // threads per CTA
 constexpr int kSWarps = kSB / 32;
 constexpr int kHeavy = 32;          // out-degree above which a whole warp handles the vertex
-constexpr int kLight = 4;           // out-degree up to which a vertex's edge loads are issued together
+constexpr int kLight = 4;
+#ifndef TBC_DIRECT_CAS
+#define TBC_DIRECT_CAS 0            // 1: claim low-degree targets with the CAS alone (no depth pre-load)
+#endif           // out-degree up to which a vertex's edge loads are issued together
 constexpr int kHeavyCap = 2048;     // heavy vertices queued per level (overflow: handled by one thread)
 
 struct SParams {
@@ -235,11 +238,12 @@ __device__ bool bcs_source(const SParams &P, SShared &sh, int64_t si, int32_t s,
                 w[q] = (lt[t] && e < b1[t]) ? P.out_idx[e] : -1;
             }
 #pragma unroll
-            for (int q = 0; q < 2 * kLight; ++q) dw[q] = w[q] >= 0 ? __ldcg(&rec[w[q]].depth) : -2;
+            for (int q = 0; q < 2 * kLight; ++q)
+                dw[q] = w[q] < 0 ? -2 : TBC_DIRECT_CAS ? atomicCAS(&rec[w[q]].depth, -1, d + 1) : __ldcg(&rec[w[q]].depth);
 #pragma unroll
             for (int q = 0; q < 2 * kLight; ++q) {
                 if (dw[q] == -1) {
-                    dw[q] = atomicCAS(&rec[w[q]].depth, -1, d + 1);
+                    if (!TBC_DIRECT_CAS) dw[q] = atomicCAS(&rec[w[q]].depth, -1, d + 1);
                     if (dw[q] == -1) {
                         order[end + atomicAdd(&sh.cnt[par], 1)] = w[q];
                         dw[q] = d + 1;

@@ -36,6 +36,9 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
     return t;
 }
 
-constexpr unsigned long long kWatchdogNs = 20ull * 1000 * 1000 * 1000;  // 20 s at one barrier
+#ifndef TBC_WATCHDOG_S
+#define TBC_WATCHDOG_S 20
+#endif
+constexpr unsigned long long kWatchdogNs = TBC_WATCHDOG_S * 1000ull * 1000 * 1000;  // at one barrier (sanitizer builds: longer)
 
 }  // namespace tbc

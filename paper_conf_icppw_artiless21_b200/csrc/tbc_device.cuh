@@ -11,6 +11,14 @@ __device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
     return v;
 }
 
+// tid.x through a volatile move: values derived from it cannot be rematerialised from S2R, so the
+// compiler keeps them in registers (see k_bcb)
+__device__ __forceinline__ unsigned tid_opaque() {
+    unsigned t;
+    asm volatile("mov.u32 %0, %%tid.x;" : "=r"(t));
+    return t;
+}
+
 __device__ __forceinline__ void fence_acq_rel() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
 
 __device__ __forceinline__ uint64_t policy_evict_first() {

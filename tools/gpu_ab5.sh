@@ -1,0 +1,6 @@
+#!/bin/bash
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests/test_gpu_full.py tests/test_gpu_parity.py -m gpu -x -q -k "bfs_batch_small or bfs_batch_kronecker or overflow or one_format_directed or cfg3_full or cfg2_full or batched or random_small or closed or hub" > gpurun_out/ab5_tests.log 2>&1
+echo "default tests rc=$? $(tail -1 gpurun_out/ab5_tests.log)"
+AB_VARIANTS="|-DTBC_OPAQUE_LANE=1" AB_CONFIGS="3|2" AB_REPS=2 AB_STEPS=3 bash tools/gpu_ab.sh
+AB_VARIANTS="|-DTBC_S_OPAQUE=1" AB_CONFIGS="4|1" AB_REPS=2 AB_STEPS=2 bash tools/gpu_ab.sh

@@ -57,9 +57,6 @@ constexpr int kPad = 8;
 #ifndef TBC_DYN_CHUNK
 #define TBC_DYN_CHUNK 1    // tiles taken per atomic in the dynamic share
 #endif
-#ifndef TBC_OPAQUE_LANE
-#define TBC_OPAQUE_LANE 0  // 1: lane / tid of every pass from an opaque tid.x read as well
-#endif
 #ifndef TBC_DYN_BIG
 #define TBC_DYN_BIG 4      // chunk multiplier on passes of > 4 M tiles
 #endif
@@ -70,12 +67,6 @@ constexpr int kBU = TBC_BUNROLL;
 constexpr int kBU64 = TBC_BUNROLL64;
 
 enum { B_PUSH = 0, B_PULL = 1, B_BWD = 2, B_BPUSH = 3 };  // B_BPUSH: one-format backward push
-
-#if TBC_OPAQUE_LANE
-#define LANE_ID() ((int)(tid_opaque() & 31u))
-#else
-#define LANE_ID() ((int)(threadIdx.x & 31))
-#endif
 
 // lane-mask word of a batch of W sources: lane l of a warp holds sources l and (W = 64) l + 32
 template <int W> struct MaskT { using T = uint32_t; };
@@ -234,7 +225,7 @@ struct BOut {
 // the start owner of every tile whose first item lies in its merge-path span (tbc_engine.cu)
 __device__ __forceinline__ void bappend(const bool (&take)[kBI], const int32_t (&v)[kBI], const uint32_t (&dg)[kBI],
                                         const uint32_t (&bg)[kBI], const BOut &o, int ebits) {
-    const int lane = LANE_ID();
+    const int lane = threadIdx.x & 31;
     const unsigned lt = (1u << lane) - 1u;
     unsigned cnt = 0;
     unsigned long long esum = 0;
@@ -287,7 +278,7 @@ __device__ __forceinline__ void span(const int64_t *ptr, int32_t v, uint32_t &dg
 // 32 x 32 bit transpose across the warp: lane l holds row l (bit c = column c); afterwards lane c
 // holds column c (bit l = row l).  Five rounds of block swaps with the partner lane l ^ j.
 __device__ __forceinline__ uint32_t transpose32(uint32_t x) {
-    const int lane = LANE_ID();
+    const int lane = threadIdx.x & 31;
     constexpr uint32_t hi[5] = {0xFFFF0000u, 0xFF00FF00u, 0xF0F0F0F0u, 0xCCCCCCCCu, 0xAAAAAAAAu};
 #pragma unroll
     for (int r = 0; r < 5; ++r) {
@@ -322,7 +313,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
     MT *fr_out = static_cast<MT *>(fr_out_);
     const MT *vis = static_cast<const MT *>(P.vis);
     const MT active = (MT)active_;
-    const int lane = LANE_ID();
+    const int lane = threadIdx.x & 31;
     const int64_t K = N + E;
     const int64_t ntiles = cdiv(K, kBT);
     const uint64_t pol = policy_evict_first();
@@ -635,7 +626,7 @@ __device__ __forceinline__ void bclear(const BParams &P, const Lv &l, void *fr_,
     MT *fr = static_cast<MT *>(fr_);
     MT *vis = static_cast<MT *>(P.vis);
     const MT *lm = static_cast<const MT *>(P.list_m);
-    const int lane = LANE_ID();
+    const int lane = threadIdx.x & 31;
     for (int64_t base = gwarp * 32; base < l.N; base += nwarps * 32) {
         const int64_t p = base + lane;
         int32_t v = -1;
@@ -675,7 +666,7 @@ __device__ __forceinline__ void bowner(const BParams &P, const Lv &l, int64_t gw
     using MT = typename MaskT<W>::T;
     constexpr int NS = W / 32;
     const MT *lm = static_cast<const MT *>(P.list_m);
-    const int lane = LANE_ID();
+    const int lane = threadIdx.x & 31;
     for (int64_t base = gwarp * 32; base < l.N; base += nwarps * 32) {
         const int64_t p = base + lane;
         int32_t v = -1;
@@ -720,11 +711,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
     // pressure (~18 % of the instructions; A/B on B200: Kronecker 22 357 -> 366, RMAT 18 ~370 -> 404)
     const unsigned wtid = tid_opaque();
     BWarpSmem &ws = reinterpret_cast<BWarpSmem *>(bsm)[wtid >> 5];
-#if TBC_OPAQUE_LANE
-    const int tid = (int)wtid, lane = tid & 31;
-#else
     const int tid = threadIdx.x, lane = tid & 31;
-#endif
     const bool cta0 = lcta == 0;
     const unsigned ncta = MULTI ? (unsigned)S.cta_per_part : gridDim.x;
     const int64_t nwarps = (int64_t)ncta * kBWarps;
@@ -1196,7 +1183,7 @@ int batch_width(const tbc_graph *g) {
 __global__ void k_source_keys(int64_t k, int64_t n, const int32_t *__restrict__ src, const int32_t *__restrict__ perm,
                               const int2 *__restrict__ deg2, const int64_t *__restrict__ out_ptr,
                               const int32_t *__restrict__ out_idx, uint32_t *keys, int32_t *vals) {
-    const int lane = LANE_ID();
+    const int lane = threadIdx.x & 31;
     const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
     for (int64_t i = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); i < k; i += nw) {
         const int32_t sc = src[i];

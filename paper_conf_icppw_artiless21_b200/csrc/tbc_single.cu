@@ -30,10 +30,6 @@
 #include "tbc_internal.cuh"
 #include "tbc_device.cuh"
 
-#ifndef TBC_S_OPAQUE
-#define TBC_S_OPAQUE 0  // 1: tid from an opaque tid.x read (see k_bcb)
-#endif
-
 namespace tbc {
 namespace {
 
@@ -176,11 +172,7 @@ struct SShared {
 template <bool XR>
 __device__ bool bcs_source(const SParams &P, SShared &sh, int64_t si, int32_t s, VRec *rec, int32_t *order,
                            int32_t *lvl) {
-#if TBC_S_OPAQUE
-    const int tid = (int)tid_opaque(), lane = tid & 31, warp = tid >> 5;
-#else
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-#endif
     const int64_t n = P.n;
     if (tid == 0) {  // level 0 (Alg.1 l.15-18)
         rec[s].depth = 0;

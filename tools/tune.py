@@ -50,7 +50,7 @@ elif os.environ.get("TUNE_SORT", "").startswith("hop2"):
         src = src[np.lexsort((-hop2[src], -cls))]
     else:  # hop2deg: out-degree, ties by 2-hop volume
         src = src[np.lexsort((-hop2[src], -od[src]))]
-G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed)
+G = tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed, one_format=os.environ.get("TUNE_ONE_FORMAT") == "1")
 s_d = torch.from_numpy(src).cuda()
 bc = torch.zeros(g.n, dtype=torch.float64, device="cuda")
 st = torch.cuda.current_stream()

@@ -118,8 +118,10 @@ enum {
                                 vertices, and above that for average degree >= 8 when the W = 64
                                 workspace fits 85 % of the free memory, else 32 (measured, DESIGN.md
                                 4.5); a W = 64 workspace that then fails to allocate falls back to 32.
-                                Workspace per SM partition ~ 16 W B/vertex of (sigma, delta_u) rows +
-                                TBC_OPT_BATCH_LIST x (12 + W/8) B/vertex of level lists + tile starts. */
+                                Workspace per SM partition ~ 8 W B/vertex of rows (sigma, overwritten by
+                                delta_u in the backward; 16 W with the separate delta_u accumulators of
+                                TBC_FLAG_ONE_FORMAT graphs) + TBC_OPT_BATCH_LIST x (12 + W/8 + 16)
+                                B/vertex of level lists and split accumulators + tile starts. */
     TBC_OPT_BATCH_PARTS = 16, /* batched engine: SM partitions (1..8, or 0 = auto, the default: 1 for
                                 graphs whose sigma rows overflow 1 GiB with average degree >= 8 or
                                 with average degree >= 64, else up to 4 (average degree >= 8) or 8
@@ -133,8 +135,9 @@ enum {
     TBC_OPT_NARROW_WIDTH = 18, /* auto engine: probe vertices per level below which the narrow-level
                                 engine runs (default 4096; setting it re-runs the probe next call) */
     TBC_OPT_BATCH_LIST = 19, /* batched engine: level-list entries allocated per vertex (1..64, default 2;
-                                capped at W).  A sweep whose lists outgrow them is re-run as two half
-                                sweeps (tbc_stats.list_overflows) and the next call doubles them. */
+                                capped at W), and split-owner accumulator values per vertex and level
+                                parity.  A sweep that outgrows either is re-run as two half sweeps
+                                (tbc_stats.list_overflows) and the next call doubles them. */
     TBC_OPT_NARROW_SLOTS = 22, /* narrow-level engine: sources run concurrently (one CTA each), 0 = auto
                                 (default: as many CTAs as are resident, within 60 % of the free memory,
                                 40 B/vertex each) */

@@ -98,7 +98,11 @@ struct BParams {
     const int64_t *__restrict__ out_ptr;
     const int32_t *__restrict__ out_idx;
     const int2 *__restrict__ deg2;
-    double *sig, *du;
+    double *sig, *du;  // du == sig when the backward runs in place (two-format graphs)
+    double *sacc;      // in place: [2][sacc_cap] split owners' partial sums by level parity
+    int64_t *scnt;     // in place: split lanes per level of the sweep
+    int64_t sacc_cap;
+    int inplace;
     void *vis;        // MaskT<W>[n]
     void *fr0, *fr1;  // MaskT<W>[n]
     int32_t *list_v;
@@ -150,6 +154,7 @@ struct __align__(16) BWarpSmem {
     int32_t own[kBT + 2];    // owner (window index) of each slot
     int32_t x[kBT];          // other end of each slot
     int32_t claim[kBT + 2];  // vertices discovered by this tile (PULL)
+    uint32_t soff[kBT + 2];  // BWD in place: split owners' offsets in the split accumulator
 };
 constexpr size_t kBSmem = sizeof(BWarpSmem) * kBWarps;
 
@@ -304,7 +309,8 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                                       const uint32_t *obeg, const void *omsk_, const int32_t *otiles, int64_t N,
                                       int64_t E, const int32_t *__restrict__ adj_idx, const void *emsk_,
                                       void *fr_out_, unsigned long long active_, int64_t gwarp, int64_t nwarps,
-                                      const BOut &out, unsigned long long *dyn) {
+                                      const BOut &out, unsigned long long *dyn, const uint32_t *soff = nullptr,
+                                      double *sacc_l = nullptr) {
     using MT = typename MaskT<W>::T;
     constexpr int NS = W / 32;                 // sources per lane
     constexpr int U2 = (NS == 1 ? kBU : kBU64) / NS > 0 ? (NS == 1 ? kBU : kBU64) / NS : 1;  // gathers in flight per lane and source
@@ -356,6 +362,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             const bool whole = isf && p < pe;
             ws.msk[j] = (MODE == B_PULL) ? (MT)(~vis[v] & active) : omsk[p];
             ws.fl[j] = (isf ? 1 : 0) | (whole ? 2 : 0);
+            if (MODE == B_BWD && soff) ws.soff[j] = whole ? 0u : soff[p];
         }
         for (int sl = lane; sl < kBT; sl += 32) ws.own[sl] = -1;
         if (lane == 0) ws.first[nwin] = ne;
@@ -455,11 +462,18 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
 #ifdef TBC_PROF
         unsigned n_own = 0;
 #endif
+        uint64_t leaf = 0;  // BWD: owners first seen here without an active slot (below)
         for (int j = 0; j < nwin; ++j) {
             uint64_t bits = act & slot_range(ws.first[j], ws.first[j + 1]);
             const int fl = ws.fl[j];
             if (MODE != B_BWD && bits == 0) continue;
-            if (MODE == B_BWD && bits == 0 && !(fl & 1)) continue;
+            if (MODE == B_BWD && bits == 0) {
+                if (!(fl & 1)) continue;
+                if (j < 64) {  // (window entry 64 never starts in the tile; kept on the path below)
+                    leaf |= 1ull << j;
+                    continue;
+                }
+            }
             (void)fl;
 #ifdef TBC_PROF
             ++n_own;
@@ -576,9 +590,23 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
 #pragma unroll
                 for (int k = 0; k < NS; ++k) {
                     if (fl & 2) {
-                        if (in[k]) P.du[row + 32 * k] = 1.0 / sv[k] + acc[k];
+                        if (in[k]) P.du[row + 32 * k] = __drcp_rn(sv[k]) + acc[k];
+                    } else if (sacc_l) {
+                        // in place: a split owner's sigma row stays intact until every tile has read
+                        // it; the partial sums meet in the split accumulator, bsplit_fin writes delta_u
+                        const int b = 32 * k + lane;
+#ifdef TBC_BCHECK
+                        if (in[k] && ws.soff[j] + __popcll((unsigned long long)m) > (uint64_t)P.sacc_cap) {
+                            printf("BCHECK pass: v %d j %d soff %u popc %d cap %lld fl %d\n", v, j, ws.soff[j],
+                                   __popcll((unsigned long long)m), (long long)P.sacc_cap, fl);
+                            __trap();
+                        }
+#endif
+                        if (in[k] && acc[k] != 0.0)
+                            atomicAdd(&sacc_l[ws.soff[j] + __popcll((unsigned long long)m & ((1ull << b) - 1ull))],
+                                      acc[k]);
                     } else {
-                        const double t = acc[k] + ((fl & 1) ? 1.0 / sv[k] : 0.0);
+                        const double t = acc[k] + ((fl & 1) ? __drcp_rn(sv[k]) : 0.0);
                         if (in[k] && t != 0.0) atomicAdd(&P.du[row + 32 * k], t);
                     }
                 }
@@ -607,6 +635,47 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                 if (cl[i]) span(P.adj_ptr, cv[i], cdg[i], cbg[i]);
             }
             bappend(cl, cv, cdg, cbg, out, P.ebits);
+        }
+        if (MODE == B_BWD) {
+            // owners whose first item is in this tile and that have no active slot here (all their
+            // lanes are DAG leaves of this level, e.g. out-degree 0): delta_u = 1/sigma (l.35 with acc
+            // = 0; added by the first tile if split), no bc term, their lanes scattered to fr_out.
+            // Independent rows, so kLeafU owners per round with their sigma loads in flight together
+            // instead of one round trip per owner in the loop above
+            constexpr int kLeafU = 4;
+            while (leaf) {
+                int jq[kLeafU];
+                double s[kLeafU][NS];
+#pragma unroll
+                for (int q = 0; q < kLeafU; ++q) {
+                    jq[q] = __ffsll((long long)leaf) - 1;
+                    leaf &= leaf - 1;
+                }
+#pragma unroll
+                for (int q = 0; q < kLeafU; ++q) {
+#pragma unroll
+                    for (int k = 0; k < NS; ++k) {
+                        s[q][k] = 1.0;
+                        if (jq[q] >= 0 && (((MT)ws.msk[jq[q]] >> (32 * k + lane)) & 1u))
+                            s[q][k] = sig[(int64_t)ws.v[jq[q]] * W + 32 * k + lane];
+                    }
+                }
+#pragma unroll
+                for (int q = 0; q < kLeafU; ++q) {
+                    if (jq[q] < 0) continue;
+                    const int32_t v = ws.v[jq[q]];
+                    const MT m = (MT)ws.msk[jq[q]];
+                    const bool whole = ws.fl[jq[q]] & 2;
+#pragma unroll
+                    for (int k = 0; k < NS; ++k) {
+                        if (!((m >> (32 * k + lane)) & 1u)) continue;
+                        double *const d = P.du + (int64_t)v * W + 32 * k + lane;
+                        if (whole) *d = __drcp_rn(s[q][k]);
+                        else if (!sacc_l) atomicAdd(d, __drcp_rn(s[q][k]));  // in place: bsplit_fin
+                    }
+                    if (lane == 0) atomicOr(&fr_out[v], m);
+                }
+            }
         }
         __syncwarp();
         BPROF(BR_OWN);
@@ -651,11 +720,127 @@ __device__ __forceinline__ void bclear(const BParams &P, const Lv &l, void *fr_,
                         P.bfs_sigma[o] = P.sig[row];
                     }
                     P.sig[row] = 0.0;
-                    P.du[row] = 0.0;
+                    if (!P.inplace) P.du[row] = 0.0;
                 }
             }
         }
     }
+}
+
+// ---- in-place backward (two-format graphs): sigma and delta_u share one [n][W] array.  Pass L
+// overwrites the level-L lanes of a whole owner's row with delta_u = 1/sigma + acc (l.35) right
+// after reading sigma; the lanes of a split owner (its items span several tiles, so several warps
+// need its sigma for the bc term) keep sigma through pass L while the tiles add their partial acc
+// into a split accumulator, and bsplit_fin writes their delta_u after the pass.  Offsets into the
+// accumulator (popc of the entry's lane mask each) are assigned one level ahead, per level parity
+// (soff: cand_pre for even levels, cand_beg for odd ones -- the candidate lists are idle in the
+// backward).
+
+// list entry p (index in its level) is split: its merge-path items -- the first at pre + p, the
+// end item out-degree items later -- fall in more than one tile
+__device__ __forceinline__ bool bsplit(const BParams &P, int64_t p0, int64_t p, int32_t v) {
+    const int64_t kf = (int64_t)P.list_pre[p0 + p] + p;
+    return kf / kBT != (kf + P.deg2[v].x) / kBT;
+}
+
+// split-accumulator offsets of level L's split entries (warp-aggregated allocation from
+// salloc[L & 1]); count: also add the level's split lanes to scnt[L]
+template <int W>
+__device__ __forceinline__ void bsplit_enum(const BParams &P, int L, bool count, bool alloc, int64_t gwarp,
+                                            int64_t nwarps) {
+    using MT = typename MaskT<W>::T;
+    const MT *lm = static_cast<const MT *>(P.list_m);
+    const int lane = threadIdx.x & 31;
+    const int64_t *l = P.lvl + 4 * (int64_t)L;
+    const int64_t p0 = l[0], N = l[1];
+    uint32_t *soff = (L & 1) ? P.cand_beg : P.cand_pre;
+    for (int64_t base = gwarp * 32; base < N; base += nwarps * 32) {
+        const int64_t p = base + lane;
+        unsigned c = 0;
+        if (p < N && bsplit(P, p0, p, P.list_v[p0 + p])) c = __popcll((unsigned long long)lm[p0 + p]);
+        unsigned incl = c;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned t = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += t;
+        }
+        const unsigned tot = __shfl_sync(FULL, incl, 31);
+        if (tot == 0) continue;
+        unsigned long long b0 = 0;
+        if (lane == 0) {
+            if (alloc) b0 = atomicAdd(&P.ctr->salloc[L & 1], (unsigned long long)tot);
+            if (count) atomicAdd((unsigned long long *)&P.scnt[L], (unsigned long long)tot);
+        }
+        if (!alloc) continue;
+        b0 = __shfl_sync(FULL, b0, 0);
+#ifdef TBC_BCHECK
+        if (c && b0 + incl > (unsigned long long)P.sacc_cap)
+            printf("BCHECK enum: L %d p %lld off %llu cap %lld (not fatal if count)\n", L, (long long)p, b0 + incl,
+                   (long long)P.sacc_cap);
+#endif
+        if (c) soff[p] = (uint32_t)(b0 + incl - c);
+    }
+}
+
+// the split lanes of every level 1..D into scnt (a sweep whose largest level needs more than
+// sacc_cap is re-run in halves), with the offsets of level D
+template <int W>
+__device__ __forceinline__ void bsplit_count(const BParams &P, int D, int64_t gwarp, int64_t nwarps) {
+    for (int L = 1; L <= D; ++L) bsplit_enum<W>(P, L, true, L == D, gwarp, nwarps);
+}
+
+// after pass L: delta_u of the split entries' level-L lanes = 1/sigma + sacc (l.35), the accumulator
+// entries re-zeroed; then the offsets of level L-1
+template <int W>
+__device__ __forceinline__ void bsplit_fin(const BParams &P, int L, int64_t gwarp, int64_t nwarps) {
+    using MT = typename MaskT<W>::T;
+    constexpr int NS = W / 32;
+    const MT *lm = static_cast<const MT *>(P.list_m);
+    const int lane = threadIdx.x & 31;
+    const int64_t *l = P.lvl + 4 * (int64_t)L;
+    const int64_t p0 = l[0], N = l[1];
+    const uint32_t *soff = (L & 1) ? P.cand_beg : P.cand_pre;
+    double *const sacc = P.sacc + (L & 1) * P.sacc_cap;
+    for (int64_t base = gwarp * 32; base < N; base += nwarps * 32) {
+        const int64_t p = base + lane;
+        int32_t v = -1;
+        MT m = 0;
+        uint32_t off = 0;
+        bool sp = false;
+        if (p < N) {
+            v = P.list_v[p0 + p];
+            sp = bsplit(P, p0, p, v);
+            if (sp) {
+                m = lm[p0 + p];
+                off = soff[p];
+            }
+        }
+        unsigned todo = __ballot_sync(FULL, sp);
+        while (todo) {
+            const int q = __ffs(todo) - 1;
+            todo &= todo - 1;
+            const int32_t vq = __shfl_sync(FULL, v, q);
+            const MT mq = __shfl_sync(FULL, m, q);
+            const uint32_t oq = __shfl_sync(FULL, off, q);
+#pragma unroll
+            for (int k = 0; k < NS; ++k) {
+                const int b = 32 * k + lane;
+                if ((mq >> b) & 1u) {
+                    const int64_t row = (int64_t)vq * W + b;
+                    const uint32_t r = oq + __popcll((unsigned long long)mq & ((1ull << b) - 1ull));
+#ifdef TBC_BCHECK
+                    if (r >= P.sacc_cap) {
+                        printf("BCHECK fin: L %d v %d off %u r %u cap %lld\n", L, vq, oq, r, (long long)P.sacc_cap);
+                        __trap();
+                    }
+#endif
+                    P.sig[row] = __drcp_rn(P.sig[row]) + sacc[r];
+                    sacc[r] = 0.0;
+                }
+            }
+        }
+    }
+    if (L >= 2) bsplit_enum<W>(P, L - 1, false, true, gwarp, nwarps);
 }
 
 // one-format owner pass of level L: for each (v, lane s) on level L the row of du holds
@@ -686,7 +871,7 @@ __device__ __forceinline__ void bowner(const BParams &P, const Lv &l, int64_t gw
                     const int64_t row = (int64_t)vq * W + 32 * k + lane;
                     const double sv = P.sig[row], acc = P.du[row];
                     c += sv * acc;
-                    P.du[row] = 1.0 / sv + acc;
+                    P.du[row] = __drcp_rn(sv) + acc;
                 }
             }
 #pragma unroll
@@ -798,6 +983,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
                 C->ilist = 0;
                 C->cand[0] = 0;
                 C->dyn[0] = C->dyn[1] = 0;
+                C->salloc[0] = C->salloc[1] = 0;
             }
         }
         unsigned ph = 0;  // edge passes of this batch so far (selects the dynamic-tile counter)
@@ -922,6 +1108,22 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             prev = cur;
             cur = nxt;
         }
+        if (!overflow && P.inplace && !P.bfs_depth && !P.fwd_only) {
+            // in-place backward: split lanes per level and level D's accumulator offsets; a sweep whose
+            // largest level needs more than the accumulator holds is re-run in halves (nothing of the
+            // backward has been written yet)
+            bsplit_count<W>(P, d, gwarp, nwarps);
+            bsync(C, gen, ncta);
+            __shared__ int s_sovf;
+            if (tid == 0) {
+                long long mx = 0;
+                for (int L = 1; L <= d; ++L) mx = max(mx, (long long)ld_volatile_u64((const unsigned long long *)&P.scnt[L]));
+                s_sovf = mx > P.sacc_cap;
+            }
+            __syncthreads();
+            overflow = s_sovf != 0;
+            __syncthreads();
+        }
         if (overflow) {
             // drop the lane set's partial forward state (grid-wide, no list needed), then run its halves
             for (int64_t i = gtid; i < P.n * W; i += nthreads) P.sig[i] = 0.0;
@@ -936,6 +1138,10 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
                 C->st_overflows += 1;
                 C->ovf_total += 1;
             }
+            // split-lane counts: zeroed only after the barrier above -- every CTA has taken its
+            // overflow decision from them by then (done before the re-run's next barrier)
+            if (P.scnt)
+                for (int64_t i = gtid; i < P.n + 2; i += nthreads) P.scnt[i] = 0;
             MT lo = 0, x = bmask;
             for (int i = __popcll((unsigned long long)bmask) / 2; i > 0; --i) {
                 lo |= x & (~x + 1);
@@ -1007,10 +1213,14 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             const int64_t *l = P.lvl + 4 * (int64_t)L;
             const Lv lv{l[0], l[1], l[2], l[3]};
             const BOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0, nullptr};
-            if (cta0 && tid == 0) C->dyn[(ph + 1) & 1] = 0;  // the next pass's counter (its last user is done)
+            if (cta0 && tid == 0) {
+                C->dyn[(ph + 1) & 1] = 0;  // the next pass's counter (its last user is done)
+                if (P.inplace) C->salloc[(L + 1) & 1] = 0;  // for level L-1's offsets (bsplit_fin)
+            }
             bpass<B_BWD, W>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.list_beg + lv.p0, list_m + lv.p0,
                          P.tiles + lv.tb, lv.N, lv.E, P.out_idx, fr[(L + 1) & 1], fr[L & 1], 0u, gwarp, nwarps, none,
-                         &C->dyn[ph & 1]);
+                         &C->dyn[ph & 1], P.inplace ? ((L & 1) ? P.cand_beg : P.cand_pre) : nullptr,
+                         P.inplace ? P.sacc + (L & 1) * P.sacc_cap : nullptr);
             ++ph;
             bwd_edges += lv.E;
             if (L + 2 <= D) {
@@ -1021,12 +1231,18 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             }
             bsync(C, gen, ncta);
             btrace(P, tr, 4, L, lv.N, lv.E, 0, 0);
+            if (P.inplace) {
+                bsplit_fin<W>(P, L, gwarp, nwarps);
+                bsync(C, gen, ncta);
+            }
         }
         // retire levels 0..min(2, D)
         for (int L = 0; L <= min(2, D); ++L) {
             const int64_t *l = P.lvl + 4 * (int64_t)L;
             bclear<W>(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps);
         }
+        if (P.scnt)
+            for (int64_t L = gtid + 1; L <= D; L += nthreads) P.scnt[L] = 0;
         if (cta0 && tid == 0) {
             C->st_bwd_edges += bwd_edges;
             C->st_scans += pulls;
@@ -1074,7 +1290,14 @@ static tbc_status batch_alloc(tbc_graph *g, int q, int W) {
     w.list_cap = f * n + kPad;
     w.tiles_cap = (w.list_cap + f * m) / kBT + n + 2 + kPad;
     w.cand_tiles_cap = (n + m) / kBT + 2 + kPad;
-    if ((e = alloc(&w.sig, (size_t)n * W)) || (e = alloc(&w.du, (size_t)n * W)) || (e = alloc(&w.vis, n * nw)) ||
+    // sigma and delta_u share one [n][W] array (the backward overwrites sigma in place); the owners
+    // whose out-edges span several tiles sum their partial accumulators in sacc first, f n values per
+    // level parity (grown with the lists; a sweep that needs more is re-run in halves)
+    const bool inplace = g->out_idx != nullptr;
+    w.sacc_cap = inplace ? f * n + kPad : 0;
+    if ((e = alloc(&w.sig, (size_t)n * W)) || (!inplace && (e = alloc(&w.du, (size_t)n * W))) ||
+        (inplace && (e = alloc(&w.sacc, 2 * (size_t)w.sacc_cap))) || (inplace && (e = alloc(&w.scnt, n + 2))) ||
+        (e = alloc(&w.vis, n * nw)) ||
         (e = alloc(&w.fr[0], n * nw)) || (e = alloc(&w.fr[1], n * nw)) || (e = alloc(&w.list_v, w.list_cap)) ||
         (e = alloc(&w.list_pre, w.list_cap)) || (e = alloc(&w.list_beg, w.list_cap)) ||
         (e = alloc(&w.list_m, w.list_cap * nw)) || (e = alloc(&w.tiles, w.tiles_cap)) ||
@@ -1086,7 +1309,9 @@ static tbc_status batch_alloc(tbc_graph *g, int q, int W) {
     }
     g->device_bytes += w.bytes;
     if ((e = cudaMemsetAsync(w.sig, 0, sizeof(double) * n * W, s)) ||
-        (e = cudaMemsetAsync(w.du, 0, sizeof(double) * n * W, s)) ||
+        (w.du && (e = cudaMemsetAsync(w.du, 0, sizeof(double) * n * W, s))) ||
+        (w.sacc && (e = cudaMemsetAsync(w.sacc, 0, sizeof(double) * 2 * w.sacc_cap, s))) ||
+        (w.scnt && (e = cudaMemsetAsync(w.scnt, 0, sizeof(int64_t) * (n + 2), s))) ||
         (e = cudaMemsetAsync(w.vis, 0, sizeof(uint32_t) * n * nw, s)) ||
         (e = cudaMemsetAsync(w.fr[0], 0, sizeof(uint32_t) * n * nw, s)) ||
         (e = cudaMemsetAsync(w.fr[1], 0, sizeof(uint32_t) * n * nw, s)) ||
@@ -1130,7 +1355,7 @@ void batch_free_one(tbc_graph *g, int q) {
         }
         (void)cudaGetLastError();
     }
-    void *ps[] = {w.sig, w.du, w.vis, w.fr[0], w.fr[1], w.list_v, w.list_pre, w.list_beg, w.list_m, w.tiles,
+    void *ps[] = {w.sig, w.du, w.sacc, w.scnt, w.vis, w.fr[0], w.fr[1], w.list_v, w.list_pre, w.list_beg, w.list_m, w.tiles,
                   w.cand_v, w.cand_pre, w.cand_beg, w.cand_tiles, w.lvl, w.ctr};
     for (void *p : ps) cudaFree(p);
     g->device_bytes -= w.bytes;
@@ -1159,7 +1384,8 @@ static int64_t batch_ws_bytes(const tbc_graph *g, int W) {  // batch_alloc's siz
     const int64_t f = g->blist_factor < W ? g->blist_factor : W;
     const int64_t list_cap = f * n + kPad;
     const int64_t tiles_cap = (list_cap + f * m) / kBT + n + 2 + kPad;
-    return 16 * W * n + 12 * n * nw + list_cap * (12 + 4 * nw) + 4 * tiles_cap + 16 * (n + kPad) +
+    const int64_t rows = g->out_idx ? 8 * W * n + 16 * list_cap + 8 * n : 16 * W * n;  // in place: + sacc, scnt
+    return rows + 12 * n * nw + list_cap * (12 + 4 * nw) + 4 * tiles_cap + 16 * (n + kPad) +
            4 * ((n + m) / kBT + 2 + kPad) + 32 * (n + 2) + (int64_t)sizeof(Ctrs);
 }
 
@@ -1325,7 +1551,11 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
         P.out_idx = g->out_idx;
         P.deg2 = g->deg2;
         P.sig = w.sig;
-        P.du = w.du;
+        P.du = w.du ? w.du : w.sig;
+        P.sacc = w.sacc;
+        P.scnt = w.scnt;
+        P.sacc_cap = w.sacc_cap;
+        P.inplace = w.du ? 0 : 1;
         P.vis = w.vis;
         P.fr0 = w.fr[0];
         P.fr1 = w.fr[1];

@@ -32,6 +32,7 @@ struct Ctrs {
     unsigned long long dyn[2];    // batched engine: dynamic tile counters of consecutive edge passes
     unsigned int ovf;             // batched engine: a level list outgrew the workspace (re-run in halves)
     unsigned long long ovf_total; // batched engine: such re-runs since the workspace was allocated
+    unsigned long long salloc[2]; // batched engine (in place): split-accumulator allocation, by level parity
     unsigned long long trace_n;   // entries written to the trace buffer
     // accumulated statistics (tbc_stats)
     long long st_sources, st_reached, st_reached_edges, st_fwd_edges, st_bwd_edges, st_levels, st_pull_levels,
@@ -133,7 +134,11 @@ struct BatchWorkspace {
     int width = 0;               // W the workspace was sized for
     size_t bytes = 0;
     double *sig = nullptr;       // [n][W] sigma of (vertex, source)
-    double *du = nullptr;        // [n][W] delta_u of (vertex, source) (backward)
+    double *du = nullptr;        // [n][W] delta_u accumulators (strict one-format graphs only; else the
+                                 // backward overwrites sigma with delta_u in place, see k_bcb)
+    double *sacc = nullptr;      // [2][sacc_cap] split owners' partial sums, by level parity (in place)
+    int64_t *scnt = nullptr;     // [n + 2] split lanes per level of the current sweep (in place)
+    int64_t sacc_cap = 0;
     uint32_t *vis = nullptr;     // [n] sources that have reached the vertex (W-bit words)
     uint32_t *fr[2] = {nullptr, nullptr};  // [n] dense level masks, by level parity (W-bit words)
     int32_t *list_v = nullptr;   // level lists (levels concatenated), capacity list_cap

@@ -60,6 +60,8 @@ def parse():
     ap.add_argument("--batch", type=int, default=-1,
                     help="engine: -1 auto (level-width probe), 0 per source, 1 batched, 2 narrow-level")
     ap.add_argument("--width", type=int, default=0, help="batched engine: sources per sweep (32, 64; 0 auto)")
+    ap.add_argument("--inplace", type=int, default=-1,
+                    help="batched engine: 1 backward overwrites sigma with delta_u in place, 0 separate rows, -1 auto")
     ap.add_argument("--order", type=int, default=1, help="batched engine: 1 group sources by 2-hop out-volume, 0 as given")
     ap.add_argument("--cost", default="", help="cost model overrides, e.g. list=10,stream=2")
     ap.add_argument("--trace", type=int, default=-1, help="print the per-level timeline of this source to stderr")
@@ -277,6 +279,7 @@ def main():
     G.set_batch(1 if args.one_format and g.directed else args.batch)
     G.set_batch_width(args.width)
     G.set_batch_order(args.order)
+    G.set_batch_inplace(args.inplace)
     if args.cost:
         G.set_cost(**{k: float(v) for k, v in (kv.split("=") for kv in args.cost.split(","))})
     src_d = torch.from_numpy(np.ascontiguousarray(my_src)).to(dev)
@@ -397,7 +400,7 @@ def main():
                              if (8 * (g.n + 1) + 4 * g.nnz) * (2 if g.directed else 1) > 126e6 else
                              "graph fits in L2 (small config); no flush",
                        "direction": args.direction, "format": args.format, "engine_kind": args.engine,
-                       "one_format": bool(args.one_format and g.directed),
+                       "one_format": bool(args.one_format and g.directed), "inplace_opt": args.inplace,
                        "engine_mode": (f"batched, {wdt} sources per sweep, {st['batch_parts']} SM partition(s)"
                                        + (", sources grouped by 2-hop out-volume" if args.order
                                           else ", sources in the given order")) if eng == 1

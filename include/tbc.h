@@ -118,10 +118,9 @@ enum {
                                 vertices, and above that for average degree >= 8 when the W = 64
                                 workspace fits 85 % of the free memory, else 32 (measured, DESIGN.md
                                 4.5); a W = 64 workspace that then fails to allocate falls back to 32.
-                                Workspace per SM partition ~ 8 W B/vertex of rows (sigma, overwritten by
-                                delta_u in the backward; 16 W with the separate delta_u accumulators of
-                                TBC_FLAG_ONE_FORMAT graphs) + TBC_OPT_BATCH_LIST x (12 + W/8 + 16)
-                                B/vertex of level lists and split accumulators + tile starts. */
+                                Workspace per SM partition ~ 16 W B/vertex of (sigma, delta_u) rows
+                                (8 W + the split accumulator with TBC_OPT_BATCH_INPLACE) +
+                                TBC_OPT_BATCH_LIST x (12 + W/8) B/vertex of level lists + tile starts. */
     TBC_OPT_BATCH_PARTS = 16, /* batched engine: SM partitions (1..8, or 0 = auto, the default: 1 for
                                 graphs whose sigma rows overflow 1 GiB with average degree >= 8 or
                                 with average degree >= 64, else up to 4 (average degree >= 8) or 8
@@ -135,9 +134,10 @@ enum {
     TBC_OPT_NARROW_WIDTH = 18, /* auto engine: probe vertices per level below which the narrow-level
                                 engine runs (default 4096; setting it re-runs the probe next call) */
     TBC_OPT_BATCH_LIST = 19, /* batched engine: level-list entries allocated per vertex (1..64, default 2;
-                                capped at W), and split-owner accumulator values per vertex and level
-                                parity.  A sweep that outgrows either is re-run as two half sweeps
-                                (tbc_stats.list_overflows) and the next call doubles them. */
+                                capped at W).  A sweep whose lists outgrow them is re-run as two half
+                                sweeps (tbc_stats.list_overflows) and the next call doubles them (in
+                                place, TBC_OPT_BATCH_INPLACE: likewise a sweep whose split-owner
+                                accumulator is too small; the next call sizes it to the need). */
     TBC_OPT_NARROW_SLOTS = 22, /* narrow-level engine: sources run concurrently (one CTA each), 0 = auto
                                 (default: as many CTAs as are resident, within 60 % of the free memory,
                                 40 B/vertex each) */
@@ -146,6 +146,12 @@ enum {
                                 re-run with extended-range sigma and delta_u (mantissa + int32
                                 exponent, exact below 2^53 like fp64; tbc_stats.xr_sources); 1 always
                                 extended range.  The other engines compute in fp64 only. */
+    TBC_OPT_BATCH_INPLACE = 23, /* batched engine, two-format graphs: 1 the backward overwrites sigma with
+                                delta_u in place (8 W B/vertex of rows instead of 16 W, plus a split-owner
+                                accumulator sized to the largest level's need; one more grid barrier
+                                per backward level: ~6 % slower on Kronecker 22/25), 0 separate delta_u
+                                rows, -1 (default) auto: in place when the separate rows would not fit
+                                85 % of the free device memory (settled once per graph) */
     TBC_OPT_STAGE = 20       /* measurement: 0 (default) forward + backward; 1 forward stage only --
                                 the batched and narrow-level engines run Alg.1 l.11-28 and skip the
                                 backward stage, leaving bc untouched (per-stage HBM traffic with ncu) */

@@ -26,7 +26,7 @@ ENGINE_CSC, ENGINE_COOT = 0, 1
 FLAG_ONE_FORMAT, FLAG_NO_VALIDATE, FLAG_NO_REORDER = 1, 2, 4
 OPT_DIRECTION, OPT_BWD_DIRECTION, OPT_TRACE, OPT_FORMAT, OPT_PARTITIONS = 1, 2, 3, 4, 11
 OPT_BATCH, OPT_BATCH_PULL, OPT_BATCH_WIDTH, OPT_BATCH_PARTS, OPT_BATCH_ORDER = 12, 13, 14, 16, 17
-OPT_NARROW_WIDTH, OPT_BATCH_LIST, OPT_STAGE, OPT_SIGMA, OPT_NARROW_SLOTS = 18, 19, 20, 21, 22
+OPT_NARROW_WIDTH, OPT_BATCH_LIST, OPT_STAGE, OPT_SIGMA, OPT_NARROW_SLOTS, OPT_BATCH_INPLACE = 18, 19, 20, 21, 22, 23
 ENGINE_AUTO, ENGINE_PER_SOURCE, ENGINE_BATCHED, ENGINE_NARROW = -1, 0, 1, 2
 OPT_COST = {"list": 5, "stream": 6, "atomic": 7, "vertex": 8, "scan": 9, "bpush": 10}
 FMT_AUTO, FMT_LIST, FMT_STREAM = 0, 1, 2
@@ -216,6 +216,11 @@ class Graph:
     def set_batch_list(self, factor: int):
         """Batched engine: level-list entries allocated per vertex (TBC_OPT_BATCH_LIST, 1..64, default 2)."""
         _check(lib().tbc_graph_set_option(self._h, OPT_BATCH_LIST, float(factor)))
+
+    def set_batch_inplace(self, mode: int):
+        """Batched engine: backward overwrites sigma with delta_u in place (TBC_OPT_BATCH_INPLACE: 1 on,
+        0 off, -1 auto = in place when the separate delta_u rows would not fit the free memory)."""
+        _check(lib().tbc_graph_set_option(self._h, OPT_BATCH_INPLACE, float(mode)))
 
     def set_stage(self, stage: int):
         """Measurement: 0 forward + backward (default), 1 forward stage only (TBC_OPT_STAGE; bc untouched)."""

@@ -575,6 +575,14 @@ tbc_status tbc_graph_set_option(tbc_graph *g, int key, double value) {
         g->stage = v;
         return TBC_OK;
     }
+    if (key == TBC_OPT_BATCH_INPLACE) {
+        int v = (int)value;
+        if (v < -1 || v > 1 || (double)v != value) return set_error(TBC_ERR_INVALID, "batch in-place mode %g", value);
+        g->binplace = v;
+        g->binplace_eff = -1;
+        for (int q = 0; q < kMaxPartitions; ++q) batch_free_one(g, q);  // reallocated at the next call
+        return TBC_OK;
+    }
     if (key == TBC_OPT_BATCH_LIST) {
         int v = (int)value;
         if (v < 1 || v > 64 || (double)v != value) return set_error(TBC_ERR_INVALID, "batch list factor %g not in [1, 64]", value);

@@ -26,6 +26,7 @@
 // (l.39, l.45, 1/2 if undirected P:180) and du[v][s] = 1/sigma_s(v) + acc_s.  A vertex whose
 // out-edges span several warp tiles is "split": its partial sums are added with fp64 atomics
 // (both bc and du are linear in acc), the tile holding its first item adds the 1/sigma term.
+#include <algorithm>
 #include <cstdio>
 
 #include <cub/device/device_radix_sort.cuh>
@@ -153,8 +154,7 @@ struct __align__(16) BWarpSmem {
     int32_t fl[kBT + 2];     // bit 0: the tile holds the owner's first item; bit 1: whole owner
     int32_t own[kBT + 2];    // owner (window index) of each slot
     int32_t x[kBT];          // other end of each slot
-    int32_t claim[kBT + 2];  // vertices discovered by this tile (PULL)
-    uint32_t soff[kBT + 2];  // BWD in place: split owners' offsets in the split accumulator
+    int32_t claim[kBT + 2];  // vertices discovered by this tile (PULL); BWD in place: split owners' offsets
 };
 constexpr size_t kBSmem = sizeof(BWarpSmem) * kBWarps;
 
@@ -304,7 +304,7 @@ __device__ __forceinline__ uint64_t slot_range(int s0, int s1) {
 //   PUSH: frontier owners, out-edges;  PULL: candidates, in-edges;  BWD: level-L owners, out-edges.
 // emsk: per-vertex lane mask of the other end (PULL: M_d, BWD: M_{L+1}; PUSH uses ~vis).
 // fr_out: PUSH/PULL the next level's dense mask, BWD the owners' level (scattered M_L).
-template <int MODE, int W>
+template <int MODE, int W, bool IP = false>
 __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int32_t *ov, const uint32_t *opre,
                                       const uint32_t *obeg, const void *omsk_, const int32_t *otiles, int64_t N,
                                       int64_t E, const int32_t *__restrict__ adj_idx, const void *emsk_,
@@ -362,7 +362,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
             const bool whole = isf && p < pe;
             ws.msk[j] = (MODE == B_PULL) ? (MT)(~vis[v] & active) : omsk[p];
             ws.fl[j] = (isf ? 1 : 0) | (whole ? 2 : 0);
-            if (MODE == B_BWD && soff) ws.soff[j] = whole ? 0u : soff[p];
+            if (MODE == B_BWD && IP) ws.claim[j] = whole ? 0 : (int32_t)soff[p];
         }
         for (int sl = lane; sl < kBT; sl += 32) ws.own[sl] = -1;
         if (lane == 0) ws.first[nwin] = ne;
@@ -591,19 +591,12 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                 for (int k = 0; k < NS; ++k) {
                     if (fl & 2) {
                         if (in[k]) P.du[row + 32 * k] = __drcp_rn(sv[k]) + acc[k];
-                    } else if (sacc_l) {
+                    } else if (IP) {
                         // in place: a split owner's sigma row stays intact until every tile has read
                         // it; the partial sums meet in the split accumulator, bsplit_fin writes delta_u
                         const int b = 32 * k + lane;
-#ifdef TBC_BCHECK
-                        if (in[k] && ws.soff[j] + __popcll((unsigned long long)m) > (uint64_t)P.sacc_cap) {
-                            printf("BCHECK pass: v %d j %d soff %u popc %d cap %lld fl %d\n", v, j, ws.soff[j],
-                                   __popcll((unsigned long long)m), (long long)P.sacc_cap, fl);
-                            __trap();
-                        }
-#endif
                         if (in[k] && acc[k] != 0.0)
-                            atomicAdd(&sacc_l[ws.soff[j] + __popcll((unsigned long long)m & ((1ull << b) - 1ull))],
+                            atomicAdd(&sacc_l[(uint32_t)ws.claim[j] + __popcll((unsigned long long)m & ((1ull << b) - 1ull))],
                                       acc[k]);
                     } else {
                         const double t = acc[k] + ((fl & 1) ? __drcp_rn(sv[k]) : 0.0);
@@ -671,7 +664,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
                         if (!((m >> (32 * k + lane)) & 1u)) continue;
                         double *const d = P.du + (int64_t)v * W + 32 * k + lane;
                         if (whole) *d = __drcp_rn(s[q][k]);
-                        else if (!sacc_l) atomicAdd(d, __drcp_rn(s[q][k]));  // in place: bsplit_fin
+                        else if (!IP) atomicAdd(d, __drcp_rn(s[q][k]));  // in place: bsplit_fin
                     }
                     if (lane == 0) atomicOr(&fr_out[v], m);
                 }
@@ -687,7 +680,7 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
 // the dense mask of its parity (atomicAnd: a concurrent scatter of another level may share the word).
 // EXPORT (tbc_bfs_batch): first write depth = level and sigma of every (vertex, lane) of the list to
 // the caller's [source][vertex] arrays (source index b W + lane word)
-template <int W, bool EXPORT = false>
+template <int W, bool EXPORT = false, bool IP = false>
 __device__ __forceinline__ void bclear(const BParams &P, const Lv &l, void *fr_, int64_t gwarp, int64_t nwarps,
                                        int level = 0, int64_t b = 0) {
     using MT = typename MaskT<W>::T;
@@ -720,7 +713,7 @@ __device__ __forceinline__ void bclear(const BParams &P, const Lv &l, void *fr_,
                         P.bfs_sigma[o] = P.sig[row];
                     }
                     P.sig[row] = 0.0;
-                    if (!P.inplace) P.du[row] = 0.0;
+                    if (!IP) P.du[row] = 0.0;
                 }
             }
         }
@@ -773,11 +766,6 @@ __device__ __forceinline__ void bsplit_enum(const BParams &P, int L, bool count,
         }
         if (!alloc) continue;
         b0 = __shfl_sync(FULL, b0, 0);
-#ifdef TBC_BCHECK
-        if (c && b0 + incl > (unsigned long long)P.sacc_cap)
-            printf("BCHECK enum: L %d p %lld off %llu cap %lld (not fatal if count)\n", L, (long long)p, b0 + incl,
-                   (long long)P.sacc_cap);
-#endif
         if (c) soff[p] = (uint32_t)(b0 + incl - c);
     }
 }
@@ -828,12 +816,6 @@ __device__ __forceinline__ void bsplit_fin(const BParams &P, int L, int64_t gwar
                 if ((mq >> b) & 1u) {
                     const int64_t row = (int64_t)vq * W + b;
                     const uint32_t r = oq + __popcll((unsigned long long)mq & ((1ull << b) - 1ull));
-#ifdef TBC_BCHECK
-                    if (r >= P.sacc_cap) {
-                        printf("BCHECK fin: L %d v %d off %u r %u cap %lld\n", L, vq, oq, r, (long long)P.sacc_cap);
-                        __trap();
-                    }
-#endif
                     P.sig[row] = __drcp_rn(P.sig[row]) + sacc[r];
                     sacc[r] = 0.0;
                 }
@@ -883,7 +865,7 @@ __device__ __forceinline__ void bowner(const BParams &P, const Lv &l, int64_t gw
 
 // MULTI = false: one partition, every parameter at a static offset (S.p[0]); MULTI = true: the
 // partition's parameters are indexed by blockIdx (costs registers, so only used when P > 1)
-template <int W, bool MULTI>
+template <int W, bool MULTI, bool IP>
 __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSet S) {
     using MT = typename MaskT<W>::T;
     constexpr int NS = W / 32;
@@ -1108,7 +1090,8 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             prev = cur;
             cur = nxt;
         }
-        if (!overflow && P.inplace && !P.bfs_depth && !P.fwd_only) {
+        bool split_ovf = false;  // the split accumulator, not a level list, was outgrown (no list growth)
+        if (IP && !overflow && !P.bfs_depth && !P.fwd_only) {
             // in-place backward: split lanes per level and level D's accumulator offsets; a sweep whose
             // largest level needs more than the accumulator holds is re-run in halves (nothing of the
             // backward has been written yet)
@@ -1119,9 +1102,11 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
                 long long mx = 0;
                 for (int L = 1; L <= d; ++L) mx = max(mx, (long long)ld_volatile_u64((const unsigned long long *)&P.scnt[L]));
                 s_sovf = mx > P.sacc_cap;
+                if (cta0 && (unsigned long long)mx > C->split_need) C->split_need = (unsigned long long)mx;
             }
             __syncthreads();
             overflow = s_sovf != 0;
+            split_ovf = overflow;
             __syncthreads();
         }
         if (overflow) {
@@ -1136,7 +1121,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             if (cta0 && tid == 0) {  // every CTA has read the flag (before the barrier above)
                 C->ovf = 0;
                 C->st_overflows += 1;
-                C->ovf_total += 1;
+                if (!split_ovf) C->ovf_total += 1;
             }
             // split-lane counts: zeroed only after the barrier above -- every CTA has taken its
             // overflow decision from them by then (done before the re-run's next barrier)
@@ -1204,7 +1189,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             }
             if (L + 2 <= D) {
                 const int64_t *l2 = P.lvl + 4 * (int64_t)(L + 2);
-                bclear<W>(P, Lv{l2[0], l2[1], l2[2], l2[3]}, fr[L & 1], gwarp, nwarps);
+                bclear<W, false, IP>(P, Lv{l2[0], l2[1], l2[2], l2[3]}, fr[L & 1], gwarp, nwarps);
             }
             bsync(C, gen, ncta);
             btrace(P, tr, 4, L, l[1], l[2], 0, 0);
@@ -1215,23 +1200,23 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
             const BOut none{nullptr, nullptr, nullptr, nullptr, nullptr, 0, 0, nullptr};
             if (cta0 && tid == 0) {
                 C->dyn[(ph + 1) & 1] = 0;  // the next pass's counter (its last user is done)
-                if (P.inplace) C->salloc[(L + 1) & 1] = 0;  // for level L-1's offsets (bsplit_fin)
+                if (IP) C->salloc[(L + 1) & 1] = 0;  // for level L-1's offsets (bsplit_fin)
             }
-            bpass<B_BWD, W>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.list_beg + lv.p0, list_m + lv.p0,
+            bpass<B_BWD, W, IP>(P, ws, P.list_v + lv.p0, P.list_pre + lv.p0, P.list_beg + lv.p0, list_m + lv.p0,
                          P.tiles + lv.tb, lv.N, lv.E, P.out_idx, fr[(L + 1) & 1], fr[L & 1], 0u, gwarp, nwarps, none,
-                         &C->dyn[ph & 1], P.inplace ? ((L & 1) ? P.cand_beg : P.cand_pre) : nullptr,
-                         P.inplace ? P.sacc + (L & 1) * P.sacc_cap : nullptr);
+                         &C->dyn[ph & 1], IP ? ((L & 1) ? P.cand_beg : P.cand_pre) : nullptr,
+                         IP ? P.sacc + (L & 1) * P.sacc_cap : nullptr);
             ++ph;
             bwd_edges += lv.E;
             if (L + 2 <= D) {
                 BPROF_START();
                 const int64_t *l2 = P.lvl + 4 * (int64_t)(L + 2);
-                bclear<W>(P, Lv{l2[0], l2[1], l2[2], l2[3]}, fr[L & 1], gwarp, nwarps);
+                bclear<W, false, IP>(P, Lv{l2[0], l2[1], l2[2], l2[3]}, fr[L & 1], gwarp, nwarps);
                 BPROF(BR_CLEAR);
             }
             bsync(C, gen, ncta);
             btrace(P, tr, 4, L, lv.N, lv.E, 0, 0);
-            if (P.inplace) {
+            if (IP) {
                 bsplit_fin<W>(P, L, gwarp, nwarps);
                 bsync(C, gen, ncta);
             }
@@ -1239,7 +1224,7 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
         // retire levels 0..min(2, D)
         for (int L = 0; L <= min(2, D); ++L) {
             const int64_t *l = P.lvl + 4 * (int64_t)L;
-            bclear<W>(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps);
+            bclear<W, false, IP>(P, Lv{l[0], l[1], l[2], l[3]}, fr[L & 1], gwarp, nwarps);
         }
         if (P.scnt)
             for (int64_t L = gtid + 1; L <= D; L += nthreads) P.scnt[L] = 0;
@@ -1267,6 +1252,22 @@ __global__ void __launch_bounds__(kBB, 1) k_bcb(const __grid_constant__ BParamSe
 
 // ------------------------------------------------------------------ host side
 
+static int64_t batch_ws_bytes(const tbc_graph *g, int W, bool inplace);
+
+// in-place backward (TBC_OPT_BATCH_INPLACE): forced, or auto when the separate delta_u rows would not
+// fit 85 % of the free memory (with the workspaces already held); settled once per graph
+static bool batch_inplace(tbc_graph *g, int W) {
+    if (!g->out_idx) return false;  // one format: the backward pushes into separate accumulators
+    if (g->binplace >= 0) return g->binplace == 1;
+    if (g->binplace_eff < 0) {
+        size_t fr = 0, tot = 0;
+        double have = cudaMemGetInfo(&fr, &tot) == cudaSuccess ? 0.85 * (double)fr : 0.0;
+        for (int q = 0; q < kMaxPartitions; ++q) have += g->bws[q].ready ? (double)g->bws[q].bytes : 0.0;
+        g->binplace_eff = (double)batch_ws_bytes(g, W, false) > have ? 1 : 0;
+    }
+    return g->binplace_eff == 1;
+}
+
 static tbc_status batch_alloc(tbc_graph *g, int q, int W) {
     BatchWorkspace &w = g->bws[q];
     if (w.ready && w.width == W) return TBC_OK;
@@ -1293,8 +1294,8 @@ static tbc_status batch_alloc(tbc_graph *g, int q, int W) {
     // sigma and delta_u share one [n][W] array (the backward overwrites sigma in place); the owners
     // whose out-edges span several tiles sum their partial accumulators in sacc first, f n values per
     // level parity (grown with the lists; a sweep that needs more is re-run in halves)
-    const bool inplace = g->out_idx != nullptr;
-    w.sacc_cap = inplace ? f * n + kPad : 0;
+    const bool inplace = batch_inplace(g, W);
+    w.sacc_cap = inplace ? (g->bsacc_cap ? g->bsacc_cap : W * n / 16) + kPad : 0;
     if ((e = alloc(&w.sig, (size_t)n * W)) || (!inplace && (e = alloc(&w.du, (size_t)n * W))) ||
         (inplace && (e = alloc(&w.sacc, 2 * (size_t)w.sacc_cap))) || (inplace && (e = alloc(&w.scnt, n + 2))) ||
         (e = alloc(&w.vis, n * nw)) ||
@@ -1321,11 +1322,13 @@ static tbc_status batch_alloc(tbc_graph *g, int q, int W) {
     }
     if (!g->bgrid) {
         int per_sm = 0, sms = 0;
-        for (const void *fn : {(const void *)k_bcb<32, false>, (const void *)k_bcb<64, false>,
-                               (const void *)k_bcb<32, true>, (const void *)k_bcb<64, true>})
+        for (const void *fn : {(const void *)k_bcb<32, false, false>, (const void *)k_bcb<64, false, false>,
+                               (const void *)k_bcb<32, true, false>, (const void *)k_bcb<64, true, false>,
+                               (const void *)k_bcb<32, false, true>, (const void *)k_bcb<64, false, true>,
+                               (const void *)k_bcb<32, true, true>, (const void *)k_bcb<64, true, true>})
             if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBSmem)))
                 return cuda_error(e, "batch smem attribute");
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, (const void *)k_bcb<64, true>, kBB, kBSmem)) ||
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, (const void *)k_bcb<64, true, true>, kBB, kBSmem)) ||
             (e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, g->device)))
             return cuda_error(e, "batch occupancy query");
         if (per_sm < 1) return set_error(TBC_ERR_CUDA, "k_bcb cannot be resident (occupancy 0)");
@@ -1362,7 +1365,7 @@ void batch_free_one(tbc_graph *g, int q) {
     w = BatchWorkspace{};
     // the partition's overflow total restarts with its counters (after cudaFree: a copy still in
     // flight from the last launch has landed by now)
-    if (g->h_bovf) g->h_bovf[q] = 0;
+    if (g->h_bovf) g->h_bovf[q] = g->h_bovf[kMaxPartitions + q] = 0;
     g->bovf_seen[q] = 0;
 }
 
@@ -1379,12 +1382,13 @@ void batch_free(tbc_graph *g) {
 // GTEPS), else 32 (the 16 M-vertex lattice: 2.03 vs 1.91, at half the workspace).  The choice is
 // made once per graph (a later change in free memory cannot flip it and reallocate), and falls
 // back to 32 if the W = 64 workspace then fails to allocate (batch_run).
-static int64_t batch_ws_bytes(const tbc_graph *g, int W) {  // batch_alloc's sizes, one partition
+static int64_t batch_ws_bytes(const tbc_graph *g, int W, bool inplace) {  // batch_alloc's sizes, one partition
     const int64_t n = g->n, m = g->m, nw = W / 32;
     const int64_t f = g->blist_factor < W ? g->blist_factor : W;
     const int64_t list_cap = f * n + kPad;
     const int64_t tiles_cap = (list_cap + f * m) / kBT + n + 2 + kPad;
-    const int64_t rows = g->out_idx ? 8 * W * n + 16 * list_cap + 8 * n : 16 * W * n;  // in place: + sacc, scnt
+    const int64_t sacc = 2 * 8 * (g->bsacc_cap ? g->bsacc_cap : W * n / 16);
+    const int64_t rows = inplace ? 8 * W * n + sacc + 8 * n : 16 * W * n;  // in place: + sacc, scnt
     return rows + 12 * n * nw + list_cap * (12 + 4 * nw) + 4 * tiles_cap + 16 * (n + kPad) +
            4 * ((n + m) / kBT + 2 + kPad) + 32 * (n + 2) + (int64_t)sizeof(Ctrs);
 }
@@ -1399,7 +1403,7 @@ int batch_width(const tbc_graph *g) {
     if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) return 32;
     double have = 0.85 * (double)fr;
     for (int q = 0; q < kMaxPartitions; ++q) have += g->bws[q].ready ? (double)g->bws[q].bytes : 0.0;
-    return (double)batch_ws_bytes(g, 64) <= have ? 64 : 32;
+    return (double)batch_ws_bytes(g, 64, g->binplace == 1) <= have ? 64 : 32;
 }
 
 // source grouping key of each source (one warp per source): its 2-hop out-volume V = sum of the
@@ -1483,7 +1487,7 @@ static int batch_auto_parts(tbc_graph *g, int W) {
     const int64_t n = g->n, m = g->m;
     if ((n * 32ll * 16 > (1ll << 30) && m >= 8 * n) || m >= 64 * n) return 1;
     const int cap = m >= 8 * n ? 4 : kMaxPartitions;  // RMAT 18: 4 beats 8; lattices: 8
-    const double per = (double)batch_ws_bytes(g, W);
+    const double per = (double)batch_ws_bytes(g, W, g->out_idx && (g->binplace == 1 || g->binplace_eff == 1));
     size_t fr = 0, tot = 0;
     if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) return 1;
     double have = 0.8 * (double)fr;
@@ -1505,6 +1509,18 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
             for (int q = 0; q < kMaxPartitions; ++q) batch_free_one(g, q);  // reallocated below
         }
         for (int q = 0; q < kMaxPartitions; ++q) g->bovf_seen[q] = g->h_bovf ? g->h_bovf[q] : 0;
+        // a level of an earlier call needed more split-accumulator values than allocated: resize
+        // (to the largest need x 5/4, never shrinking) the partitions that were short
+        int64_t need = 0;
+        for (int q = 0; q < kMaxPartitions; ++q)
+            if (g->h_bovf && g->bws[q].ready && g->bws[q].sacc &&
+                (int64_t)g->h_bovf[kMaxPartitions + q] > g->bws[q].sacc_cap - kPad)
+                need = std::max(need, (int64_t)g->h_bovf[kMaxPartitions + q]);
+        if (need > 0) {
+            g->bsacc_cap = std::max(g->bsacc_cap, need + need / 4 + 1024);
+            for (int q = 0; q < kMaxPartitions; ++q)
+                if (g->bws[q].ready && g->bws[q].sacc && g->bws[q].sacc_cap - kPad < g->bsacc_cap) batch_free_one(g, q);
+        }
     }
     // tbc_bfs_batch exports per list index: batches are cut from the list as given
     const bool grouped = g->batch_order && k > 1 && k < (1ll << 31) && !bfs_depth;
@@ -1597,17 +1613,22 @@ tbc_status batch_run(tbc_graph *g, const int32_t *d_sources, int64_t k, double *
     g->last_width = W;
     g->last_parts = np;
     void *args[] = {&S};
-    const void *fn = np > 1 ? (W == 64 ? (const void *)k_bcb<64, true> : (const void *)k_bcb<32, true>)
-                            : (W == 64 ? (const void *)k_bcb<64, false> : (const void *)k_bcb<32, false>);
+    const bool ip = S.p[0].inplace != 0;
+    const void *fn = ip ? (np > 1 ? (W == 64 ? (const void *)k_bcb<64, true, true> : (const void *)k_bcb<32, true, true>)
+                                  : (W == 64 ? (const void *)k_bcb<64, false, true> : (const void *)k_bcb<32, false, true>))
+                        : (np > 1 ? (W == 64 ? (const void *)k_bcb<64, true, false> : (const void *)k_bcb<32, true, false>)
+                                  : (W == 64 ? (const void *)k_bcb<64, false, false> : (const void *)k_bcb<32, false, false>));
     cudaError_t e = cudaLaunchCooperativeKernel(fn, dim3(S.cta_per_part * np), dim3(kBB), args, kBSmem, stream);
     if (e != cudaSuccess) return cuda_error(e, "cudaLaunchCooperativeKernel(k_bcb)");
-    if (!g->h_bovf && (e = cudaMallocHost(&g->h_bovf, sizeof(unsigned long long) * kMaxPartitions)) == cudaSuccess)
-        for (int q = 0; q < kMaxPartitions; ++q) g->h_bovf[q] = 0;
+    if (!g->h_bovf && (e = cudaMallocHost(&g->h_bovf, sizeof(unsigned long long) * 2 * kMaxPartitions)) == cudaSuccess)
+        for (int q = 0; q < 2 * kMaxPartitions; ++q) g->h_bovf[q] = 0;
     (void)cudaGetLastError();
     if (g->h_bovf)  // overflow totals, read by the next call (no synchronisation here)
         for (int q = 0; q < np; ++q)
             if ((e = cudaMemcpyAsync(&g->h_bovf[q], &g->bws[q].ctr->ovf_total, sizeof(unsigned long long),
-                                     cudaMemcpyDeviceToHost, stream)))
+                                     cudaMemcpyDeviceToHost, stream)) ||
+                (e = cudaMemcpyAsync(&g->h_bovf[kMaxPartitions + q], &g->bws[q].ctr->split_need,
+                                     sizeof(unsigned long long), cudaMemcpyDeviceToHost, stream)))
                 return cuda_error(e, "overflow counter copy");
     return TBC_OK;
 }

@@ -33,6 +33,7 @@ struct Ctrs {
     unsigned int ovf;             // batched engine: a level list outgrew the workspace (re-run in halves)
     unsigned long long ovf_total; // batched engine: such re-runs since the workspace was allocated
     unsigned long long salloc[2]; // batched engine (in place): split-accumulator allocation, by level parity
+    unsigned long long split_need;// batched engine (in place): most split lanes of one level seen (sizes sacc)
     unsigned long long trace_n;   // entries written to the trace buffer
     // accumulated statistics (tbc_stats)
     long long st_sources, st_reached, st_reached_edges, st_fwd_edges, st_bwd_edges, st_levels, st_pull_levels,
@@ -230,7 +231,12 @@ struct tbc_graph {
     int auto_width = 0;           // batch width the auto rule settled on for this graph (0: not yet)
     int last_width = 0, last_parts = 0;  // of the latest batched call (tbc_stats)
     int64_t blist_factor = 2;     // batched engine: level-list entries per vertex allocated (grows x2)
-    unsigned long long *h_bovf = nullptr;  // pinned: per-partition overflow totals after the latest call
+    unsigned long long *h_bovf = nullptr;  // pinned [2][kMaxPartitions]: per-partition list-overflow totals
+                                           // and split-accumulator needs (largest level) after the latest call
+    int binplace = -1;            // TBC_OPT_BATCH_INPLACE (-1 auto, 0 off, 1 on)
+    int binplace_eff = -1;        // auto: settled at the first allocation (0 / 1)
+    int64_t bsacc_cap = 0;        // batched engine (in place): split-accumulator values per level parity
+                                  // (0 = initial W n / 16; grows to the largest level seen x 5/4)
     unsigned long long bovf_seen[tbc::kMaxPartitions] = {};
     tbc::Ctrs retired = {};       // statistics of freed batched workspaces (kept for tbc_stats)
     int32_t *bfs_depth = nullptr; // tbc_bfs_batch device outputs (grow-only)

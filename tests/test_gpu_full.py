@@ -56,7 +56,7 @@ def test_kronecker_generator_identical_on_host_and_device(directed):
 
 # ------------------------------------------------------------------ full source lists vs cached oracle
 
-def _check_full_list(cfg, name=None, k=None):
+def _check_full_list(cfg, name=None, k=None, setup=None):
     meta, z = _fixture(name or f"oracle_cfg{cfg}")
     g, src = gg.make_config(cfg, device="cpu" if gg.CONFIGS[cfg]["kind"] != "kron" else "cuda")
     src = src[: meta["k"]]
@@ -65,6 +65,8 @@ def _check_full_list(cfg, name=None, k=None):
     assert _sha(g.row_idx.astype(np.int32)) == meta["row_idx_sha"]
     assert _sha(np.ascontiguousarray(src, dtype=np.int32)) == meta["src_sha"]
     with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:  # bench launch configuration
+        if setup:
+            setup(G)
         got = G.bc(src)
         st = G.stats()
     assert st["sources"] == meta["k"] and st["bad_sources"] == 0
@@ -287,6 +289,55 @@ def test_batched_list_overflow_reruns_halves(width):
             G.reset_stats()
             assert_bc(G.bc(src), want)
         assert G.stats()["list_overflows"] == 0
+
+
+# ------------------------------------------------------------------ in-place backward (TBC_OPT_BATCH_INPLACE)
+
+INPLACE_CASES = [gg.star(9), gg.path(9, directed=True), gg.cycle(11), gg.complete(7), gg.grid(9, 8),
+                 gg.mycielski(7), gg.random_tree(300, 3)]
+
+
+@pytest.mark.parametrize("width", [32, 64])
+@pytest.mark.parametrize("g", INPLACE_CASES, ids=lambda g: g.name)
+def test_inplace_backward_small(g, width):
+    """sigma rows overwritten by delta_u, split owners through the split accumulator: the oracle's bc
+    on closed-form graphs, over two calls (the first may re-run sweeps whose accumulator is short,
+    the second runs with the accumulator sized from the first)."""
+    src = np.concatenate([np.arange(g.n), np.arange(min(g.n, 40))]).astype(np.int32)  # repeats (R18)
+    want = oracle.bc(g.col_ptr, g.row_idx, g.directed, src)
+    with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+        G.set_batch(tbc.ENGINE_BATCHED)
+        G.set_batch_width(width)
+        G.set_batch_inplace(1)
+        for _ in range(2):
+            assert_bc(G.bc(src), want)
+
+
+@pytest.mark.parametrize("directed", [False, True])
+@pytest.mark.parametrize("parts", [1, 3])
+def test_inplace_backward_kronecker(directed, parts):
+    """Kronecker 14 (hubs: owners spanning hundreds of tiles, most tiles holding a split owner), W = 64,
+    1 or 3 SM partitions; and the workspace is smaller than with separate delta_u rows."""
+    g = gg.kronecker(14, 16, seed=21, directed=directed, device="cuda")
+    src = gg.sources(g, 200, seed=5)
+    want = oracle.bc(g.col_ptr, g.row_idx, directed, src)
+    ws = {}
+    for mode in (1, 0):
+        with tbc.Graph.from_csc(g.col_ptr, g.row_idx, g.directed) as G:
+            G.set_batch(tbc.ENGINE_BATCHED)
+            G.set_batch_width(64)
+            G.set_batch_parts(parts)
+            G.set_batch_inplace(mode)
+            for _ in range(2):
+                G.reset_stats()
+                assert_bc(G.bc(src), want)
+            ws[mode] = G.stats()["workspace_bytes"]
+    assert ws[1] < ws[0]
+
+
+def test_inplace_cfg3_full_source_list_cached_oracle():
+    """The bench workload (Kronecker 22 directed, all 4096 sources) with the in-place backward."""
+    _check_full_list(3, setup=lambda G: G.set_batch_inplace(1))
 
 
 # ------------------------------------------------------------------ strict single format (NEXT-4)

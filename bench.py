@@ -30,7 +30,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = "BC GTEPS and sec/source at 1/2/4/8 B200; HBM GB/s fraction of peak"
 # the configs' source lists (BASELINE.json configs); strong scaling splits them over the ranks
-SOURCES_TOTAL = {1: 1024, 2: 1024, 3: 4096, 4: 1024, 5: 8192, 6: None, 7: 1024}
+SOURCES_TOTAL = {1: 1024, 2: 1024, 3: 4096, 4: 1024, 5: 8192, 6: None, 7: 1024, 8: 1024}
 # the paper's printed figure for the SAME workload (context: Titan Xp), GTEPS
 PAPER_GTEPS = {6: (10.257, "Table 5 P:452: exact BC of mycielski16, 159.8 s, 10,257 MTEPs on a Titan Xp"),
                7: (18.470, "Table 3 P:380: one source of mycielski19, 48.9 ms, 18,470 MTEPs on a Titan Xp")}

@@ -12,6 +12,8 @@ timeout 300 python bench.py --config 1 --steps 50 --warmup 5 > gpurun_out/f2_cfg
 timeout 300 python bench.py --config 2 --steps 10 --warmup 3 > gpurun_out/f2_cfg2.json 2>&1
 timeout 900 python bench.py --config 4 --steps 3 --warmup 3 > gpurun_out/f2_cfg4.json 2>&1
 timeout 900 python bench.py --config 5 --steps 3 --warmup 3 > gpurun_out/f2_cfg5.json 2>&1
+timeout 900 python bench.py --config 5 --steps 3 --warmup 3 --inplace 1 --no-cpu-baseline > gpurun_out/f2_cfg5_inplace.json 2>&1
+timeout 900 python bench.py --config 5 --steps 3 --warmup 3 --inplace 1 --width 32 --no-cpu-baseline > gpurun_out/f2_cfg5_inplace_w32.json 2>&1
 timeout 600 python bench.py --config 6 --steps 3 --warmup 3 --order 0 --no-cpu-baseline > gpurun_out/f2_cfg6.json 2>&1
 timeout 600 python bench.py --config 7 --steps 3 --warmup 3 --no-cpu-baseline > gpurun_out/f2_cfg7.json 2>&1
 timeout 900 python bench.py --config 8 --steps 2 --warmup 3 > gpurun_out/f2_cfg8.json 2>&1
@@ -23,3 +25,5 @@ PROF_TAG=f2c3 bash tools/gpu_prof_bcb.sh; tail -1 gpurun_out/prof_f2c3.log
 python tools/ncu_inst.py gpurun_out/prof_f2c3_source.csv 40 > gpurun_out/prof_f2c3_inst.txt 2>&1
 python tools/ncu_stalls.py gpurun_out/prof_f2c3_source.csv > gpurun_out/prof_f2c3_stalls.txt 2>&1
 rm -f gpurun_out/prof_f2c3.ncu-rep gpurun_out/prof_f2c3_source.csv
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/f2_smoke.log 2>&1; echo "smoke rc=$?"; tail -1 gpurun_out/f2_smoke.log
+timeout 1800 python -m pytest tests -m gpu -q > gpurun_out/f2_gputests.log 2>&1; echo "gpu tests rc=$? $(tail -1 gpurun_out/f2_gputests.log)"

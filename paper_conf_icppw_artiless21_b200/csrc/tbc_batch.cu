@@ -58,9 +58,6 @@ constexpr int kPad = 8;
 #ifndef TBC_DYN_CHUNK
 #define TBC_DYN_CHUNK 1    // tiles taken per atomic in the dynamic share
 #endif
-#ifndef TBC_OTILE_PF
-#define TBC_OTILE_PF 0
-#endif
 #ifndef TBC_DYN_BIG
 #define TBC_DYN_BIG 4      // chunk multiplier on passes of > 4 M tiles
 #endif
@@ -335,10 +332,6 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
     // largest passes have ~1 M tiles, is best at 1; Kronecker 25, ~16 M, at 4: 402 -> 426 GTEPS)
     const int chunk = ntiles > (4ll << 20) ? TBC_DYN_BIG * TBC_DYN_CHUNK : TBC_DYN_CHUNK;
     int64_t dend = -1;  // end of the warp's current dynamic chunk
-#if TBC_OTILE_PF
-    int64_t pf_tile = -1;
-    int32_t pf_ps = 0, pf_pe = 0;
-#endif
     for (int64_t tile = gwarp;;) {
         if (tile >= nstat && tile >= dend) {
             unsigned long long t = 0;
@@ -350,19 +343,8 @@ __device__ __forceinline__ void bpass(const BParams &P, BWarpSmem &ws, const int
         BPROF_START();
         const int64_t ks = tile * kBT;
         const int64_t ke = min(ks + (int64_t)kBT, K);
-#if TBC_OTILE_PF
-        // the next static tile's owner range is loaded one tile ahead (its round trip overlaps this tile)
-        const int64_t ps = tile == pf_tile ? (int64_t)pf_ps : (int64_t)otiles[tile];
-        const int64_t pe = tile == pf_tile ? (int64_t)pf_pe : ((tile + 1 < ntiles) ? (int64_t)otiles[tile + 1] : N);
-        if (tile < nstat && tile + nwarps < nstat) {
-            pf_tile = tile + nwarps;
-            pf_ps = otiles[pf_tile];
-            pf_pe = pf_tile + 1 < ntiles ? otiles[pf_tile + 1] : (int32_t)N;
-        }
-#else
         const int64_t ps = otiles[tile];
         const int64_t pe = (tile + 1 < ntiles) ? (int64_t)otiles[tile + 1] : N;
-#endif
         const int64_t es = ks - ps, ee = ke - pe;
         const int nwin = (int)(min(pe, N - 1) - ps + 1);
         const int ne = (int)(ee - es);

@@ -53,7 +53,9 @@ constexpr int kPad = 8;
 #define TBC_BUNROLL64 8
 #endif
 #ifndef TBC_STATIC_PCT
-#define TBC_STATIC_PCT 60  // share of a pass's tiles dealt statically (the rest: dynamic)
+#define TBC_STATIC_PCT 80  // share of a pass's tiles dealt statically (the rest: dynamic); A/B on B200
+                           // (round 2): 80 vs 60 -- Kronecker 22 379 vs 369 GTEPS, RMAT 18 404 vs 401,
+                           // Kronecker 25 475 vs 476, mycielski19 1095 vs 1100; 90 loses on RMAT / mycielski
 #endif
 #ifndef TBC_DYN_CHUNK
 #define TBC_DYN_CHUNK 1    // tiles taken per atomic in the dynamic share
